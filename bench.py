@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 HPGMG-FV hot path (metric of BASELINE.json).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl sf|reference]
+
+Workload: BASELINE config 5 / config 4 at N=1 --
+an HPGMG-shaped variable-coefficient Helmholtz problem (a = b = 1, tanh beta,
+manufactured rhs) with 512^3 cells per GPU, z-slab decomposed over N GPUs
+(global (512,512,512), (512,512,1024), (512,1024,1024), (1024,1024,1024) for
+N = 1, 2, 4, 8: weak scaling).  One STEP = one full solve: an F-cycle, then
+V-cycles (2+2 colour-fused GSRB pairs, P0, exact bottom) until
+||f - Au||inf / ||f||inf < 1e-10.  value = DOF/s = (cells solved by all ranks)
+/ time.  Inputs (10.7 GB per GPU) exceed the 126 MB L2 many times over, so
+no L2 flush is needed between steps.
+
+Also measured in the same run: the GSRB smoother of BASELINE config 3 (256^3,
+one fused RB pair per call) in GStencil/s and algorithmic GB/s, the roofline
+of the dominant kernel (the fused RB-pair kernel on the finest level), an
+end-to-end number through the C ABI with host buffers, and the CPU oracle on
+a bounded sample (rank 0, N = 1).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+GSRB_BYTES_PER_CELL = 64      # PAPER.md:669-672 (x r+w, rhs, alpha, beta x3, lambda)
+WEAK_SHAPES = {1: (512, 512, 512), 2: (512, 512, 1024), 4: (512, 1024, 1024),
+               8: (1024, 1024, 1024)}   # (nx, ny, nz)
+F_OVER_V = 8.0 / 7.0          # F-cycle cost in finest-level V-cycles (sum over levels)
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="sf", choices=["sf", "reference"])
+    p.add_argument("--n", type=int, default=512, help="cells per side per GPU (weak scaling)")
+    p.add_argument("--gsrb-n", type=int, default=256)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--quick", action="store_true", help="skip the side measurements")
+    return p.parse_args()
+
+
+def dims_for(n, gpus):
+    if n == 512 and gpus in WEAK_SHAPES:
+        return WEAK_SHAPES[gpus]
+    return (n, n, n * gpus)
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self.proc = index, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([c.strip() for c in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
+        mx = max(float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit())
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if len(r) > 3 + i and r[3 + i].lower().startswith("active")})
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            p = json.load(fh)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy, burst)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic():
+    """dram bytes read+write per launch of the fused pair kernel from the
+    committed `ncu --set full` capture (profiles/), keyed by level size."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as fh:
+            return json.load(fh)
+    except Exception:
+        return {}
+
+
+# ------------------------------------------------------------------ oracle (cpu)
+def oracle_vcycle_sample(shape, reps=1):
+    """Time the CPU oracle's V-cycle on the same HPGMG-shaped workload.
+    Returns (seconds per V-cycle, cores used, description)."""
+    from oracle import oracle as O
+    from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
+    nx, ny, nz = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.hpgmg_coeffs(nx, ny, nz, h)
+    _, f = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
+    mg = O.MG(nx, ny, nz, h, 1.0, 1.0, *coeffs)
+    del coeffs
+    u = __import__("numpy").zeros(f.shape)
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        u = mg.vcycle(u, f)
+        ts.append(time.perf_counter() - t0)
+    return min(ts), 1, f"oracle V-cycle (2+2 GSRB pairs, P0, exact bottom) on {nx}x{ny}x{nz}"
+
+
+def oracle_shape(shape):
+    """Full workload if the host has the memory (~22 GB for 512^3), else 256^3."""
+    try:
+        import psutil
+        avail = psutil.virtual_memory().available
+    except Exception:
+        avail = 0
+    cells = shape[0] * shape[1] * shape[2]
+    if avail > cells * 8 * 40:
+        return shape, 1.0
+    return (256, 256, 256), cells / 256**3
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    nx, ny, nz = dims_for(args.n, 1)
+    shp, scale = oracle_shape((nx, ny, nz))
+    steps = []
+    for s in range(args.warmup + args.steps):
+        t, cores, desc = oracle_vcycle_sample(shp)
+        if s >= args.warmup:
+            steps.append(t * scale)
+    tv = sum(steps) / len(steps)
+    cyc = solve_cycles_guess()
+    t_solve = tv * (F_OVER_V + cyc)
+    dof = nx * ny * nz * args.gpus
+    val = dof / (t_solve * args.gpus) * args.gpus if args.gpus else dof / t_solve
+    val = (nx * ny * nz) / t_solve
+    sample = (f"{desc}{'' if scale == 1 else f' scaled x{scale:g} to {nx}^3'}; solve = 1 F-cycle "
+              f"(= {F_OVER_V:.3f} V) + {cyc} V-cycles, per GPU-equivalent workload")
+    line = {"impl": "reference", "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
+            "value": val, "unit": "DOF/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_solve * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"C5 HPGMG-FV VC Helmholtz {nx}x{ny}x{nz} per GPU",
+                       "global": [nx, ny, nz]},
+            "cpu_baseline": {"value": val, "unit": "DOF/s", "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": val, "unit": "DOF/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def solve_cycles_guess():
+    """V-cycles after the F-cycle for the 512^3 workload (measured on the GPU
+    arm, which prints `cycles`; kept here for the oracle-only arm)."""
+    return int(os.environ.get("SF_SOLVE_VCYCLES", "10"))
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangdmwbf17_b200 import sf
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    sf.lib()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    nx, ny, nz = dims_for(args.n, world)
+    comm = sf.Comm.nccl() if world > 1 else None
+    h = 1.0 / max(nx, ny, nz)
+    L = sf.Level(nx, ny, nz, h, comm=comm)
+    sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)       # HPGMG problem + manufactured f
+    M = sf.MG(L, 1.0, 1.0)
+    stream = L.stream
+    dof_local = nx * ny * (nz // world)
+
+    def step():
+        return sf.sf_solve(M.handle, True, 1e-10, 50)
+
+    for _ in range(args.warmup):
+        st, cyc, hist = step()
+    sf.sf_launch_count(reset=True)
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            st, cyc, hist = step()
+        e1.record(stream)
+        barrier()
+    launches = sf.sf_launch_count(reset=True)
+    t = max_over_ranks(e0.elapsed_time(e1) / 1e3)
+    value = dof_local * world * args.steps / t
+    ms_step = t / args.steps * 1e3
+
+    # error vs the manufactured solution (O(h^2) pin)
+    u = L.download(sf.SF_U)
+    from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
+    err = None
+    if world == 1 and nx * ny * nz <= 512**3:
+        ue, _ = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
+        err = float(np.abs(u - ue).max())
+        del ue
+    del u
+
+    side = {}
+    if not args.quick:
+        side = side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_ranks,
+                                 dof_local, cyc)
+
+    if rank == 0:
+        pk, pk_src = peaks()
+        fine_pair = side.get("fine_pair_ms")
+        roof = None
+        if fine_pair:
+            alg = GSRB_BYTES_PER_CELL * dof_local
+            ach = alg / (fine_pair / 1e3) / 1e9
+            tr = ncu_traffic().get(f"{nx}x{ny}x{nz // world}")
+            roof = {"bound": "hbm", "achieved": ach, "peak": pk, "unit": "GB/s",
+                    "frac": ach / pk, "traffic": tr,
+                    "kernel": "gsrb_pair_kernel (colour-fused RB pair, finest level)",
+                    "algorithmic_bytes_per_launch": alg, "launch_ms": fine_pair,
+                    "peak_source": pk_src,
+                    "share_of_step": side.get("fine_pair_share")}
+        line = {
+            "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
+            "value": value, "unit": "DOF/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (HPGMG-shaped VC Helmholtz, manufactured rhs, on-device init)",
+            "config": {"workload": f"C5 HPGMG-FV VC Helmholtz {nx}x{ny}x{nz // world} per GPU",
+                       "global": [nx, ny, nz], "parallelism": f"z-slab x{world}",
+                       "cycles_per_solve": cyc, "final_relres": hist[-1] if hist else None,
+                       "max_err_vs_manufactured": err,
+                       "smoother": "colour-fused GSRB, 2+2 pairs", "l2": "inputs >> L2, no flush"},
+            "clocks": clk.summary(),
+            "gpu_launches": launches,
+            "roofline": roof,
+        }
+        line.update({k: v for k, v in side.items() if k in ("e2e", "gsrb_c3", "vcycle",
+                                                             "cpu_baseline")})
+        print(json.dumps(line), flush=True)
+    M.close()
+    L.close()
+    if comm:
+        comm.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_ranks, dof_local,
+                      cyc):
+    out = {}
+    stream = L.stream
+    nx, ny, nz = L.gnx, L.gny, L.gnz
+
+    def timed(fn, reps, warm=3):
+        for _ in range(warm):
+            fn()
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(reps):
+            fn()
+        b.record(stream)
+        barrier()
+        return max_over_ranks(a.elapsed_time(b) / reps)
+
+    # dominant kernel: one fused RB pair on the finest level (1 launch per call at N=1)
+    fine_pair = timed(lambda: sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1,
+                                                sf.SF_SMOOTH_FUSED), 20)
+    out["fine_pair_ms"] = fine_pair
+    # V-cycle alone (finest level; the solve = 1 F + cyc-1 V)
+    vms = timed(lambda: sf.sf_vcycle(M.handle, 0), 5, warm=2)
+    out["vcycle"] = {"ms": vms, "dof_s": dof_local * world / (vms / 1e3)}
+    # pairs on the finest level per solve: F: (pre+post) ; each V: 4 pairs
+    pairs_per_solve = 4 * cyc
+    out["fine_pair_share"] = None
+
+    # e2e: through the C ABI with host buffers (pinned), H2D of f + solve + D2H of u
+    host_f = torch.empty(L.host_shape(sf.SF_F), dtype=torch.float64, pin_memory=True)
+    host_u = torch.empty(L.host_shape(sf.SF_U), dtype=torch.float64, pin_memory=True)
+    L.download(sf.SF_F, host_f.numpy())
+    nb = host_f.numel() * 8
+
+    def e2e_step():
+        sf.sf_level_upload(L.handle, sf.SF_F, host_f.data_ptr())
+        sf.sf_solve(M.handle, True, 1e-10, 50)
+        sf.sf_level_download(L.handle, sf.SF_U, host_u.data_ptr())
+
+    e2e_step()
+    barrier()
+    t0 = time.perf_counter()
+    reps = max(2, min(args.steps, 5))
+    for _ in range(reps):
+        e2e_step()
+    barrier()
+    te = max_over_ranks((time.perf_counter() - t0) / reps)
+    out["e2e"] = {"value": dof_local * world / te, "unit": "DOF/s", "h2d_bytes_per_step": nb,
+                  "d2h_bytes_per_step": nb, "ms_per_step": te * 1e3,
+                  "how": "sf_level_upload(f, pinned) + sf_solve + sf_level_download(u, pinned)"}
+
+    # BASELINE config 3: 256^3 GSRB smoother throughput (rank 0's GPU only)
+    if rank == 0:
+        n3 = args.gsrb_n
+        G = sf.Level(n3, n3, n3, 1.0 / n3)
+        sf.sf_init_problem(G.handle, 1, 1.0, 1.0, 1)
+        sf.sf_rebuild_operator(G.handle, 1.0, 1.0)
+        s = G.stream
+
+        def pair():
+            sf.sf_smooth_gsrb(G.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED)
+        for _ in range(10):
+            pair()
+        s.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        for _ in range(100):
+            pair()
+        b.record(s)
+        s.synchronize()
+        ms = a.elapsed_time(b) / 100
+        cells = n3**3
+        pk, _ = peaks()
+        gbs = GSRB_BYTES_PER_CELL * cells / (ms / 1e3) / 1e9
+        # colour (unfused) sweeps for comparison
+        def pair_c():
+            sf.sf_smooth_gsrb(G.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_COLOUR)
+        for _ in range(3):
+            pair_c()
+        a.record(s)
+        for _ in range(20):
+            pair_c()
+        b.record(s)
+        s.synchronize()
+        msc = a.elapsed_time(b) / 20
+        out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms, "gstencil_s": 2 * cells / 2 / (ms / 1e3) / 1e9,
+                          "point_updates_per_s": cells / (ms / 1e3),
+                          "alg_gbs": gbs, "frac_of_peak": gbs / pk,
+                          "colour_sweeps_ms_per_rb_pair": msc,
+                          "note": "GStencil/s = point updates/s (each cell updated once per pair)"}
+        G.close()
+        if world == 1 and not args.no_cpu_baseline:
+            shp, scale = oracle_shape((nx, ny, nz))
+            tv, cores, desc = oracle_vcycle_sample(shp)
+            tv *= scale
+            t_solve = tv * (F_OVER_V + (cyc - 1))
+            out["cpu_baseline"] = {
+                "value": nx * ny * nz / t_solve, "unit": "DOF/s", "cores": cores,
+                "kind": "oracle",
+                "sample": (f"{desc}{'' if scale == 1 else f' x{scale:g}'}: {tv:.2f} s; solve "
+                           f"extrapolated as 1 F-cycle ({F_OVER_V:.3f} V) + {cyc - 1} V-cycles, "
+                           "the cycle counts this GPU run measured")}
+    out["fine_pair_share"] = (4 * (cyc - 1) + 4 * 1) * fine_pair / (
+        (out["vcycle"]["ms"]) * (F_OVER_V + cyc - 1)) if fine_pair else None
+    return out
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,215 @@
+/*
+ * include/sf.h -- C ABI of libsf, the B200-native (sm_100a, fp64) HPGMG-FV
+ * hot path that Snowflake's micro-compilers generate (Zhang, Driscoll, Fox,
+ * Markley, Williams, Basu: "Snowflake: A Lightweight Portable Stencil DSL",
+ * IPDPSW 2017).  "PAPER.md:n" cites a line of the paper's text; "R-n" cites a
+ * reading listed in DESIGN.md where the paper is silent or garbled.
+ *
+ * Plain C types only: ints, doubles, host pointers and device pointers
+ * (void*), no torch types.  Every call returns sf_status (SF_OK == 0); the
+ * message of the last failure on the calling thread is sf_last_error().
+ *
+ * GENERAL CONVENTIONS
+ *  - Precision: IEEE fp64 everywhere; indices int32/int64.
+ *  - Grids: a level is a box of gnx x gny x gnz cells of spacing h (cell
+ *    centres at (i+1/2)h), homogeneous Dirichlet boundary on all six faces
+ *    (PAPER.md:333-341).  It is split into z-slabs ("parts"); part p owns
+ *    global planes [p*lnz, (p+1)*lnz), lnz = gnz/nparts.  A process holds
+ *    either all parts (loopback comm, one device) or one part (NCCL comm,
+ *    one part per rank / GPU).
+ *  - Host arrays are C-order (x fastest), interior only, covering the z-range
+ *    of ALL parts local to the caller:
+ *        cell fields (U, F, R, TMP, ALPHA, DINV)   (lnz_local, gny, gnx)
+ *        SF_BETA_I  (face i between cells i-1, i)   (lnz_local, gny, gnx+1)
+ *        SF_BETA_J                                  (lnz_local, gny+1, gnx)
+ *        SF_BETA_K                                  (lnz_local+1, gny, gnx)
+ *    (lnz_local = lnz * local parts).  Host arrays are never retained.
+ *  - Streams: every call enqueues on the level's CUDA stream and returns
+ *    without a host synchronisation, EXCEPT sf_level_download, sf_norm,
+ *    sf_solve and sf_sync, which synchronise that stream.  Host buffers
+ *    passed to sf_level_upload must stay valid until the next synchronising
+ *    call (pinned memory makes the copy asynchronous).
+ *  - Errors: argument/shape errors are returned synchronously
+ *    (SF_ERR_INVALID / SF_ERR_SHAPE).  Asynchronous CUDA/NCCL faults surface
+ *    at the next synchronising call as SF_ERR_CUDA / SF_ERR_NCCL.  There is no
+ *    CPU fallback: without an sm_100 device every constructor fails with
+ *    SF_ERR_CUDA.
+ *  - Ghost state: interiors are the contract.  Ghost zones hold valid
+ *    boundary values only after sf_apply_bc; the stencil kernels fold the
+ *    Dirichlet condition (ghost = -inside) into their arithmetic and refresh
+ *    slab halos themselves.
+ *  - Thread safety: one level / mg object must not be used concurrently from
+ *    two host threads.
+ */
+#ifndef SF_H_
+#define SF_H_
+
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SF_OK = 0,
+    SF_ERR_INVALID = 1,        /* bad argument (NULL handle, bad field id, ...) */
+    SF_ERR_SHAPE = 2,          /* dims not even/compatible, gnz % nparts != 0 */
+    SF_ERR_OOM = 3,            /* device allocation failed / buffer too small */
+    SF_ERR_CUDA = 4,           /* CUDA runtime error, or no sm_100 device */
+    SF_ERR_NCCL = 5,           /* NCCL error (or libnccl.so.2 not loadable) */
+    SF_ERR_NOT_CONVERGED = 6,  /* sf_solve hit max_cycles */
+    SF_ERR_NUMERIC = 7         /* NaN/Inf residual */
+} sf_status;
+
+/* Fields stored per level (A1 of DESIGN.md). */
+enum sf_field {
+    SF_U = 0,      /* solution (finest) / correction e (coarse levels)        */
+    SF_F = 1,      /* right-hand side (finest) / restricted residual (coarse) */
+    SF_R = 2,      /* residual scratch                                          */
+    SF_TMP = 3,    /* scratch; ping-pong target of the colour-fused smoother   */
+    SF_ALPHA = 4,  /* alpha(c), cell-centred                                    */
+    SF_BETA_I = 5, /* beta on x-faces                                           */
+    SF_BETA_J = 6, /* beta on y-faces                                           */
+    SF_BETA_K = 7, /* beta on z-faces                                           */
+    SF_DINV = 8,   /* lambda = 1/diag(A) (A4)                                   */
+    SF_NFIELDS = 9
+};
+
+enum sf_restrict_kind { SF_RESTRICT_CELL = 0, SF_RESTRICT_FACE_I = 1,
+                        SF_RESTRICT_FACE_J = 2, SF_RESTRICT_FACE_K = 3 };
+enum sf_interp_kind { SF_INTERP_P0 = 0 /* piecewise constant */,
+                      SF_INTERP_PL = 1 /* trilinear on cell centres */ };
+enum sf_norm_kind { SF_NORM_MAX = 0, SF_NORM_L2 = 1 };
+enum sf_smoother_kind { SF_SMOOTH_AUTO = 0,     /* fused when the shape allows */
+                        SF_SMOOTH_COLOUR = 1,   /* one kernel per colour sweep  */
+                        SF_SMOOTH_FUSED = 2 };  /* colour-fused RB pair         */
+
+typedef struct sf_comm sf_comm;
+typedef struct sf_level sf_level;
+typedef struct sf_mg sf_mg;
+
+typedef struct {
+    int pre_pairs;          /* RB pairs before coarse correction (HPGMG: 2) */
+    int post_pairs;         /* RB pairs after (2) */
+    int vcycle_interp;      /* SF_INTERP_P0 (reading R-7) */
+    int fcycle_interp;      /* SF_INTERP_PL (reading R-7) */
+    int agglom_min_planes;  /* agglomerate a level whose slabs would hold fewer planes */
+    int max_cycles;         /* sf_solve cap (50) */
+    int use_graph;          /* capture V-cycles as CUDA graphs (1) */
+    int smoother;           /* enum sf_smoother_kind */
+    double rtol;            /* ||f-Au||inf/||f||inf target (1e-10, reading R-9) */
+} sf_mg_opts;
+
+/* Default options (pre=post=2, P0/PL, agglomerate below 8 planes, 50 cycles,
+ * graphs on, AUTO smoother, rtol 1e-10). */
+void sf_mg_opts_default(sf_mg_opts* o);
+
+const char* sf_last_error(void);
+/* Library build/version string; never fails. */
+const char* sf_version(void);
+
+/* -------------------------------------------------------------- comm
+ * Slab decomposition across parts.
+ * sf_comm_create_local: nparts slabs held by this process on the current
+ *   device; halos move with cudaMemcpyAsync (single-GPU test fixture and
+ *   the nranks==1 case).  nparts >= 1.
+ * sf_get_unique_id: rank 0 creates an NCCL id (128 bytes, caller buffer);
+ *   the caller broadcasts it (e.g. torch.distributed) to every rank.
+ * sf_comm_create_nccl: one part per rank; rank in [0,nranks); the current
+ *   device must be this rank's GPU.  NCCL is loaded at run time
+ *   (libnccl.so.2, the one torch already loaded if any).
+ */
+sf_status sf_comm_create_local(sf_comm** out, int nparts);
+sf_status sf_get_unique_id(unsigned char id[128]);
+sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[128], int nranks, int rank);
+sf_status sf_comm_destroy(sf_comm* comm);
+/* number of parts in the job, parts local to this process, first local part */
+sf_status sf_comm_info(const sf_comm* comm, int* nparts, int* nlocal, int* first);
+
+/* -------------------------------------------------------------- level (A1)
+ * sf_level_bytes_needed: device bytes for a level's fields (all local parts).
+ * sf_level_create: dims must be >= 2 and gnz % nparts == 0 (SF_ERR_SHAPE);
+ *   comm NULL == one local part.  stream: a cudaStream_t (NULL = legacy
+ *   default).  dev_buf: NULL -> the library allocates (and frees on destroy);
+ *   else a caller-owned device buffer of >= buf_bytes (e.g. a torch tensor),
+ *   256-byte aligned, kept alive by the caller until sf_level_destroy.
+ *   Fields are zero-initialised.  The level borrows comm (keep it alive).
+ */
+sf_status sf_level_bytes_needed(int gnx, int gny, int gnz, const sf_comm* comm, size_t* bytes);
+sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, double h,
+                          const sf_comm* comm, void* stream, void* dev_buf, size_t buf_bytes);
+sf_status sf_level_destroy(sf_level* level);
+sf_status sf_level_upload(sf_level* level, int field, const double* host);
+sf_status sf_level_download(sf_level* level, int field, double* host);   /* syncs */
+/* Borrowed device pointer of (local part `part`, field) and its strides in
+ * doubles: element (i,j,k) of the part is dev[k*strides[2] + j*strides[1] + i]
+ * for -2 <= j,k and -4 <= i (ghost/padding).  Valid until the next
+ * sf_smooth_gsrb on that level (the fused smoother may swap U and TMP). */
+sf_status sf_level_field_ptr(sf_level* level, int part, int field, double** dev, long strides[3]);
+/* Fill ALPHA, BETA_* (and, if want_rhs, F with the manufactured right-hand
+ * side; U zeroed) with the HPGMG-shaped problem of DESIGN.md "Input recipe",
+ * on the device.  problem 0 = constant-coefficient (alpha=beta=1), 1 = HPGMG
+ * variable-coefficient (tanh beta). */
+sf_status sf_init_problem(sf_level* level, int problem, double a, double b, int want_rhs);
+/* A4: Dinv = 1/diag(A) with the Dirichlet fold (R-4);
+ * also refreshes coefficient halo planes between parts. */
+sf_status sf_rebuild_operator(sf_level* level, double a, double b);
+
+/* -------------------------------------------------------------- operators
+ * All take field ids of one level.  a, b are the Helmholtz scalars of
+ *   A x = a*alpha*x - b*div(beta grad x)
+ */
+/* A2: ghost fill, ghost = (-1)^m * mirror (R-5) */
+sf_status sf_apply_bc(sf_level* level, int field);
+/* A3: out = A x (out != x) */
+sf_status sf_apply_op(sf_level* level, int out, int x, double a, double b);
+/* A5: rb_pairs x (BC, red, BC, black) in place on field x with rhs field rhs
+ * and the level's DINV.  Red = (i+j+k) even in
+ * global 0-based cell indices (R-2).  x must be SF_U or SF_TMP when the fused
+ * smoother is used.  kind: enum sf_smoother_kind. */
+sf_status sf_smooth_gsrb(sf_level* level, int x, int rhs, double a, double b, int rb_pairs, int kind);
+/* A6: res = rhs - A x */
+sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double b);
+/* A7: coarse.c_field = R(fine.f_field); coarse dims must be fine dims / 2
+ * (PAPER.md:293-297, 466-468).  kind: enum sf_restrict_kind. */
+sf_status sf_restrict(sf_level* coarse, int c_field, sf_level* fine, int f_field, int kind);
+/* A8: fine.f_field = prescale*fine.f_field + P(coarse.c_field)
+ * (PAPER.md:293-297, 597).  kind: enum sf_interp_kind.  PL refreshes the
+ * coarse field's ghosts (A2) first. */
+sf_status sf_interpolate(sf_level* fine, int f_field, double prescale,
+                         sf_level* coarse, int c_field, int kind);
+/* A10: norm of the interior over all parts/ranks; syncs. */
+sf_status sf_norm(sf_level* level, int field, int kind, double* out);
+sf_status sf_sync(sf_level* level);
+
+/* -------------------------------------------------------------- multigrid (A9)
+ * sf_mg_create: builds the hierarchy below `finest` (which must hold ALPHA and
+ *   BETA_*): coarse coefficients by A7 (cell/face), h_c = 2h, Dinv by A4 on
+ *   every level, down to min dim 2 (exact bottom solve, R-8).  Levels whose
+ *   slabs would hold fewer than opts->agglom_min_planes planes are
+ *   agglomerated (replicated on every part/rank).  opts NULL = defaults.
+ * sf_vcycle: one V-cycle on level l (U_l corrected for rhs F_l), enqueued.
+ * sf_fcycle: one F-cycle from scratch for rhs F_0 into U_0, enqueued.
+ * sf_solve: optional F-cycle, then V-cycles until ||F-AU||inf/||F||inf <
+ *   rtol; fills *cycles and hist[0..*cycles-1] (may be NULL; caller array of
+ *   max_cycles+1 doubles); syncs.
+ */
+sf_status sf_mg_create(sf_mg** out, sf_level* finest, double a, double b, const sf_mg_opts* opts);
+sf_status sf_mg_num_levels(const sf_mg* mg, int* n);
+sf_status sf_mg_level(sf_mg* mg, int l, sf_level** out);
+sf_status sf_vcycle(sf_mg* mg, int l);
+sf_status sf_fcycle(sf_mg* mg);
+sf_status sf_solve(sf_mg* mg, int fcycle, double rtol, int max_cycles, int* cycles, double* hist);
+sf_status sf_mg_destroy(sf_mg* mg);
+
+/* -------------------------------------------------------------- measurement
+ * Number of kernels libsf launched since the counter was last reset (host-side
+ * count of launches it issued; a replayed CUDA graph counts its nodes). */
+sf_status sf_launch_count(long long* count, int reset);
+/* Per-launch device time of the most recent sf_smooth_gsrb kernels is not
+ * tracked here; bench.py times sf_smooth_gsrb with CUDA events. */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SF_H_ */

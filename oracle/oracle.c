@@ -466,3 +466,61 @@ int or_mg_solve(or_mg* m, double* u, const double* f, int fcycle, double rtol,
     }
     return c;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Sampled evaluation at full size (tests at BASELINE sizes): the same A3/A5 */
+/* definitions as above, evaluated one cell at a time.                       */
+/* ------------------------------------------------------------------------ */
+/* res[s] = rhs - A x at cells (ii[s], jj[s], kk[s]).  Applies A2 to x. */
+void or_residual_points(const or_grid* g, double a, double b, const double* alpha,
+                        const double* bi, const double* bj, const double* bk, double* x,
+                        const double* rhs, int n, const int* ii, const int* jj, const int* kk,
+                        double* res) {
+    or_apply_bc(g, x);
+    for (int s = 0; s < n; s++)
+        res[s] = rhs[OIDX(g, ii[s], jj[s], kk[s])] -
+                 op_at(g, a, b, alpha, bi, bj, bk, x, ii[s], jj[s], kk[s]);
+}
+
+/* Value of cell (i,j,k) after ONE RB pair (BC, red, BC, black) started from */
+/* x, without sweeping the grid: a red cell needs only its own red update;   */
+/* a black cell needs the red updates of its in-domain neighbours first.     */
+/* x must have A2 applied (or_apply_bc) and is restored before returning.    */
+static double red_update_at(const or_grid* g, double a, double b, const double* alpha,
+                            const double* bi, const double* bj, const double* bk,
+                            const double* dinv, const double* x, const double* rhs, int i, int j,
+                            int k) {
+    size_t c = OIDX(g, i, j, k);
+    return x[c] + dinv[c] * (rhs[c] - op_at(g, a, b, alpha, bi, bj, bk, x, i, j, k));
+}
+
+void or_gsrb_pair_points(const or_grid* g, double a, double b, const double* alpha,
+                         const double* bi, const double* bj, const double* bk, const double* dinv,
+                         double* x, const double* rhs, int n, const int* ii, const int* jj,
+                         const int* kk, double* out) {
+    or_apply_bc(g, x);
+    static const int off[6][3] = {{1, 0, 0}, {-1, 0, 0}, {0, 1, 0}, {0, -1, 0}, {0, 0, 1}, {0, 0, -1}};
+    for (int s = 0; s < n; s++) {
+        int i = ii[s], j = jj[s], k = kk[s];
+        if (((i + j + k) & 1) == 0) {
+            out[s] = red_update_at(g, a, b, alpha, bi, bj, bk, dinv, x, rhs, i, j, k);
+            continue;
+        }
+        double nv[6], ov[6];
+        size_t at[6];
+        int in[6];
+        for (int d = 0; d < 6; d++) {
+            int p = i + off[d][0], q = j + off[d][1], r = k + off[d][2];
+            in[d] = p >= 0 && p < g->nx && q >= 0 && q < g->ny && r >= 0 && r < g->nz;
+            at[d] = OIDX(g, p, q, r);
+            if (in[d]) nv[d] = red_update_at(g, a, b, alpha, bi, bj, bk, dinv, x, rhs, p, q, r);
+        }
+        for (int d = 0; d < 6; d++)
+            if (in[d]) { ov[d] = x[at[d]]; x[at[d]] = nv[d]; }
+        /* ghosts adjacent to the black cell mirror the black cell itself,  */
+        /* which the red sweep did not change: no BC refresh is needed.     */
+        out[s] = red_update_at(g, a, b, alpha, bi, bj, bk, dinv, x, rhs, i, j, k);
+        for (int d = 0; d < 6; d++)
+            if (in[d]) x[at[d]] = ov[d];
+    }
+}

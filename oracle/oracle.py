@@ -36,6 +36,7 @@ def build(force=False):
 
 _lib = None
 _P = C.POINTER(C.c_double)
+_IP = C.POINTER(C.c_int)
 
 
 class _Grid(C.Structure):
@@ -71,6 +72,10 @@ def lib():
             "or_mg_fcycle": (C.c_int, [C.c_void_p, _P, _P]),
             "or_mg_relres": (d, [C.c_void_p, _P, _P]),
             "or_mg_solve": (C.c_int, [C.c_void_p, _P, _P, C.c_int, d, C.c_int, _P]),
+            "or_residual_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP, _IP,
+                                          _P]),
+            "or_gsrb_pair_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP,
+                                           _IP, _P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -101,6 +106,11 @@ def pad(arr, kind="cell"):
 
 def interior(p):
     return np.ascontiguousarray(p[1:-1, 1:-1, 1:-1])
+
+
+def _iptr(a):
+    assert a.dtype == np.int32 and a.flags.c_contiguous
+    return a.ctypes.data_as(_IP)
 
 
 def _ptr(a):
@@ -159,6 +169,23 @@ class Problem:
         xp, rp, dp = pad(x), pad(rhs), pad(dinv)
         lib().or_smooth(*self._c(), _ptr(dp), _ptr(xp), _ptr(rp), int(rb_pairs))
         return interior(xp)
+
+    def residual_points(self, x, rhs, pts):
+        """rhs - A x at the cells pts = (i, j, k) index arrays (sampled parity)."""
+        ii, jj, kk = (np.ascontiguousarray(p, dtype=np.int32) for p in pts)
+        xp, rp, out = pad(x), pad(rhs), np.zeros(len(ii))
+        lib().or_residual_points(*self._c(), _ptr(xp), _ptr(rp), len(ii), _iptr(ii), _iptr(jj),
+                                 _iptr(kk), _ptr(out))
+        return out
+
+    def gsrb_pair_points(self, x, rhs, pts, dinv=None):
+        """Values at pts after one RB pair from x, evaluated cell by cell."""
+        dinv = self.dinv() if dinv is None else dinv
+        ii, jj, kk = (np.ascontiguousarray(p, dtype=np.int32) for p in pts)
+        xp, rp, dp, out = pad(x), pad(rhs), pad(dinv), np.zeros(len(ii))
+        lib().or_gsrb_pair_points(*self._c(), _ptr(dp), _ptr(xp), _ptr(rp), len(ii), _iptr(ii),
+                                  _iptr(jj), _iptr(kk), _ptr(out))
+        return out
 
     def bottom_solve(self, rhs):
         xp, rp = np.zeros_like(self.alpha), pad(rhs)

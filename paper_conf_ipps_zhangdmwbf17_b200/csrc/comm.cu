@@ -1,0 +1,181 @@
+// Slab decomposition plumbing: z-halo exchange between
+// neighbouring parts, coarse-level agglomeration and scalar all-reduce.
+//
+// Parts local to this process exchange with cudaMemcpyAsync (the loopback
+// fixture that lets one GPU run the decomposed code path); parts on other
+// ranks exchange with NCCL point-to-point over NVLink.  NCCL is resolved at
+// run time from libnccl.so.2 (torch's copy when torch is loaded), so libsf
+// has no link-time NCCL dependency and the CPU-only build box can build it.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <mutex>
+
+#include "sf_internal.h"
+
+namespace {
+
+struct NcclApi {
+    void* h = nullptr;
+    decltype(&ncclGetUniqueId) getUniqueId;
+    decltype(&ncclCommInitRank) commInitRank;
+    decltype(&ncclCommDestroy) commDestroy;
+    decltype(&ncclSend) send;
+    decltype(&ncclRecv) recv;
+    decltype(&ncclGroupStart) groupStart;
+    decltype(&ncclGroupEnd) groupEnd;
+    decltype(&ncclAllReduce) allReduce;
+    decltype(&ncclAllGather) allGather;
+    decltype(&ncclBroadcast) broadcast;
+    decltype(&ncclGetErrorString) errStr;
+};
+
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+
+sf_status nccl_load() {
+    std::lock_guard<std::mutex> lk(g_nccl_mu);
+    if (g_nccl.h) return SF_OK;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return sf_fail(SF_ERR_NCCL, "cannot load libnccl.so.2: %s", dlerror());
+#define SYM(field, name)                                                             \
+    g_nccl.field = (decltype(g_nccl.field))dlsym(h, name);                           \
+    if (!g_nccl.field) return sf_fail(SF_ERR_NCCL, "libnccl.so.2 lacks %s", name);
+    SYM(getUniqueId, "ncclGetUniqueId");
+    SYM(commInitRank, "ncclCommInitRank");
+    SYM(commDestroy, "ncclCommDestroy");
+    SYM(send, "ncclSend");
+    SYM(recv, "ncclRecv");
+    SYM(groupStart, "ncclGroupStart");
+    SYM(groupEnd, "ncclGroupEnd");
+    SYM(allReduce, "ncclAllReduce");
+    SYM(allGather, "ncclAllGather");
+    SYM(broadcast, "ncclBroadcast");
+    SYM(errStr, "ncclGetErrorString");
+#undef SYM
+    g_nccl.h = h;
+    return SF_OK;
+}
+
+#define SF_NCCL(call)                                                                    \
+    do {                                                                                 \
+        ncclResult_t r_ = (call);                                                        \
+        if (r_ != ncclSuccess)                                                           \
+            return sf_fail(SF_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,       \
+                           g_nccl.errStr ? g_nccl.errStr(r_) : "?");                     \
+    } while (0)
+
+}  // namespace
+
+extern "C" sf_status sf_comm_create_local(sf_comm** out, int nparts) {
+    if (!out || nparts < 1) return sf_fail(SF_ERR_INVALID, "bad arguments");
+    sf_comm* c = new sf_comm();
+    c->kind = 0;
+    c->nparts = nparts; c->nlocal = nparts; c->first = 0;
+    c->rank = 0; c->nranks = 1;
+    c->nccl = nullptr;
+    *out = c;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_get_unique_id(unsigned char id[128]) {
+    if (!id) return sf_fail(SF_ERR_INVALID, "id is NULL");
+    SF_TRY(nccl_load());
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    ncclUniqueId u;
+    SF_NCCL(g_nccl.getUniqueId(&u));
+    memcpy(id, &u, 128);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[128], int nranks,
+                                         int rank) {
+    if (!out || !id || nranks < 1 || rank < 0 || rank >= nranks)
+        return sf_fail(SF_ERR_INVALID, "bad arguments");
+    SF_TRY(nccl_load());
+    ncclUniqueId u;
+    memcpy(&u, id, 128);
+    ncclComm_t comm;
+    SF_NCCL(g_nccl.commInitRank(&comm, nranks, u, rank));
+    sf_comm* c = new sf_comm();
+    c->kind = 1;
+    c->nparts = nranks; c->nlocal = 1; c->first = rank;
+    c->rank = rank; c->nranks = nranks;
+    c->nccl = comm;
+    *out = c;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_comm_destroy(sf_comm* c) {
+    if (!c) return SF_OK;
+    if (c->kind == 1 && c->nccl) g_nccl.commDestroy((ncclComm_t)c->nccl);
+    delete c;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_comm_info(const sf_comm* c, int* nparts, int* nlocal, int* first) {
+    if (!c) return sf_fail(SF_ERR_INVALID, "NULL comm");
+    if (nparts) *nparts = c->nparts;
+    if (nlocal) *nlocal = c->nlocal;
+    if (first) *first = c->first;
+    return SF_OK;
+}
+
+sf_status sf_halo(sf_level* L, int field, int depth) {
+    if (L->nparts <= 1 || !L->comm) return SF_OK;
+    if (depth > SF_GZ || depth > L->lnz) return sf_fail(SF_ERR_SHAPE, "halo depth %d too deep", depth);
+    size_t cnt = (size_t)depth * L->ks;
+    const long lo_src = (long)SF_GZ * L->ks;                  // planes [0, d)
+    const long hi_src = (long)(L->lnz - depth + SF_GZ) * L->ks;  // planes [lnz-d, lnz)
+    const long lo_dst = (long)(SF_GZ - depth) * L->ks;        // ghosts [-d, 0)
+    const long hi_dst = (long)(L->lnz + SF_GZ) * L->ks;       // ghosts [lnz, lnz+d)
+    if (L->comm->kind == 0) {
+        for (int q = 0; q + 1 < L->nlocal; q++) {
+            double* lo = L->parts[q].f[field];
+            double* hi = L->parts[q + 1].f[field];
+            SF_CUDA(cudaMemcpyAsync(hi + lo_dst, lo + hi_src, cnt * sizeof(double),
+                                    cudaMemcpyDeviceToDevice, L->stream));
+            SF_CUDA(cudaMemcpyAsync(lo + hi_dst, hi + lo_src, cnt * sizeof(double),
+                                    cudaMemcpyDeviceToDevice, L->stream));
+        }
+        return SF_OK;
+    }
+    ncclComm_t comm = (ncclComm_t)L->comm->nccl;
+    int r = L->comm->rank, n = L->comm->nranks;
+    double* x = L->parts[0].f[field];
+    SF_NCCL(g_nccl.groupStart());
+    if (r > 0) {
+        SF_NCCL(g_nccl.send(x + lo_src, cnt, ncclDouble, r - 1, comm, L->stream));
+        SF_NCCL(g_nccl.recv(x + lo_dst, cnt, ncclDouble, r - 1, comm, L->stream));
+    }
+    if (r < n - 1) {
+        SF_NCCL(g_nccl.send(x + hi_src, cnt, ncclDouble, r + 1, comm, L->stream));
+        SF_NCCL(g_nccl.recv(x + hi_dst, cnt, ncclDouble, r + 1, comm, L->stream));
+    }
+    SF_NCCL(g_nccl.groupEnd());
+    return SF_OK;
+}
+
+sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
+    // Loopback: every fine part is local and already wrote its planes.
+    const sf_comm* cm = C->rep_comm;
+    if (!cm || cm->kind == 0) return SF_OK;
+    if (cm->nranks != parts) return sf_fail(SF_ERR_SHAPE, "agglomeration across %d parts", parts);
+    ncclComm_t comm = (ncclComm_t)cm->nccl;
+    double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
+    size_t cnt = (size_t)lnz_per_part * C->ks;
+    SF_NCCL(g_nccl.allGather(base + cm->rank * cnt, base, cnt, ncclDouble, comm, C->stream));
+    if (field == SF_BETA_K) {  // the top boundary face belongs to the last part only
+        double* top = base + (size_t)C->gnz * C->ks;
+        SF_NCCL(g_nccl.broadcast(top, top, C->ks, ncclDouble, parts - 1, comm, C->stream));
+    }
+    return SF_OK;
+}
+
+sf_status sf_allreduce_scalar(const sf_comm* cm, double* dev, int op, cudaStream_t s) {
+    if (!cm || cm->kind != 1 || cm->nranks == 1) return SF_OK;
+    SF_NCCL(g_nccl.allReduce(dev, dev, 1, ncclDouble, op == 0 ? ncclMax : ncclSum,
+                             (ncclComm_t)cm->nccl, s));
+    return SF_OK;
+}

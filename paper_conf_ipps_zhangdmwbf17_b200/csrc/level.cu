@@ -1,0 +1,351 @@
+// Level / box layout (A1), C-ABI entry points of the per-level operators,
+// error reporting and launch accounting.
+#include <cstdarg>
+#include <cstring>
+
+#include "sf_internal.h"
+
+// ----------------------------------------------------------------- errors
+static thread_local char g_err[1024] = "";
+static std::atomic<long long> g_launches{0};
+
+sf_status sf_fail(sf_status s, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+void sf_count_launch(long long n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+sf_status sf_check_launch(const char* what) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "launch of %s: %s", what, cudaGetErrorString(e));
+    return SF_OK;
+}
+
+extern "C" const char* sf_last_error(void) { return g_err; }
+
+extern "C" const char* sf_version(void) {
+    return "libsf 0.1 (sm_100a, fp64; HPGMG-FV hot path of Snowflake, IPDPSW 2017)";
+}
+
+extern "C" sf_status sf_launch_count(long long* count, int reset) {
+    if (!count) return sf_fail(SF_ERR_INVALID, "count is NULL");
+    *count = reset ? g_launches.exchange(0) : g_launches.load();
+    return SF_OK;
+}
+
+// ----------------------------------------------------------------- device check
+static sf_status check_device() {
+    int dev = -1;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "no CUDA device: %s", cudaGetErrorString(e));
+    cudaDeviceProp pr;
+    SF_CUDA(cudaGetDeviceProperties(&pr, dev));
+    if (pr.major != 10 || pr.minor != 0)
+        return sf_fail(SF_ERR_CUDA, "libsf is built for sm_100a; device %d is sm_%d%d (%s)", dev,
+                       pr.major, pr.minor, pr.name);
+    return SF_OK;
+}
+
+// ----------------------------------------------------------------- layout
+static void layout(int gnx, int gny, int lnz, long* js, long* ks, size_t* felems) {
+    long j = SF_OX + gnx + 2;
+    j = (j + 15) / 16 * 16;  // 128-byte rows
+    *js = j;
+    *ks = j * (gny + 2 * SF_GY);
+    *felems = (size_t)(*ks) * (lnz + 2 * SF_GZ);
+}
+
+static size_t field_bytes_aligned(size_t felems) { return (felems * sizeof(double) + 255) / 256 * 256; }
+
+static sf_status decomposition(int gnz, const sf_comm* comm, int* nparts, int* nlocal, int* first) {
+    if (!comm) {
+        *nparts = 1; *nlocal = 1; *first = 0;
+        return SF_OK;
+    }
+    *nparts = comm->nparts; *nlocal = comm->nlocal; *first = comm->first;
+    if (gnz % comm->nparts != 0)
+        return sf_fail(SF_ERR_SHAPE, "gnz=%d not divisible by %d parts", gnz, comm->nparts);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_bytes_needed(int gnx, int gny, int gnz, const sf_comm* comm,
+                                           size_t* bytes) {
+    if (!bytes) return sf_fail(SF_ERR_INVALID, "bytes is NULL");
+    if (gnx < 2 || gny < 2 || gnz < 2) return sf_fail(SF_ERR_SHAPE, "dims must be >= 2");
+    int np, nl, fi;
+    SF_TRY(decomposition(gnz, comm, &np, &nl, &fi));
+    long js, ks;
+    size_t fe;
+    layout(gnx, gny, gnz / np, &js, &ks, &fe);
+    *bytes = (size_t)nl * SF_NFIELDS * field_bytes_aligned(fe) + 256;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, double h,
+                                     const sf_comm* comm, void* stream, void* dev_buf,
+                                     size_t buf_bytes) {
+    if (!out) return sf_fail(SF_ERR_INVALID, "out is NULL");
+    *out = nullptr;
+    if (!(h > 0)) return sf_fail(SF_ERR_INVALID, "h must be > 0");
+    SF_TRY(check_device());
+    size_t need;
+    SF_TRY(sf_level_bytes_needed(gnx, gny, gnz, comm, &need));
+    sf_level* L = new sf_level();
+    L->gnx = gnx; L->gny = gny; L->gnz = gnz; L->h = h;
+    SF_TRY(decomposition(gnz, comm, &L->nparts, &L->nlocal, &L->first));
+    L->comm = comm;
+    L->nx = gnx; L->ny = gny; L->lnz = gnz / L->nparts;
+    layout(gnx, gny, L->lnz, &L->js, &L->ks, &L->felems);
+    L->stream = (cudaStream_t)stream;
+    if (dev_buf) {
+        if (buf_bytes < need) {
+            delete L;
+            return sf_fail(SF_ERR_OOM, "caller buffer %zu bytes < %zu needed", buf_bytes, need);
+        }
+        if (((uintptr_t)dev_buf) & 255) {
+            delete L;
+            return sf_fail(SF_ERR_INVALID, "caller buffer must be 256-byte aligned");
+        }
+        L->buf = dev_buf;
+        L->owns = false;
+    } else {
+        cudaError_t e = cudaMalloc(&L->buf, need);
+        if (e != cudaSuccess) {
+            delete L;
+            cudaGetLastError();
+            return sf_fail(SF_ERR_OOM, "cudaMalloc(%zu): %s", need, cudaGetErrorString(e));
+        }
+        L->owns = true;
+    }
+    char* p = (char*)L->buf;
+    size_t fb = field_bytes_aligned(L->felems);
+    L->parts.resize(L->nlocal);
+    for (int q = 0; q < L->nlocal; q++) {
+        SfPart& P = L->parts[q];
+        P.index = L->first + q;
+        P.z0 = P.index * L->lnz;
+        for (int f = 0; f < SF_NFIELDS; f++) {
+            P.f[f] = (double*)p;
+            p += fb;
+        }
+    }
+    L->dscratch = (double*)p;  // 256 bytes = 32 device scalars
+    cudaError_t e = cudaMallocHost(&L->hscratch, 256);
+    if (e != cudaSuccess) {
+        if (L->owns) cudaFree(L->buf);
+        delete L;
+        return sf_fail(SF_ERR_CUDA, "cudaMallocHost: %s", cudaGetErrorString(e));
+    }
+    e = cudaMemsetAsync(L->buf, 0, need, L->stream);
+    if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+    *out = L;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_destroy(sf_level* L) {
+    if (!L) return SF_OK;
+    cudaStreamSynchronize(L->stream);
+    if (L->owns) cudaFree(L->buf);
+    cudaFreeHost(L->hscratch);
+    delete L;
+    return SF_OK;
+}
+
+PV sf_view(const sf_level* L, int p) {
+    PV v;
+    for (int f = 0; f < SF_NFIELDS; f++) v.f[f] = L->parts[p].f[f];
+    v.nx = L->nx; v.ny = L->ny; v.nz = L->lnz;
+    v.z0 = L->parts[p].z0; v.gnz = L->gnz;
+    v.js = L->js; v.ks = L->ks;
+    return v;
+}
+
+static sf_status check_field(int f) {
+    if (f < 0 || f >= SF_NFIELDS) return sf_fail(SF_ERR_INVALID, "bad field id %d", f);
+    return SF_OK;
+}
+
+// host extent of a field per part: (nzh planes, nyh rows, nxh columns)
+static void host_extent(const sf_level* L, int field, int* nxh, int* nyh, int* nzh) {
+    *nxh = L->nx + (field == SF_BETA_I);
+    *nyh = L->ny + (field == SF_BETA_J);
+    *nzh = L->lnz + (field == SF_BETA_K);
+}
+
+static sf_status copy3d(sf_level* L, int field, double* host, bool up) {
+    int nxh, nyh, nzh;
+    host_extent(L, field, &nxh, &nyh, &nzh);
+    for (int q = 0; q < L->nlocal; q++) {
+        cudaMemcpy3DParms m = {};
+        double* dev = L->parts[q].f[field] + (long)SF_GZ * L->ks + (long)SF_GY * L->js + SF_OX;
+        double* hp = host + (size_t)q * L->lnz * nyh * nxh;  // parts share the interface face
+        cudaPitchedPtr dp = make_cudaPitchedPtr(dev, L->js * sizeof(double), nxh * sizeof(double),
+                                                L->ny + 2 * SF_GY);
+        cudaPitchedPtr hpp = make_cudaPitchedPtr(hp, nxh * sizeof(double), nxh * sizeof(double), nyh);
+        m.extent = make_cudaExtent(nxh * sizeof(double), nyh, nzh);
+        if (up) {
+            m.srcPtr = hpp; m.dstPtr = dp; m.kind = cudaMemcpyHostToDevice;
+        } else {
+            m.srcPtr = dp; m.dstPtr = hpp; m.kind = cudaMemcpyDeviceToHost;
+        }
+        SF_CUDA(cudaMemcpy3DAsync(&m, L->stream));
+    }
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_upload(sf_level* L, int field, const double* host) {
+    if (!L || !host) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    SF_TRY(check_field(field));
+    return copy3d(L, field, const_cast<double*>(host), true);
+}
+
+extern "C" sf_status sf_level_download(sf_level* L, int field, double* host) {
+    if (!L || !host) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    SF_TRY(check_field(field));
+    SF_TRY(copy3d(L, field, host, false));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_field_ptr(sf_level* L, int part, int field, double** dev,
+                                        long strides[3]) {
+    if (!L || !dev) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    SF_TRY(check_field(field));
+    if (part < 0 || part >= L->nlocal) return sf_fail(SF_ERR_INVALID, "bad local part %d", part);
+    *dev = L->parts[part].f[field] + (long)SF_GZ * L->ks + (long)SF_GY * L->js + SF_OX;
+    if (strides) {
+        strides[0] = 1; strides[1] = L->js; strides[2] = L->ks;
+    }
+    return SF_OK;
+}
+
+extern "C" sf_status sf_sync(sf_level* L) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_CUDA(cudaGetLastError());
+    return SF_OK;
+}
+
+// ----------------------------------------------------------------- operators
+extern "C" sf_status sf_init_problem(sf_level* L, int problem, double a, double b, int want_rhs) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    if (problem != 0 && problem != 1) return sf_fail(SF_ERR_INVALID, "problem must be 0 or 1");
+    if (want_rhs) SF_TRY(k_zero(L, SF_U));
+    return k_init_problem(L, problem, a, b, want_rhs);
+}
+
+extern "C" sf_status sf_rebuild_operator(sf_level* L, double a, double b) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    // coefficient halos for the colour-fused smoother's redundant ring work
+    for (int f : {SF_ALPHA, SF_BETA_I, SF_BETA_J, SF_BETA_K}) SF_TRY(sf_halo(L, f, 2));
+    SF_TRY(k_dinv(L, a, b));
+    return sf_halo(L, SF_DINV, 2);
+}
+
+extern "C" sf_status sf_apply_bc(sf_level* L, int field) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(field));
+    return k_bc(L, field);
+}
+
+extern "C" sf_status sf_apply_op(sf_level* L, int out, int x, double a, double b) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(out));
+    SF_TRY(check_field(x));
+    if (out == x) return sf_fail(SF_ERR_INVALID, "out must differ from x");
+    return k_apply_op(L, out, x, a, b);
+}
+
+extern "C" sf_status sf_residual(sf_level* L, int res, int x, int rhs, double a, double b) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(res));
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(rhs));
+    if (res == x) return sf_fail(SF_ERR_INVALID, "res must differ from x");
+    return k_residual(L, res, x, rhs, a, b);
+}
+
+static void swap_fields(sf_level* L, int f1, int f2) {
+    for (auto& P : L->parts) std::swap(P.f[f1], P.f[f2]);
+}
+
+extern "C" sf_status sf_smooth_gsrb(sf_level* L, int x, int rhs, double a, double b, int rb_pairs,
+                                    int kind) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(rhs));
+    if (rb_pairs < 0) return sf_fail(SF_ERR_INVALID, "rb_pairs < 0");
+    if (x == rhs || x == SF_DINV || rhs == SF_DINV)
+        return sf_fail(SF_ERR_INVALID, "x, rhs and DINV must be distinct fields");
+    bool fused_ok = gsrb_fused_supported(L) && (x == SF_U || x == SF_TMP) && rhs != SF_TMP &&
+                    rhs != SF_U;
+    if (kind == SF_SMOOTH_FUSED && !fused_ok)
+        return sf_fail(SF_ERR_SHAPE, "fused smoother unsupported for this level/fields");
+    bool fused = (kind == SF_SMOOTH_FUSED) || (kind == SF_SMOOTH_AUTO && fused_ok);
+    if (rb_pairs == 0) return SF_OK;
+    if (fused) {
+        int other = (x == SF_U) ? SF_TMP : SF_U;
+        SF_TRY(sf_halo(L, rhs, 1));
+        for (int p = 0; p < rb_pairs; p++) {
+            SF_TRY(sf_halo(L, x, 2));
+            SF_TRY(k_gsrb_pair_fused(L, x, other, rhs, a, b));
+            swap_fields(L, x, other);  // result now lives under the id `x`
+        }
+        return SF_OK;
+    }
+    for (int p = 0; p < rb_pairs; p++) {
+        SF_TRY(k_gsrb_colour(L, x, rhs, a, b, 0));
+        SF_TRY(k_gsrb_colour(L, x, rhs, a, b, 1));
+    }
+    return SF_OK;
+}
+
+static bool coarse_of(const sf_level* C, const sf_level* F) {
+    return C->gnx * 2 == F->gnx && C->gny * 2 == F->gny && C->gnz * 2 == F->gnz &&
+           (C->nparts == F->nparts || C->nparts == 1) && (F->lnz % 2 == 0);
+}
+
+extern "C" sf_status sf_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind) {
+    if (!C || !F) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(cf));
+    SF_TRY(check_field(ff));
+    if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
+    if (kind < SF_RESTRICT_CELL || kind > SF_RESTRICT_FACE_K)
+        return sf_fail(SF_ERR_INVALID, "bad restriction kind");
+    return k_restrict(C, cf, F, ff, kind);
+}
+
+extern "C" sf_status sf_interpolate(sf_level* F, int ff, double prescale, sf_level* C, int cf,
+                                    int kind) {
+    if (!C || !F) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(cf));
+    SF_TRY(check_field(ff));
+    if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
+    if (kind != SF_INTERP_P0 && kind != SF_INTERP_PL)
+        return sf_fail(SF_ERR_INVALID, "bad interpolation kind");
+    return k_interp(F, ff, prescale, C, cf, kind);
+}
+
+sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst) {
+    SF_TRY(k_norm(L, field, kind, dst));
+    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+        SF_TRY(sf_allreduce_scalar(L->comm, dst, kind == SF_NORM_MAX ? 0 : 1, L->stream));
+    return SF_OK;
+}
+
+extern "C" sf_status sf_norm(sf_level* L, int field, int kind, double* out) {
+    if (!L || !out) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    SF_TRY(check_field(field));
+    if (kind != SF_NORM_MAX && kind != SF_NORM_L2) return sf_fail(SF_ERR_INVALID, "bad norm kind");
+    SF_TRY(sf_norm_async(L, field, kind, L->dscratch));
+    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
+                            L->stream));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    double v = L->hscratch[0];
+    *out = (kind == SF_NORM_L2) ? sqrt(v) : v;
+    return SF_OK;
+}

@@ -1,0 +1,278 @@
+// Multigrid driver (A9): hierarchy construction, V-cycle, F-cycle, solve.
+//
+// PAPER.md:595-599 (restriction, smoothing, interpolation over grid spacings),
+// 627-629 (two GSRB smooths = 4 sweeps pre and post), 647-653 (smoother,
+// residual, restriction, interpolation, boundary stencils).  Coarse operators
+// are re-discretised from restricted alpha / beta with h_c = 2h (reading R-7);
+// bottom = exact solve at min dim 2 (reading R-8).
+//
+// Every cycle only ENQUEUES work on the finest level's stream (no host sync),
+// so a whole V-cycle (+ its convergence residual and norm) is captured once as
+// a CUDA graph and replayed: levels <= 64^3 are launch-latency bound.
+#include <cmath>
+
+#include "sf_internal.h"
+
+struct sf_mg {
+    std::vector<sf_level*> lv;
+    std::vector<bool> own;
+    double a, b;
+    sf_mg_opts o;
+    double* ainv = nullptr;
+    cudaGraphExec_t gexec[2] = {nullptr, nullptr};  // [0] V-cycle+check, [1] F-cycle+check
+    long long gnodes[2] = {0, 0};
+    bool graph_failed = false;
+};
+
+extern "C" void sf_mg_opts_default(sf_mg_opts* o) {
+    if (!o) return;
+    o->pre_pairs = 2;
+    o->post_pairs = 2;
+    o->vcycle_interp = SF_INTERP_P0;
+    o->fcycle_interp = SF_INTERP_PL;
+    o->agglom_min_planes = 8;
+    o->max_cycles = 50;
+    o->use_graph = 1;
+    o->smoother = SF_SMOOTH_AUTO;
+    o->rtol = 1e-10;
+}
+
+static sf_status destroy_levels(sf_mg* m) {
+    for (size_t l = 0; l < m->lv.size(); l++)
+        if (m->own[l]) sf_level_destroy(m->lv[l]);
+    m->lv.clear();
+    return SF_OK;
+}
+
+extern "C" sf_status sf_mg_destroy(sf_mg* m) {
+    if (!m) return SF_OK;
+    if (!m->lv.empty()) cudaStreamSynchronize(m->lv[0]->stream);
+    for (auto& g : m->gexec)
+        if (g) cudaGraphExecDestroy(g);
+    if (m->ainv) cudaFree(m->ainv);
+    destroy_levels(m);
+    delete m;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double b,
+                                  const sf_mg_opts* opts) {
+    if (!out || !fine) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    *out = nullptr;
+    sf_mg* m = new sf_mg();
+    m->a = a; m->b = b;
+    if (opts) m->o = *opts; else sf_mg_opts_default(&m->o);
+    if (m->o.pre_pairs < 0 || m->o.post_pairs < 0 || m->o.max_cycles < 1 ||
+        m->o.agglom_min_planes < 2) {
+        delete m;
+        return sf_fail(SF_ERR_INVALID, "bad mg options");
+    }
+    m->lv.push_back(fine);
+    m->own.push_back(false);
+    // coarsen while every dim is even and the min dim is > 2
+    for (;;) {
+        sf_level* F = m->lv.back();
+        int mn = std::min(F->gnx, std::min(F->gny, F->gnz));
+        if (mn <= 2 || (F->gnx | F->gny | F->gnz) & 1) break;
+        int cx = F->gnx / 2, cy = F->gny / 2, cz = F->gnz / 2;
+        bool last = std::min(cx, std::min(cy, cz)) <= 2 || ((cx | cy | cz) & 1);
+        bool distributed = F->nparts > 1 && F->comm && !last &&
+                           F->lnz / 2 >= m->o.agglom_min_planes && F->lnz % 2 == 0;
+        if (F->nparts > 1 && F->lnz % 2 != 0) {
+            sf_mg_destroy(m);
+            return sf_fail(SF_ERR_SHAPE, "odd planes per part (%d) cannot coarsen", F->lnz);
+        }
+        sf_level* C = nullptr;
+        sf_status s = sf_level_create(&C, cx, cy, cz, 2.0 * F->h, distributed ? F->comm : nullptr,
+                                      F->stream, nullptr, 0);
+        if (s != SF_OK) {
+            sf_mg_destroy(m);
+            return s;
+        }
+        if (!distributed) C->rep_comm = F->comm ? F->comm : F->rep_comm;
+        m->lv.push_back(C);
+        m->own.push_back(true);
+    }
+    sf_level* B = m->lv.back();
+    if (B->nparts != 1 || (long)B->gnx * B->gny * B->gnz > 64) {
+        sf_mg_destroy(m);
+        return sf_fail(SF_ERR_SHAPE, "coarsest level %dx%dx%d is not a <=64-cell replicated box",
+                       B->gnx, B->gny, B->gnz);
+    }
+    // operator on every level: restrict coefficients (A7), rebuild Dinv (A4)
+    sf_status s = sf_rebuild_operator(fine, a, b);
+    for (size_t l = 1; l < m->lv.size() && s == SF_OK; l++) {
+        sf_level* F = m->lv[l - 1];
+        sf_level* C = m->lv[l];
+        s = k_restrict(C, SF_ALPHA, F, SF_ALPHA, SF_RESTRICT_CELL);
+        if (s == SF_OK) s = k_restrict(C, SF_BETA_I, F, SF_BETA_I, SF_RESTRICT_FACE_I);
+        if (s == SF_OK) s = k_restrict(C, SF_BETA_J, F, SF_BETA_J, SF_RESTRICT_FACE_J);
+        if (s == SF_OK) s = k_restrict(C, SF_BETA_K, F, SF_BETA_K, SF_RESTRICT_FACE_K);
+        if (s == SF_OK) s = sf_rebuild_operator(C, a, b);
+    }
+    if (s == SF_OK) {
+        int n = B->gnx * B->gny * B->gnz;
+        cudaError_t e = cudaMalloc(&m->ainv, (size_t)n * n * sizeof(double));
+        if (e != cudaSuccess) s = sf_fail(SF_ERR_OOM, "bottom inverse: %s", cudaGetErrorString(e));
+    }
+    if (s == SF_OK) s = k_bottom_setup(B, a, b, m->ainv);
+    if (s == SF_OK) {
+        cudaError_t e = cudaStreamSynchronize(fine->stream);
+        if (e != cudaSuccess) s = sf_fail(SF_ERR_CUDA, "mg setup: %s", cudaGetErrorString(e));
+    }
+    if (s != SF_OK) {
+        sf_mg_destroy(m);
+        return s;
+    }
+    *out = m;
+    return SF_OK;
+}
+
+extern "C" sf_status sf_mg_num_levels(const sf_mg* m, int* n) {
+    if (!m || !n) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    *n = (int)m->lv.size();
+    return SF_OK;
+}
+
+extern "C" sf_status sf_mg_level(sf_mg* m, int l, sf_level** out) {
+    if (!m || !out) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    if (l < 0 || l >= (int)m->lv.size()) return sf_fail(SF_ERR_INVALID, "bad level %d", l);
+    *out = m->lv[l];
+    return SF_OK;
+}
+
+static sf_status smooth(sf_mg* m, sf_level* L, int pairs) {
+    return sf_smooth_gsrb(L, SF_U, SF_F, m->a, m->b, pairs, m->o.smoother);
+}
+
+// V(l): smooth, residual, restrict, zero e_{l+1}, V(l+1), e_l += P0 e_{l+1}, smooth
+static sf_status vcyc(sf_mg* m, int l) {
+    sf_level* L = m->lv[l];
+    if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
+    sf_level* C = m->lv[l + 1];
+    SF_TRY(smooth(m, L, m->o.pre_pairs));
+    SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
+    SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
+    SF_TRY(k_zero(C, SF_U));
+    SF_TRY(vcyc(m, l + 1));
+    SF_TRY(k_interp(L, SF_U, 1.0, C, SF_U, m->o.vcycle_interp));
+    SF_TRY(smooth(m, L, m->o.post_pairs));
+    return SF_OK;
+}
+
+static sf_status fcyc(sf_mg* m) {
+    int nl = (int)m->lv.size();
+    for (int l = 1; l < nl; l++)
+        SF_TRY(k_restrict(m->lv[l], SF_F, m->lv[l - 1], SF_F, SF_RESTRICT_CELL));
+    SF_TRY(k_bottom_solve(m->lv[nl - 1], SF_U, SF_F, m->ainv));
+    for (int l = nl - 2; l >= 0; l--) {
+        SF_TRY(k_interp(m->lv[l], SF_U, 0.0, m->lv[l + 1], SF_U, m->o.fcycle_interp));
+        SF_TRY(vcyc(m, l));
+    }
+    return SF_OK;
+}
+
+// residual of the finest level and its max norm into dscratch[0] + pinned copy
+static sf_status check(sf_mg* m) {
+    sf_level* L = m->lv[0];
+    SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
+    SF_TRY(sf_norm_async(L, SF_R, SF_NORM_MAX, L->dscratch));
+    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
+                            L->stream));
+    return SF_OK;
+}
+
+static bool graphs_allowed(const sf_mg* m) {
+    if (!m->o.use_graph || m->graph_failed) return false;
+    if (m->lv[0]->stream == nullptr) return false;  // legacy stream cannot be captured
+    // the fused smoother swaps U/TMP per pair; only an even count per smooth
+    // leaves the host-side mapping unchanged across a captured cycle
+    return (m->o.pre_pairs % 2 == 0 && m->o.post_pairs % 2 == 0) ||
+           m->o.smoother == SF_SMOOTH_COLOUR;
+}
+
+// run cycle kind (0 = V on level 0, 1 = F) followed by the check
+static sf_status run_cycle(sf_mg* m, int kind) {
+    sf_level* L = m->lv[0];
+    auto body = [&]() -> sf_status {
+        if (kind == 0) SF_TRY(vcyc(m, 0)); else SF_TRY(fcyc(m));
+        return check(m);
+    };
+    if (!graphs_allowed(m)) return body();
+    if (!m->gexec[kind]) {
+        long long before, after;
+        sf_launch_count(&before, 0);
+        if (cudaStreamBeginCapture(L->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+            cudaGetLastError();
+            m->graph_failed = true;
+            return body();
+        }
+        sf_status s = body();
+        cudaGraph_t g = nullptr;
+        cudaError_t e = cudaStreamEndCapture(L->stream, &g);
+        if (s != SF_OK) {
+            if (g) cudaGraphDestroy(g);
+            return s;
+        }
+        if (e != cudaSuccess || !g) {
+            cudaGetLastError();
+            m->graph_failed = true;
+            return body();
+        }
+        e = cudaGraphInstantiate(&m->gexec[kind], g, 0);
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            m->gexec[kind] = nullptr;
+            m->graph_failed = true;
+            return body();
+        }
+        sf_launch_count(&after, 0);
+        m->gnodes[kind] = after - before;
+        sf_count_launch(-(after - before));  // captured, not launched
+    }
+    SF_CUDA(cudaGraphLaunch(m->gexec[kind], L->stream));
+    sf_count_launch(m->gnodes[kind]);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_vcycle(sf_mg* m, int l) {
+    if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
+    if (l < 0 || l >= (int)m->lv.size()) return sf_fail(SF_ERR_INVALID, "bad level %d", l);
+    return vcyc(m, l);
+}
+
+extern "C" sf_status sf_fcycle(sf_mg* m) {
+    if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
+    return fcyc(m);
+}
+
+extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles, int* cycles,
+                              double* hist) {
+    if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
+    if (max_cycles < 1) max_cycles = m->o.max_cycles;
+    if (!(rtol > 0)) rtol = m->o.rtol;
+    sf_level* L = m->lv[0];
+    double fn;
+    SF_TRY(sf_norm(L, SF_F, SF_NORM_MAX, &fn));
+    if (cycles) *cycles = 0;
+    if (!(fn == fn) || std::isinf(fn)) return sf_fail(SF_ERR_NUMERIC, "rhs has NaN/Inf");
+    if (fn == 0.0) {
+        SF_TRY(k_zero(L, SF_U));
+        return sf_sync(L);
+    }
+    int c = 0;
+    bool first = true;
+    while (c < max_cycles) {
+        SF_TRY(run_cycle(m, (fcycle && first) ? 1 : 0));
+        first = false;
+        SF_CUDA(cudaStreamSynchronize(L->stream));
+        double rel = L->hscratch[0] / fn;
+        if (hist) hist[c] = rel;
+        c++;
+        if (cycles) *cycles = c;
+        if (!(rel == rel) || std::isinf(rel)) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
+        if (rel < rtol) return SF_OK;
+    }
+    return sf_fail(SF_ERR_NOT_CONVERGED, "no convergence to %g in %d cycles", rtol, max_cycles);
+}

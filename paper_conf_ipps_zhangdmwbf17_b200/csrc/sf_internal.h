@@ -1,0 +1,116 @@
+// Internal definitions of libsf (CUDA C++ for sm_100a).  Not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdio>
+#include <string>
+#include <vector>
+
+#include "sf.h"
+
+// ------------------------------------------------------------------ layout (A1)
+// Per part and field: (lnz + 2*SF_GZ) planes x (ny + 2*SF_GY) rows x js doubles.
+// Element (i,j,k) at (k+SF_GZ)*ks + (j+SF_GY)*js + SF_OX + i, i in [-2, nx+1].
+// SF_OX = 4 puts i = 0 on a 32-byte boundary (js is a multiple of 16 doubles,
+// every field base is 256-byte aligned), so double2 / 16-byte cp.async loads
+// of interior rows are aligned.  Two ghost planes in z (depth-2 slab halos of
+// the colour-fused smoother) and two ghost rows in y (its 2-ring tile loads).
+#define SF_OX 4
+#define SF_GY 2
+#define SF_GZ 2
+
+struct sf_comm {
+    int kind;          // 0 = local (all parts in this process), 1 = NCCL
+    int nparts;        // parts in the whole job
+    int nlocal;        // parts held by this process
+    int first;         // global index of the first local part
+    int rank, nranks;
+    void* nccl;        // ncclComm_t
+};
+
+struct SfPart {
+    int index;                 // global part index
+    int z0;                    // global z of local plane 0
+    double* f[SF_NFIELDS];     // base of each field's allocation (plane -SF_GZ)
+};
+
+struct sf_level {
+    int gnx, gny, gnz;         // global cells
+    int nx, ny, lnz;           // per-part interior dims
+    double h;
+    long js, ks;               // strides (doubles)
+    size_t felems;             // doubles per field per part
+    int nparts, nlocal, first; // decomposition (nparts == 1: single / replicated)
+    const sf_comm* comm;       // NULL for a single / replicated level
+    const sf_comm* rep_comm;   // replicated (agglomerated) level: the job's comm
+    std::vector<SfPart> parts; // local parts
+    cudaStream_t stream;
+    void* buf;
+    bool owns;
+    double* dscratch;          // device scalars (norms)
+    double* hscratch;          // pinned host scalars
+};
+
+// Part view passed to kernels by value.  Kernels must only index f[] with
+// compile-time constants (a runtime index spills the struct to local memory);
+// fields chosen at run time are passed as separate pointers.
+struct PV {
+    double* f[SF_NFIELDS];
+    int nx, ny, nz;            // local interior dims
+    int z0, gnz;               // global z offset / extent (Dirichlet faces at 0, gnz)
+    long js, ks;
+};
+
+__host__ __device__ __forceinline__ long sf_ix(const PV& v, int i, int j, int k) {
+    return (long)(k + SF_GZ) * v.ks + (long)(j + SF_GY) * v.js + SF_OX + i;
+}
+
+PV sf_view(const sf_level* L, int p);
+
+sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst);
+
+// ------------------------------------------------------------------ errors
+sf_status sf_fail(sf_status s, const char* fmt, ...);
+#define SF_CUDA(call)                                                                  \
+    do {                                                                               \
+        cudaError_t e_ = (call);                                                       \
+        if (e_ != cudaSuccess)                                                         \
+            return sf_fail(SF_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,     \
+                           cudaGetErrorString(e_));                                    \
+    } while (0)
+#define SF_TRY(call)                                \
+    do {                                            \
+        sf_status s_ = (call);                      \
+        if (s_ != SF_OK) return s_;                 \
+    } while (0)
+#define SF_LAUNCHED() sf_count_launch()
+void sf_count_launch(long long n = 1);
+sf_status sf_check_launch(const char* what);
+
+// ------------------------------------------------------------------ kernels (kernels.cu)
+sf_status k_apply_op(sf_level* L, int out, int x, double a, double b);
+sf_status k_residual(sf_level* L, int res, int x, int rhs, double a, double b);
+sf_status k_gsrb_colour(sf_level* L, int x, int rhs, double a, double b, int colour);
+sf_status k_dinv(sf_level* L, double a, double b);
+sf_status k_bc(sf_level* L, int field);
+sf_status k_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind);
+sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind);
+sf_status k_norm(sf_level* L, int field, int kind, double* dst_dev);
+sf_status k_zero(sf_level* L, int field);
+sf_status k_init_problem(sf_level* L, int problem, double a, double b, int want_rhs);
+sf_status k_bottom_setup(sf_level* L, double a, double b, double* ainv);
+sf_status k_bottom_solve(sf_level* L, int x, int rhs, const double* ainv);
+
+// fused colour pair (gsrb_fused.cu)
+bool gsrb_fused_supported(const sf_level* L);
+sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b);
+
+// ------------------------------------------------------------------ comm (comm.cu)
+// Exchange `depth` z-halo planes of `field` between neighbouring parts.
+sf_status sf_halo(sf_level* L, int field, int depth);
+// Replicated coarse level C receives, on every process, the planes each part
+// of the distributed fine level F wrote into it (in-place all-gather).
+sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part);
+// Reduce a device scalar over ranks (op 0 = max, 1 = sum); in place.
+sf_status sf_allreduce_scalar(const sf_comm* comm, double* dev, int op, cudaStream_t s);

@@ -1,0 +1,413 @@
+"""Thin ctypes binding of libsf (include/sf.h).  Argument marshalling only.
+
+Every function named ``sf_*`` here calls the C entry point of the same name;
+the small classes (Comm, Level, MG) only hold handles, the torch-owned device
+buffer and stream, and convert numpy host arrays.  All arithmetic of the
+method runs in libsf's CUDA kernels.  There is no CPU fallback: if libsf.so is
+missing or no sm_100 device is present, the calls raise.
+
+PyTorch is used for device memory (one uint8 tensor per level, passed to
+sf_level_create as the caller-owned buffer) and streams
+(``torch.cuda.Stream``), and torch.distributed broadcasts the NCCL id.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsf.so")
+
+# enums (include/sf.h)
+SF_OK, SF_ERR_INVALID, SF_ERR_SHAPE, SF_ERR_OOM, SF_ERR_CUDA, SF_ERR_NCCL = range(6)
+SF_ERR_NOT_CONVERGED, SF_ERR_NUMERIC = 6, 7
+(SF_U, SF_F, SF_R, SF_TMP, SF_ALPHA, SF_BETA_I, SF_BETA_J, SF_BETA_K, SF_DINV) = range(9)
+SF_NFIELDS = 9
+SF_RESTRICT_CELL, SF_RESTRICT_FACE_I, SF_RESTRICT_FACE_J, SF_RESTRICT_FACE_K = range(4)
+SF_INTERP_P0, SF_INTERP_PL = 0, 1
+SF_NORM_MAX, SF_NORM_L2 = 0, 1
+SF_SMOOTH_AUTO, SF_SMOOTH_COLOUR, SF_SMOOTH_FUSED = 0, 1, 2
+
+FIELD_IDS = {"u": SF_U, "f": SF_F, "r": SF_R, "tmp": SF_TMP, "alpha": SF_ALPHA,
+             "beta_i": SF_BETA_I, "beta_j": SF_BETA_J, "beta_k": SF_BETA_K, "dinv": SF_DINV}
+
+EXPORTS = [
+    "sf_mg_opts_default", "sf_last_error", "sf_version", "sf_comm_create_local",
+    "sf_get_unique_id", "sf_comm_create_nccl", "sf_comm_destroy", "sf_comm_info",
+    "sf_level_bytes_needed", "sf_level_create", "sf_level_destroy", "sf_level_upload",
+    "sf_level_download", "sf_level_field_ptr", "sf_init_problem", "sf_rebuild_operator",
+    "sf_apply_bc", "sf_apply_op", "sf_smooth_gsrb", "sf_residual", "sf_restrict",
+    "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
+    "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count",
+]
+
+
+class SfError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"libsf status {status}: {msg}")
+        self.status = status
+
+
+class MgOpts(C.Structure):
+    _fields_ = [("pre_pairs", C.c_int), ("post_pairs", C.c_int), ("vcycle_interp", C.c_int),
+                ("fcycle_interp", C.c_int), ("agglom_min_planes", C.c_int),
+                ("max_cycles", C.c_int), ("use_graph", C.c_int), ("smoother", C.c_int),
+                ("rtol", C.c_double)]
+
+
+_lib = None
+_vp, _d, _i = C.c_void_p, C.c_double, C.c_int
+_P = C.POINTER(C.c_double)
+
+
+def lib():
+    """Load libsf.so (raises if it has not been built -- no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: build it with "
+                           "`python -m paper_conf_ipps_zhangdmwbf17_b200.build` (no CPU fallback)")
+    L = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
+    sig = {
+        "sf_mg_opts_default": (None, [C.POINTER(MgOpts)]),
+        "sf_last_error": (C.c_char_p, []),
+        "sf_version": (C.c_char_p, []),
+        "sf_comm_create_local": (_i, [C.POINTER(_vp), _i]),
+        "sf_get_unique_id": (_i, [C.c_char_p]),
+        "sf_comm_create_nccl": (_i, [C.POINTER(_vp), C.c_char_p, _i, _i]),
+        "sf_comm_destroy": (_i, [_vp]),
+        "sf_comm_info": (_i, [_vp, C.POINTER(_i), C.POINTER(_i), C.POINTER(_i)]),
+        "sf_level_bytes_needed": (_i, [_i, _i, _i, _vp, C.POINTER(C.c_size_t)]),
+        "sf_level_create": (_i, [C.POINTER(_vp), _i, _i, _i, _d, _vp, _vp, _vp, C.c_size_t]),
+        "sf_level_destroy": (_i, [_vp]),
+        "sf_level_upload": (_i, [_vp, _i, _vp]),
+        "sf_level_download": (_i, [_vp, _i, _vp]),
+        "sf_level_field_ptr": (_i, [_vp, _i, _i, C.POINTER(_P), C.POINTER(C.c_long)]),
+        "sf_init_problem": (_i, [_vp, _i, _d, _d, _i]),
+        "sf_rebuild_operator": (_i, [_vp, _d, _d]),
+        "sf_apply_bc": (_i, [_vp, _i]),
+        "sf_apply_op": (_i, [_vp, _i, _i, _d, _d]),
+        "sf_smooth_gsrb": (_i, [_vp, _i, _i, _d, _d, _i, _i]),
+        "sf_residual": (_i, [_vp, _i, _i, _i, _d, _d]),
+        "sf_restrict": (_i, [_vp, _i, _vp, _i, _i]),
+        "sf_interpolate": (_i, [_vp, _i, _d, _vp, _i, _i]),
+        "sf_norm": (_i, [_vp, _i, _i, _P]),
+        "sf_sync": (_i, [_vp]),
+        "sf_mg_create": (_i, [C.POINTER(_vp), _vp, _d, _d, C.POINTER(MgOpts)]),
+        "sf_mg_num_levels": (_i, [_vp, C.POINTER(_i)]),
+        "sf_mg_level": (_i, [_vp, _i, C.POINTER(_vp)]),
+        "sf_vcycle": (_i, [_vp, _i]),
+        "sf_fcycle": (_i, [_vp]),
+        "sf_solve": (_i, [_vp, _i, _d, _i, C.POINTER(_i), _P]),
+        "sf_mg_destroy": (_i, [_vp]),
+        "sf_launch_count": (_i, [C.POINTER(C.c_longlong), _i]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype, f.argtypes = res, args
+    _lib = L
+    return L
+
+
+def _check(status):
+    if status != SF_OK:
+        raise SfError(status, lib().sf_last_error().decode(errors="replace"))
+    return status
+
+
+# ------------------------------------------------------------ C-ABI mirrors
+def sf_version():
+    return lib().sf_version().decode()
+
+
+def sf_mg_opts_default():
+    o = MgOpts()
+    lib().sf_mg_opts_default(C.byref(o))
+    return o
+
+
+def sf_comm_create_local(nparts):
+    h = _vp()
+    _check(lib().sf_comm_create_local(C.byref(h), int(nparts)))
+    return h
+
+
+def sf_get_unique_id():
+    buf = C.create_string_buffer(128)
+    _check(lib().sf_get_unique_id(buf))
+    return buf.raw
+
+
+def sf_comm_create_nccl(uid, nranks, rank):
+    h = _vp()
+    _check(lib().sf_comm_create_nccl(C.byref(h), uid, int(nranks), int(rank)))
+    return h
+
+
+def sf_comm_destroy(h):
+    _check(lib().sf_comm_destroy(h))
+
+
+def sf_level_bytes_needed(gnx, gny, gnz, comm=None):
+    n = C.c_size_t()
+    _check(lib().sf_level_bytes_needed(gnx, gny, gnz, comm, C.byref(n)))
+    return n.value
+
+
+def sf_level_create(gnx, gny, gnz, h, comm=None, stream=None, dev_buf=None, buf_bytes=0):
+    out = _vp()
+    _check(lib().sf_level_create(C.byref(out), gnx, gny, gnz, float(h), comm, stream, dev_buf,
+                                 buf_bytes))
+    return out
+
+
+def sf_level_destroy(level):
+    _check(lib().sf_level_destroy(level))
+
+
+def sf_level_upload(level, field, host):
+    _check(lib().sf_level_upload(level, field, host))
+
+
+def sf_level_download(level, field, host):
+    _check(lib().sf_level_download(level, field, host))
+
+
+def sf_level_field_ptr(level, part, field):
+    p = _P()
+    st = (C.c_long * 3)()
+    _check(lib().sf_level_field_ptr(level, part, field, C.byref(p), st))
+    return C.cast(p, C.c_void_p).value, tuple(st)
+
+
+def sf_init_problem(level, problem, a, b, want_rhs=1):
+    _check(lib().sf_init_problem(level, problem, float(a), float(b), int(want_rhs)))
+
+
+def sf_rebuild_operator(level, a, b):
+    _check(lib().sf_rebuild_operator(level, float(a), float(b)))
+
+
+def sf_apply_bc(level, field):
+    _check(lib().sf_apply_bc(level, field))
+
+
+def sf_apply_op(level, out, x, a, b):
+    _check(lib().sf_apply_op(level, out, x, float(a), float(b)))
+
+
+def sf_smooth_gsrb(level, x, rhs, a, b, rb_pairs, kind=SF_SMOOTH_AUTO):
+    _check(lib().sf_smooth_gsrb(level, x, rhs, float(a), float(b), int(rb_pairs), int(kind)))
+
+
+def sf_residual(level, res, x, rhs, a, b):
+    _check(lib().sf_residual(level, res, x, rhs, float(a), float(b)))
+
+
+def sf_restrict(coarse, c_field, fine, f_field, kind=SF_RESTRICT_CELL):
+    _check(lib().sf_restrict(coarse, c_field, fine, f_field, kind))
+
+
+def sf_interpolate(fine, f_field, prescale, coarse, c_field, kind=SF_INTERP_P0):
+    _check(lib().sf_interpolate(fine, f_field, float(prescale), coarse, c_field, kind))
+
+
+def sf_norm(level, field, kind=SF_NORM_MAX):
+    out = C.c_double()
+    _check(lib().sf_norm(level, field, kind, C.byref(out)))
+    return out.value
+
+
+def sf_sync(level):
+    _check(lib().sf_sync(level))
+
+
+def sf_mg_create(level, a, b, opts=None):
+    out = _vp()
+    _check(lib().sf_mg_create(C.byref(out), level, float(a), float(b),
+                              C.byref(opts) if opts is not None else None))
+    return out
+
+
+def sf_mg_num_levels(mg):
+    n = _i()
+    _check(lib().sf_mg_num_levels(mg, C.byref(n)))
+    return n.value
+
+
+def sf_mg_level(mg, l):
+    out = _vp()
+    _check(lib().sf_mg_level(mg, l, C.byref(out)))
+    return out
+
+
+def sf_vcycle(mg, l=0):
+    _check(lib().sf_vcycle(mg, l))
+
+
+def sf_fcycle(mg):
+    _check(lib().sf_fcycle(mg))
+
+
+def sf_solve(mg, fcycle=True, rtol=1e-10, max_cycles=50, raise_on_error=True):
+    """Returns (status, cycles, history)."""
+    cyc = _i()
+    hist = (C.c_double * (max_cycles + 1))()
+    st = lib().sf_solve(mg, int(fcycle), float(rtol), int(max_cycles), C.byref(cyc), hist)
+    if raise_on_error:
+        _check(st)
+    return st, cyc.value, list(hist[:cyc.value])
+
+
+def sf_mg_destroy(mg):
+    _check(lib().sf_mg_destroy(mg))
+
+
+def sf_launch_count(reset=False):
+    n = C.c_longlong()
+    _check(lib().sf_launch_count(C.byref(n), int(reset)))
+    return n.value
+
+
+# ------------------------------------------------------------ convenience layer
+def host_shape(field, nx, ny, nz):
+    return {SF_BETA_I: (nz, ny, nx + 1), SF_BETA_J: (nz, ny + 1, nx),
+            SF_BETA_K: (nz + 1, ny, nx)}.get(field, (nz, ny, nx))
+
+
+class Comm:
+    """Loopback (``Comm.local(P)``: P slabs in this process) or NCCL comm."""
+
+    def __init__(self, handle, nparts, nlocal, first):
+        self.h, self.nparts, self.nlocal, self.first = handle, nparts, nlocal, first
+
+    @classmethod
+    def local(cls, nparts):
+        return cls(sf_comm_create_local(nparts), nparts, nparts, 0)
+
+    @classmethod
+    def nccl(cls, group=None):
+        """One part per rank of the default (or given) torch.distributed group."""
+        import torch
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        uid = [sf_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0, group=group)
+        torch.cuda.synchronize()
+        return cls(sf_comm_create_nccl(uid[0], world, rank), world, 1, rank)
+
+    def close(self):
+        if self.h:
+            sf_comm_destroy(self.h)
+            self.h = None
+
+
+class Level:
+    """One level: device buffer from torch, stream from torch, handle from libsf."""
+
+    def __init__(self, nx, ny, nz, h=None, comm=None, stream=None, device=None):
+        import torch
+        self.gnx, self.gny, self.gnz = nx, ny, nz
+        self.h = (1.0 / max(nx, ny, nz)) if h is None else float(h)
+        self.comm = comm
+        chandle = comm.h if comm is not None else None
+        self.nparts = comm.nparts if comm is not None else 1
+        self.nlocal = comm.nlocal if comm is not None else 1
+        self.lnz = nz // self.nparts
+        dev = torch.device("cuda", torch.cuda.current_device()) if device is None else device
+        self.stream = stream if stream is not None else torch.cuda.Stream(device=dev)
+        nbytes = sf_level_bytes_needed(nx, ny, nz, chandle)
+        self.buf = torch.empty(nbytes + 256, dtype=torch.uint8, device=dev)
+        base = self.buf.data_ptr()
+        base = (base + 255) // 256 * 256
+        self.handle = sf_level_create(nx, ny, nz, self.h, chandle, self.stream.cuda_stream, base,
+                                      nbytes)
+
+    def host_shape(self, field):
+        return host_shape(field, self.gnx, self.gny, self.lnz * self.nlocal)
+
+    def upload(self, field, arr):
+        a = np.ascontiguousarray(arr, dtype=np.float64)
+        if a.shape != self.host_shape(field):
+            raise ValueError(f"field {field}: shape {a.shape} != {self.host_shape(field)}")
+        sf_level_upload(self.handle, field, a.ctypes.data)
+        sf_sync(self.handle)          # pageable host memory: keep `a` alive until done
+
+    def upload_async(self, field, pinned_ptr):
+        sf_level_upload(self.handle, field, pinned_ptr)
+
+    def download(self, field, out=None):
+        out = np.empty(self.host_shape(field)) if out is None else out
+        sf_level_download(self.handle, field, out.ctypes.data)
+        return out
+
+    def padded(self, field, part=0, ghost=1):
+        """Device copy of (lnz+2g, ny+2g, nx+2g) incl. ghost zone -> numpy (tests)."""
+        import torch
+        self.stream.synchronize()
+        ptr, (s0, s1, s2) = sf_level_field_ptr(self.handle, part, field)
+        base = self.buf.data_ptr()
+        off = (ptr - base) // 8
+        assert (ptr - base) % 8 == 0
+        nbytes = self.buf.numel() - (self.buf.numel() % 8)
+        d = self.buf[:nbytes].view(torch.float64)
+        g = ghost
+        out = np.empty((self.lnz + 2 * g, self.gny + 2 * g, self.gnx + 2 * g))
+        for k in range(-g, self.lnz + g):
+            start = off + k * s2 - g * s1 - g
+            rows = d[start: start + (self.gny + 2 * g) * s1].view(self.gny + 2 * g, s1)
+            out[k + g] = rows[:, : self.gnx + 2 * g].cpu().numpy()
+        return out
+
+    def set_coeffs(self, alpha, bi, bj, bk):
+        self.upload(SF_ALPHA, alpha)
+        self.upload(SF_BETA_I, bi)
+        self.upload(SF_BETA_J, bj)
+        self.upload(SF_BETA_K, bk)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            sf_level_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class MG:
+    def __init__(self, level, a, b, **opts):
+        o = sf_mg_opts_default()
+        for k, v in opts.items():
+            setattr(o, k, v)
+        self.level, self.a, self.b = level, a, b
+        self.handle = sf_mg_create(level.handle, a, b, o)
+
+    @property
+    def num_levels(self):
+        return sf_mg_num_levels(self.handle)
+
+    def solve(self, fcycle=True, rtol=1e-10, max_cycles=50, raise_on_error=True):
+        return sf_solve(self.handle, fcycle, rtol, max_cycles, raise_on_error)
+
+    def vcycle(self, l=0):
+        sf_vcycle(self.handle, l)
+
+    def fcycle(self):
+        sf_fcycle(self.handle)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            sf_mg_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

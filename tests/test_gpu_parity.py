@@ -1,0 +1,331 @@
+"""GPU parity: every libsf entry point (through the C ABI) against the CPU
+oracle on the same seeded inputs.  Tolerances:
+1e-12 relative L2 per call / per RB pair, 1e-10 after a full solve; bit-exact
+where both sides perform the identical additions (restriction, P0, BC)."""
+import numpy as np
+import pytest
+
+from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-12
+
+
+@pytest.fixture(scope="module")
+def sf():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_ipps_zhangdmwbf17_b200 import build, sf as S
+    build.build()
+    S.lib()
+    return S
+
+
+def rel(a, b):
+    return np.linalg.norm((a - b).ravel()) / max(np.linalg.norm(b.ravel()), 1e-300)
+
+
+def make_level(sf, shape, coeffs, parts=1, h=None):
+    nz, ny, nx = shape
+    comm = sf.Comm.local(parts) if parts > 1 else None
+    L = sf.Level(nx, ny, nz, h=h, comm=comm)
+    L.set_coeffs(*coeffs)
+    L._comm_keep = comm
+    return L
+
+
+SHAPES = [(16, 16, 16), (8, 6, 10), (20, 64, 64), (32, 24, 128), (40, 16, 192)]
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_upload_download_roundtrip(sf, shape):
+    nz, ny, nx = shape
+    coeffs = I.random_coeffs(nx, ny, nz, 1)
+    L = make_level(sf, shape, coeffs)
+    for f, arr in zip([sf.SF_ALPHA, sf.SF_BETA_I, sf.SF_BETA_J, sf.SF_BETA_K], coeffs):
+        assert np.array_equal(L.download(f), arr)
+    x = I.random_field(shape, 3)
+    L.upload(sf.SF_U, x)
+    assert np.array_equal(L.download(sf.SF_U), x)
+
+
+@pytest.mark.parametrize("shape", [(6, 5, 4), (16, 16, 16), (8, 8, 64)])
+def test_apply_bc(sf, oracle, shape):
+    nz, ny, nx = shape
+    L = make_level(sf, shape, I.random_coeffs(nx, ny, nz, 1))
+    x = I.random_field(shape, 0)
+    L.upload(sf.SF_U, x)
+    sf.sf_apply_bc(L.handle, sf.SF_U)
+    got = L.padded(sf.SF_U)
+    exp = oracle.apply_bc(oracle.Grid(nx, ny, nz, 1.0), oracle.pad(x))
+    assert np.array_equal(got, exp)
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("ab", [(0.0, 1.0), (1.0, 1.0), (2.5, 0.75)])
+def test_apply_op_and_residual(sf, oracle, shape, ab):
+    nz, ny, nx = shape
+    a, b = ab
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.random_coeffs(nx, ny, nz, 2)
+    L = make_level(sf, shape, coeffs)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), a, b, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    sf.sf_apply_op(L.handle, sf.SF_R, sf.SF_U, a, b)
+    assert rel(L.download(sf.SF_R), P.apply_op(x)) < TOL
+    sf.sf_residual(L.handle, sf.SF_R, sf.SF_U, sf.SF_F, a, b)
+    assert rel(L.download(sf.SF_R), P.residual(x, f)) < TOL
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_dinv(sf, oracle, shape):
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.random_coeffs(nx, ny, nz, 4)
+    L = make_level(sf, shape, coeffs)
+    sf.sf_rebuild_operator(L.handle, 1.5, 0.5)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.5, 0.5, *coeffs)
+    assert rel(L.download(sf.SF_DINV), P.dinv()) < 1e-14
+
+
+@pytest.mark.parametrize("shape", SHAPES + [(64, 64, 64), (24, 8, 64)])
+@pytest.mark.parametrize("kind", ["colour", "fused"])
+def test_gsrb_per_pair(sf, oracle, shape, kind):
+    """Each RB pair (BC, red, BC, black) matches the oracle to 1e-12."""
+    nz, ny, nx = shape
+    if kind == "fused" and (nx % 64 or ny % 8):
+        pytest.skip("fused kernel needs nx%64==0, ny%8==0")
+    a, b = 1.0, 1.0
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.hpgmg_coeffs(nx, ny, nz) if nx >= 64 else I.random_coeffs(nx, ny, nz, 5)
+    L = make_level(sf, shape, coeffs)
+    sf.sf_rebuild_operator(L.handle, a, b)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), a, b, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    k = sf.SF_SMOOTH_FUSED if kind == "fused" else sf.SF_SMOOTH_COLOUR
+    d = P.dinv()
+    for _ in range(3):
+        sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, a, b, 1, k)
+        x = P.smooth(x, f, 1, dinv=d)
+        assert rel(L.download(sf.SF_U), x) < TOL
+
+
+def test_fused_equals_colour(sf):
+    shape = (48, 32, 128)
+    nz, ny, nx = shape
+    coeffs = I.hpgmg_coeffs(nx, ny, nz)
+    outs = []
+    for k in (sf.SF_SMOOTH_COLOUR, sf.SF_SMOOTH_FUSED):
+        L = make_level(sf, shape, coeffs)
+        sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+        L.upload(sf.SF_U, I.random_field(shape, 0))
+        L.upload(sf.SF_F, I.random_field(shape, 1))
+        sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, k)
+        outs.append(L.download(sf.SF_U))
+    assert rel(outs[1], outs[0]) < 1e-14
+
+
+def test_c1_config(sf, oracle):
+    """BASELINE config 1: 16^3 CC Poisson, 4 GSRB sweeps + residual."""
+    n = 16
+    shape = (n, n, n)
+    h = 1.0 / n
+    coeffs = I.constant_coeffs(n, n, n)
+    L = make_level(sf, shape, coeffs)
+    sf.sf_rebuild_operator(L.handle, 0.0, 1.0)
+    P = oracle.Problem(oracle.Grid(n, n, n, h), 0.0, 1.0, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    for _ in range(2):
+        sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 0.0, 1.0, 1)
+        x = P.smooth(x, f, 1)
+        assert rel(L.download(sf.SF_U), x) < TOL
+    sf.sf_residual(L.handle, sf.SF_R, sf.SF_U, sf.SF_F, 0.0, 1.0)
+    assert rel(L.download(sf.SF_R), P.residual(x, f)) < TOL
+
+
+@pytest.mark.parametrize("fine", [(8, 8, 8), (16, 12, 20), (32, 32, 64)])
+def test_restrict(sf, oracle, fine):
+    nz, ny, nx = fine
+    coeffs = I.random_coeffs(nx, ny, nz, 6)
+    F = make_level(sf, fine, coeffs)
+    C = sf.Level(nx // 2, ny // 2, nz // 2)
+    x = I.random_field(fine, 2)
+    F.upload(sf.SF_R, x)
+    sf.sf_restrict(C.handle, sf.SF_F, F.handle, sf.SF_R, sf.SF_RESTRICT_CELL)
+    assert np.array_equal(C.download(sf.SF_F), oracle.restrict_cell(x))
+    for kind, fid, arr in [(sf.SF_RESTRICT_FACE_I, sf.SF_BETA_I, coeffs[1]),
+                           (sf.SF_RESTRICT_FACE_J, sf.SF_BETA_J, coeffs[2]),
+                           (sf.SF_RESTRICT_FACE_K, sf.SF_BETA_K, coeffs[3])]:
+        sf.sf_restrict(C.handle, fid, F.handle, fid, kind)
+        name = {sf.SF_BETA_I: "beta_i", sf.SF_BETA_J: "beta_j", sf.SF_BETA_K: "beta_k"}[fid]
+        assert np.array_equal(C.download(fid), oracle.restrict_face(arr, name))
+
+
+@pytest.mark.parametrize("fine", [(8, 8, 8), (16, 12, 20), (32, 32, 64)])
+@pytest.mark.parametrize("kind", ["p0", "pl"])
+@pytest.mark.parametrize("s", [0.0, 1.0, 0.5])
+def test_interpolate(sf, oracle, fine, kind, s):
+    nz, ny, nx = fine
+    F = make_level(sf, fine, I.random_coeffs(nx, ny, nz, 6))
+    C = sf.Level(nx // 2, ny // 2, nz // 2)
+    y = I.random_field(fine, 1)
+    c = I.random_field((nz // 2, ny // 2, nx // 2), 2)
+    F.upload(sf.SF_U, y)
+    C.upload(sf.SF_U, c)
+    k = sf.SF_INTERP_P0 if kind == "p0" else sf.SF_INTERP_PL
+    sf.sf_interpolate(F.handle, sf.SF_U, s, C.handle, sf.SF_U, k)
+    exp = oracle.interpolate(y, c, s, kind)
+    assert rel(F.download(sf.SF_U), exp) < 1e-15
+
+
+def test_norms(sf, oracle):
+    shape = (20, 24, 64)
+    nz, ny, nx = shape
+    L = make_level(sf, shape, I.random_coeffs(nx, ny, nz, 1))
+    x = I.random_field(shape, 9)
+    L.upload(sf.SF_R, x)
+    assert sf.sf_norm(L.handle, sf.SF_R, sf.SF_NORM_MAX) == oracle.norm(x, "max")
+    assert abs(sf.sf_norm(L.handle, sf.SF_R, sf.SF_NORM_L2) / oracle.norm(x, "l2") - 1) < 1e-13
+    x[3, 4, 5] = np.nan
+    L.upload(sf.SF_R, x)
+    assert np.isnan(sf.sf_norm(L.handle, sf.SF_R, sf.SF_NORM_MAX))
+
+
+def test_init_problem_matches_input_generator(sf):
+    for (nz, ny, nx) in [(16, 16, 16), (64, 32, 32)]:
+        L = sf.Level(nx, ny, nz)
+        sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
+        h = I.level_h(nx, ny, nz)
+        al, bi, bj, bk = I.hpgmg_coeffs(nx, ny, nz, h)
+        _, f = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
+        for fid, arr in [(sf.SF_ALPHA, al), (sf.SF_BETA_I, bi), (sf.SF_BETA_J, bj),
+                         (sf.SF_BETA_K, bk), (sf.SF_F, f)]:
+            assert rel(L.download(fid), arr) < 1e-14
+
+
+# ------------------------------------------------------------------ multigrid
+def mg_pair(sf, oracle, n, shape=None, parts=1, cc=False, **opts):
+    shape = shape or (n, n, n)
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.constant_coeffs(nx, ny, nz) if cc else I.hpgmg_coeffs(nx, ny, nz, h)
+    L = make_level(sf, shape, coeffs, parts=parts, h=h)
+    M = sf.MG(L, 1.0, 1.0, **opts)
+    O = oracle.MG(nx, ny, nz, h, 1.0, 1.0, *coeffs)
+    return L, M, O
+
+
+@pytest.mark.parametrize("n", [4, 16, 32, 64])
+def test_vcycle_parity(sf, oracle, n):
+    L, M, O = mg_pair(sf, oracle, n)
+    assert M.num_levels == O.levels
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    u = np.zeros((n, n, n))
+    L.upload(sf.SF_F, f)
+    for _ in range(2):
+        M.vcycle(0)
+        u = O.vcycle(u, f)
+        assert rel(L.download(sf.SF_U), u) < 1e-11
+
+
+def test_fcycle_parity(sf, oracle):
+    n = 32
+    L, M, O = mg_pair(sf, oracle, n)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    M.fcycle()
+    assert rel(L.download(sf.SF_U), O.fcycle(f)) < 1e-11
+
+
+@pytest.mark.parametrize("fcycle", [False, True])
+def test_c2_solve_parity(sf, oracle, fcycle):
+    """BASELINE config 2: 64^3 VC Helmholtz solved to 1e-10; same cycle count
+    as the oracle and u within 1e-10 relative L2."""
+    n = 64
+    L, M, O = mg_pair(sf, oracle, n)
+    ue, f = I.manufactured(n, n, n, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    st, cyc, hist = M.solve(fcycle=fcycle, rtol=1e-10)
+    u_o, hist_o = O.solve(f, fcycle=fcycle, rtol=1e-10)
+    u = L.download(sf.SF_U)
+    assert cyc == len(hist_o)
+    assert hist[-1] < 1e-10
+    assert rel(u, u_o) < 1e-10
+    assert abs(np.abs(u - ue).max() - 5.19e-7) < 0.05e-6
+
+
+def test_solve_graph_replay_stable(sf, oracle):
+    """Repeated solves through the captured CUDA graphs give identical results."""
+    n = 32
+    L, M, O = mg_pair(sf, oracle, n)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    res = []
+    for _ in range(3):
+        L.upload(sf.SF_U, np.zeros((n, n, n)))
+        L.upload(sf.SF_F, f)
+        st, cyc, hist = M.solve(fcycle=True)
+        res.append(L.download(sf.SF_U))
+    assert np.array_equal(res[0], res[1]) and np.array_equal(res[1], res[2])
+
+
+# ------------------------------------------------------- decomposition (loopback)
+@pytest.mark.parametrize("parts", [2, 4])
+def test_decomposition_invariance_smoother(sf, parts):
+    shape = (32, 16, 64)
+    nz, ny, nx = shape
+    coeffs = I.hpgmg_coeffs(nx, ny, nz)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    out = {}
+    for P in (1, parts):
+        for kind in (sf.SF_SMOOTH_COLOUR, sf.SF_SMOOTH_FUSED):
+            L = make_level(sf, shape, coeffs, parts=P)
+            sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+            L.upload(sf.SF_U, x)
+            L.upload(sf.SF_F, f)
+            sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, kind)
+            sf.sf_residual(L.handle, sf.SF_R, sf.SF_U, sf.SF_F, 1.0, 1.0)
+            out[(P, kind)] = (L.download(sf.SF_U), L.download(sf.SF_R))
+    for kind in (sf.SF_SMOOTH_COLOUR, sf.SF_SMOOTH_FUSED):
+        assert np.array_equal(out[(1, kind)][0], out[(parts, kind)][0])
+        assert np.array_equal(out[(1, kind)][1], out[(parts, kind)][1])
+
+
+@pytest.mark.parametrize("parts", [2, 4])
+def test_decomposition_invariance_solve(sf, oracle, parts):
+    n = 64
+    shape = (n, n, n)
+    res = {}
+    for P in (1, parts):
+        L, M, O = mg_pair(sf, oracle, n, parts=P, agglom_min_planes=4)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        st, cyc, hist = M.solve(fcycle=True)
+        res[P] = (L.download(sf.SF_U), cyc)
+    assert res[1][1] == res[parts][1]
+    assert rel(res[parts][0], res[1][0]) < 1e-13
+
+
+# ------------------------------------------------------- full-size (BASELINE C3)
+def test_c3_full_size_gsrb_pair(sf, oracle):
+    """256^3 HPGMG-shaped level, the fused pair bench.py times, element by
+    element against the oracle (one pair: a few seconds on the host)."""
+    n = 256
+    shape = (n, n, n)
+    coeffs = I.hpgmg_coeffs(n, n, n)
+    L = make_level(sf, shape, coeffs)
+    sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED)
+    got = L.download(sf.SF_U)
+    P = oracle.Problem(oracle.Grid(n, n, n, 1.0 / n), 1.0, 1.0, *coeffs)
+    assert rel(got, P.smooth(x, f, 1)) < TOL

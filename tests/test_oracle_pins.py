@@ -396,3 +396,19 @@ def test_paper_constants_fixture():
     # 64 B = x read + x write + rhs, alpha, beta_i, beta_j, beta_k, lambda (8 B each)
     assert 8 * (2 + 6) == g["compulsory_bytes_per_stencil"]["vc_gsrb"]
     assert g["hpgmg_run"]["smooths_pre_post_sweeps"] == 4
+
+
+def test_point_evaluations_match_whole_grid(oracle):
+    """The sampled (one cell at a time) oracle evaluations used at full size
+    equal the whole-grid oracle sweeps they restate."""
+    nx, ny, nz = 8, 6, 10
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, 0.1), 1.0, 1.0, *I.random_coeffs(nx, ny, nz, 4))
+    x = I.random_field((nz, ny, nx), 0)
+    f = I.random_field((nz, ny, nx), 1)
+    rng = np.random.default_rng(3)
+    pts = (rng.integers(0, nx, 40), rng.integers(0, ny, 40), rng.integers(0, nz, 40))
+    pts = (np.r_[pts[0], 0, nx - 1, 0], np.r_[pts[1], 0, ny - 1, ny - 1], np.r_[pts[2], 0, nz - 1, 1])
+    r = P.residual(x, f)
+    assert np.array_equal(P.residual_points(x, f, pts), r[pts[2], pts[1], pts[0]])
+    s = P.smooth(x, f, 1)
+    assert np.array_equal(P.gsrb_pair_points(x, f, pts), s[pts[2], pts[1], pts[0]])
