@@ -34,6 +34,8 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
+#include <cstdlib>
+
 #include "sf_internal.h"
 
 namespace {
@@ -112,9 +114,121 @@ struct Geo {
     long js, ks;
 };
 
-__global__ void __launch_bounds__(NT, 1)
+// Per-step state shared by the templated step bodies.
+struct StepCtx {
+    const double* Xk;   // x(p)      (written: red-new of plane p)
+    const double* Xm;   // x(p-1)
+    const double* Xp;   // x(p+1)
+    const double* Xmm;  // x(p-2)
+    const double* C;    // coefficients of plane p
+    const double* Klo;  // beta_k(p)
+    const double* Khi;  // beta_k(p+1)
+};
+
+// R(p) for the pair at smem offsets (xo_: x box, co_: coef box).  SEL = 1 if
+// the odd cell of the pair is red at this plane (warp-uniform).  Returns the
+// red-new value; leaves the black cell's coefficients of plane p in nb.
+template <int SEL>
+__device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
+                                           int gy, const Geo& g, bool zlo, bool zhi, double a,
+                                           double bh2, double* nb) {
+    double2 xp2 = *(const double2*)&s.Xk[xo_];
+    double2 al2 = *(const double2*)&s.C[CA_AL * CARR + co_];
+    double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
+    double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
+    double2 bi2 = *(const double2*)&s.C[CA_BI * CARR + co_];
+    double2 bjl = *(const double2*)&s.C[CA_BJ * CARR + co_];
+    double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
+    double2 bkl = *(const double2*)&s.Klo[co_];
+    double2 bkh = *(const double2*)&s.Khi[co_];
+    double bie = __shfl_down_sync(0xffffffffu, bi2.x, 1);
+    if (lane == 31) bie = s.C[CA_BI * CARR + co_ + 2];
+    double xc, xw, xe;
+    if (SEL == 0) {
+        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1);
+        if (lane == 0) xl = s.Xk[xo_ - 1];
+        xc = xp2.x; xw = xl; xe = xp2.y;
+    } else {
+        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1);
+        if (lane == 31) xr = s.Xk[xo_ + 2];
+        xc = xp2.y; xw = xp2.x; xe = xr;
+    }
+    const int gxr = gx + SEL;
+    if (gxr == 0) xw = -xc;
+    if (gxr == g.nx - 1) xe = -xc;
+    const int col = xo_ + SEL;
+    double xs = (gy == 0) ? -xc : s.Xk[col - W];
+    double xn = (gy == g.ny - 1) ? -xc : s.Xk[col + W];
+    double xb = zlo ? -xc : s.Xm[col];
+    double xt = zhi ? -xc : s.Xp[col];
+    double r;
+    if (SEL == 0) {
+        r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x, al2.x,
+                      dv2.x, rh2.x, a, bh2);
+        nb[0] = bi2.y; nb[1] = bie; nb[2] = bjl.y; nb[3] = bjh.y; nb[4] = bkl.y; nb[5] = bkh.y;
+        nb[6] = al2.y; nb[7] = dv2.y; nb[8] = rh2.y;
+    } else {
+        r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y, al2.y,
+                      dv2.y, rh2.y, a, bh2);
+        nb[0] = bi2.x; nb[1] = bi2.y; nb[2] = bjl.x; nb[3] = bjh.x; nb[4] = bkl.x; nb[5] = bkh.x;
+        nb[6] = al2.x; nb[7] = dv2.x; nb[8] = rh2.x;
+    }
+    return r;
+}
+
+// B(p-1) for the pair; the black cell of plane p-1 sits at the same pair
+// position as the red cell of plane p (SEL).  Returns the output pair.
+template <int SEL>
+__device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int lane, int gx, int gy,
+                                              const Geo& g, int gkm, double a, double bh2,
+                                              const double* rb) {
+    double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
+    double xc, xw, xe;
+    if (SEL == 0) {
+        double ql = __shfl_up_sync(0xffffffffu, q2.y, 1);
+        if (lane == 0) ql = s.Xm[xo_ - 1];
+        xc = q2.x; xw = ql; xe = q2.y;
+    } else {
+        double qr = __shfl_down_sync(0xffffffffu, q2.x, 1);
+        if (lane == 31) qr = s.Xm[xo_ + 2];
+        xc = q2.y; xw = q2.x; xe = qr;
+    }
+    const int gxb = gx + SEL;
+    if (gxb == 0) xw = -xc;
+    if (gxb == g.nx - 1) xe = -xc;
+    const int col = xo_ + SEL;
+    double xs = (gy == 0) ? -xc : s.Xm[col - W];
+    double xn = (gy == g.ny - 1) ? -xc : s.Xm[col + W];
+    double xb = (gkm == 0) ? -xc : s.Xmm[col];
+    double xt = (gkm == g.gnz - 1) ? -xc : s.Xk[col];
+    double bnew = gs_update(xc, xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5],
+                            rb[6], rb[7], rb[8], a, bh2);
+    return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
+}
+
+// Ring red cell at smem offsets (xo_, co_) (scalar loads; bounds in flags)
+__device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, int flags, double a,
+                                           double bh2, bool zlo, bool zhi) {
+    double xc = s.Xk[xo_];
+    double xw = (flags & 1) ? -xc : s.Xk[xo_ - 1];
+    double xe = (flags & 2) ? -xc : s.Xk[xo_ + 1];
+    double xs = (flags & 4) ? -xc : s.Xk[xo_ - W];
+    double xn = (flags & 8) ? -xc : s.Xk[xo_ + W];
+    double xb = zlo ? -xc : s.Xm[xo_];
+    double xt = zhi ? -xc : s.Xp[xo_];
+    return gs_update(xc, xw, xe, xs, xn, xb, xt, s.C[CA_BI * CARR + co_],
+                     s.C[CA_BI * CARR + co_ + 1], s.C[CA_BJ * CARR + co_],
+                     s.C[CA_BJ * CARR + co_ + W], s.Klo[co_], s.Khi[co_],
+                     s.C[CA_AL * CARR + co_], s.C[CA_DV * CARR + co_], s.C[CA_RH * CARR + co_],
+                     a, bh2);
+}
+
+template <int RPW>
+__global__ void __launch_bounds__(32 * TY / RPW, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems) {
+    constexpr int NWARP = TY / RPW;
+    constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
     double* Cs = Xs + NXS * XSLOT;                    // [NCS][NCA][CHH][W]
@@ -139,8 +253,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
 
         // bundle p: x(p+1), alpha/Dinv/rhs/beta_i/beta_j (p), beta_k(p+1)
         auto issue = [&](int p) {
-            unsigned s = seq0 + 2 + (p - z0);
-            unsigned long long* b = &mbar[s % NMB];
+            unsigned sq = seq0 + 2 + (p - z0);
+            unsigned long long* b = &mbar[sq % NMB];
             mbar_expect(b, BUNDLE_BYTES);
             tma3(Xs + md(p + 1, NXS) * XSLOT, &mp.x, cx, cyx, p + 1 + SF_GZ, b);
             double* c = Cs + md(p, NCS) * CSLOT;
@@ -161,145 +275,127 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             issue(z0 - 1);
             if (z0 <= z1) issue(z0);
         }
-        mbar_wait(&mbar[seq0 % NMB], (seq0 / NMB) & 1);
 
-        // this thread's pair: row gy, cells gxa (x even) and gxa+1
-        const int gy = y0 + w, gxa = x0 + 2 * lane;
-        const int xr = w + 2, cr = w + 1, c0 = 2 * lane + 2;
-        double rb[9];  // black-cell coefficients of the previous plane (for B)
+        // this thread's pairs: rows y0 + w + r*NWARP, cells gxa (even) and gxa+1
+        const int gxa = x0 + 2 * lane;
+        int xoff[RPW], coff[RPW], gyr[RPW];
 #pragma unroll
-        for (int i = 0; i < 9; i++) rb[i] = 0.0;
-
-        for (int p = z0 - 1; p <= z1; p++) {
-            const unsigned s = seq0 + 2 + (p - z0);
-            mbar_wait(&mbar[s % NMB], (s / NMB) & 1);
-            const int gk = g.z0 + p;
-            const bool kin = gk >= 0 && gk < g.gnz;
-            const bool zlo = gk == 0, zhi = gk == g.gnz - 1;
-            const double* Xk = Xs + md(p, NXS) * XSLOT;
-            const double* Xm = Xs + md(p - 1, NXS) * XSLOT;
-            const double* Xp = Xs + md(p + 1, NXS) * XSLOT;
-            const double* C = Cs + md(p, NCS) * CSLOT;
-            const double* Klo = Ks + md(p, NKS) * CARR;
-            const double* Khi = Ks + md(p + 1, NKS) * CARR;
-
-            // ------------------------------------------------ R(p): tile
-            const int sel = (gy + gk) & 1;  // 1: the red cell is the odd one (b)
-            double2 xp2 = *(const double2*)&Xk[xr * W + c0];
-            double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1);
-            double xr_ = __shfl_down_sync(0xffffffffu, xp2.x, 1);
-            if (lane == 0) xl = Xk[xr * W + 1];
-            if (lane == 31) xr_ = Xk[xr * W + TX + 2];
-            double2 al2 = *(const double2*)&C[CA_AL * CARR + cr * W + c0];
-            double2 dv2 = *(const double2*)&C[CA_DV * CARR + cr * W + c0];
-            double2 rh2 = *(const double2*)&C[CA_RH * CARR + cr * W + c0];
-            double2 bi2 = *(const double2*)&C[CA_BI * CARR + cr * W + c0];
-            double bie = __shfl_down_sync(0xffffffffu, bi2.x, 1);
-            if (lane == 31) bie = C[CA_BI * CARR + cr * W + TX + 2];
-            double2 bjl = *(const double2*)&C[CA_BJ * CARR + cr * W + c0];
-            double2 bjh = *(const double2*)&C[CA_BJ * CARR + (cr + 1) * W + c0];
-            double2 bkl = *(const double2*)&Klo[cr * W + c0];
-            double2 bkh = *(const double2*)&Khi[cr * W + c0];
-            double rnew = 0.0;
-            if (kin) {
-                const int gx = gxa + sel, col = c0 + sel;
-                double xc = sel ? xp2.y : xp2.x;
-                double xw = sel ? xp2.x : xl;
-                double xe = sel ? xr_ : xp2.y;
-                if (gx == 0) xw = -xc;
-                if (gx == g.nx - 1) xe = -xc;
-                double xs = (gy == 0) ? -xc : Xk[(xr - 1) * W + col];
-                double xn = (gy == g.ny - 1) ? -xc : Xk[(xr + 1) * W + col];
-                double xb = zlo ? -xc : Xm[xr * W + col];
-                double xt = zhi ? -xc : Xp[xr * W + col];
-                rnew = gs_update(xc, xw, xe, xs, xn, xb, xt, sel ? bi2.y : bi2.x,
-                                 sel ? bie : bi2.y, sel ? bjl.y : bjl.x, sel ? bjh.y : bjh.x,
-                                 sel ? bkl.y : bkl.x, sel ? bkh.y : bkh.x, sel ? al2.y : al2.x,
-                                 sel ? dv2.y : dv2.x, sel ? rh2.y : rh2.x, a, bh2);
-            }
-            // black cell of this plane = the other one; keep its coefficients
-            double nb[9] = {sel ? bi2.x : bi2.y, sel ? bi2.y : bie, sel ? bjl.x : bjl.y,
-                            sel ? bjh.x : bjh.y, sel ? bkl.x : bkl.y, sel ? bkh.x : bkh.y,
-                            sel ? al2.x : al2.y, sel ? dv2.x : dv2.y, sel ? rh2.x : rh2.y};
-
-            // ------------------------------------------------ R(p): ring (9 per warp)
-            int rt = w * 9 + lane;
-            bool ring = kin && lane < 9 && rt < NRING;
-            int rgx = 0, rgy = 0, rxr = 0, rcol = 0;
-            if (ring) {
+        for (int r = 0; r < RPW; r++) {
+            int row = w + r * NWARP;
+            gyr[r] = y0 + row;
+            xoff[r] = (row + 2) * W + 2 * lane + 2;
+            coff[r] = (row + 1) * W + 2 * lane + 2;
+        }
+        // ring cell of this thread for both parities of gk (offsets + BC flags)
+        int rxo[2], rco[2], rfl[2];
+        bool rok[2];
+        {
+            const int rt = w * RING_PER_WARP + lane;
+#pragma unroll
+            for (int par = 0; par < 2; par++) {
+                int rgx = 0, rgy = 0;
+                bool ok = lane < RING_PER_WARP && rt < NRING;
                 if (rt < TX) {
                     int pp = rt % (TX / 2);
                     rgy = (rt < TX / 2) ? y0 - 1 : y0 + TY;
-                    int s2 = (rgy + gk) & 1;
-                    rgx = x0 + 2 * pp + s2;
+                    rgx = x0 + 2 * pp + ((rgy + par) & 1);
                 } else {
                     int m = rt - TX, side = m / (TY / 2);
                     m -= side * (TY / 2);
                     rgx = side ? x0 + TX : x0 - 1;
                     int gyp = y0 + 2 * m;
-                    rgy = gyp + ((rgx + gyp + gk) & 1);
+                    rgy = gyp + ((rgx + gyp + par) & 1);
                 }
-                ring = rgx >= 0 && rgx < g.nx && rgy >= 0 && rgy < g.ny;
-                rxr = rgy - y0 + 2;
-                rcol = rgx - x0 + 2;
+                ok = ok && rgx >= 0 && rgx < g.nx && rgy >= 0 && rgy < g.ny;
+                rok[par] = ok;
+                rxo[par] = (rgy - y0 + 2) * W + rgx - x0 + 2;
+                rco[par] = (rgy - y0 + 1) * W + rgx - x0 + 2;
+                rfl[par] = (rgx == 0) | ((rgx == g.nx - 1) << 1) | ((rgy == 0) << 2) |
+                           ((rgy == g.ny - 1) << 3);
             }
-            double ringnew = 0.0;
-            if (ring) {
-                const int rcr = rxr - 1;
-                double xc = Xk[rxr * W + rcol];
-                double xw = (rgx == 0) ? -xc : Xk[rxr * W + rcol - 1];
-                double xe = (rgx == g.nx - 1) ? -xc : Xk[rxr * W + rcol + 1];
-                double xs = (rgy == 0) ? -xc : Xk[(rxr - 1) * W + rcol];
-                double xn = (rgy == g.ny - 1) ? -xc : Xk[(rxr + 1) * W + rcol];
-                double xb = zlo ? -xc : Xm[rxr * W + rcol];
-                double xt = zhi ? -xc : Xp[rxr * W + rcol];
-                ringnew = gs_update(xc, xw, xe, xs, xn, xb, xt, C[CA_BI * CARR + rcr * W + rcol],
-                                    C[CA_BI * CARR + rcr * W + rcol + 1],
-                                    C[CA_BJ * CARR + rcr * W + rcol],
-                                    C[CA_BJ * CARR + (rcr + 1) * W + rcol], Klo[rcr * W + rcol],
-                                    Khi[rcr * W + rcol], C[CA_AL * CARR + rcr * W + rcol],
-                                    C[CA_DV * CARR + rcr * W + rcol],
-                                    C[CA_RH * CARR + rcr * W + rcol], a, bh2);
+        }
+        double rb[RPW][9];
+#pragma unroll
+        for (int r = 0; r < RPW; r++)
+#pragma unroll
+            for (int i = 0; i < 9; i++) rb[r][i] = 0.0;
+
+        // rotating slot indices (no modulo in the loop)
+        int ixmm = md(z0 - 3, NXS), ixm = md(z0 - 2, NXS), ix = md(z0 - 1, NXS),
+            ixp = md(z0, NXS);
+        int ic = md(z0 - 1, NCS);
+        int iklo = md(z0 - 1, NKS), ikhi = md(z0, NKS);
+        mbar_wait(&mbar[seq0 % NMB], (seq0 / NMB) & 1);
+
+        for (int p = z0 - 1; p <= z1; p++) {
+            const unsigned sq = seq0 + 2 + (p - z0);
+            mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
+            const int gk = g.z0 + p;
+            const bool kin = gk >= 0 && gk < g.gnz;
+            const bool zlo = gk == 0, zhi = gk == g.gnz - 1;
+            StepCtx s;
+            s.Xk = Xs + ix * XSLOT;
+            s.Xm = Xs + ixm * XSLOT;
+            s.Xp = Xs + ixp * XSLOT;
+            s.Xmm = Xs + ixmm * XSLOT;
+            s.C = Cs + ic * CSLOT;
+            s.Klo = Ks + iklo * CARR;
+            s.Khi = Ks + ikhi * CARR;
+            double* Xkw = Xs + ix * XSLOT;
+            const int par = gk & 1;
+            const int sel = (y0 + w + gk) & 1;  // same for all RPW rows (rows differ by NWARP, even)
+
+            double nb[RPW][9];
+            if (kin) {
+                double rn[RPW];
+                if (sel == 0) {
+#pragma unroll
+                    for (int r = 0; r < RPW; r++)
+                        rn[r] = red_pair<0>(s, xoff[r], coff[r], lane, gxa, gyr[r], g, zlo, zhi,
+                                            a, bh2, nb[r]);
+                } else {
+#pragma unroll
+                    for (int r = 0; r < RPW; r++)
+                        rn[r] = red_pair<1>(s, xoff[r], coff[r], lane, gxa, gyr[r], g, zlo, zhi,
+                                            a, bh2, nb[r]);
+                }
+                double rr = 0.0;
+                const bool ring = par ? rok[1] : rok[0];
+                const int ro = par ? rxo[1] : rxo[0];
+                if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], a, bh2,
+                                        zlo, zhi);
+                // R(p) reads only black cells of plane p (and cells of planes
+                // p+-1 that are black there): writing red cells now is safe.
+#pragma unroll
+                for (int r = 0; r < RPW; r++) Xkw[xoff[r] + sel] = rn[r];
+                if (ring) Xkw[ro] = rr;
             }
-            // R(p) reads only black cells of plane p (and planes p+-1 at
-            // positions that are black there), so writing red cells now is safe.
-            double* Xkw = Xs + md(p, NXS) * XSLOT;
-            if (kin) Xkw[xr * W + c0 + sel] = rnew;
-            if (ring) Xkw[rxr * W + rcol] = ringnew;
             fence_proxy_async();
             __syncthreads();
 
             // refill: bundle p+2 (its slots were last read by B(p-2), before this barrier)
             if (tid == 0 && p + 2 <= z1) issue(p + 2);
 
-            // ------------------------------------------------ B(p-1): tile
+            // ------------------------------------------------ B(p-1)
             if (p - 1 >= z0) {
                 const int gkm = gk - 1;
-                const double* Xmm = Xs + md(p - 2, NXS) * XSLOT;
-                const int bsel = 1 - ((gy + gkm) & 1);  // black cell of plane p-1
-                double2 q2 = *(const double2*)&Xm[xr * W + c0];  // (red-new, black-old) pair
-                double ql = __shfl_up_sync(0xffffffffu, q2.y, 1);
-                double qr = __shfl_down_sync(0xffffffffu, q2.x, 1);
-                if (lane == 0) ql = Xm[xr * W + 1];
-                if (lane == 31) qr = Xm[xr * W + TX + 2];
-                const int gx = gxa + bsel, col = c0 + bsel;
-                double xc = bsel ? q2.y : q2.x;
-                double xw = bsel ? q2.x : ql;
-                double xe = bsel ? qr : q2.y;
-                if (gx == 0) xw = -xc;
-                if (gx == g.nx - 1) xe = -xc;
-                double xs = (gy == 0) ? -xc : Xm[(xr - 1) * W + col];
-                double xn = (gy == g.ny - 1) ? -xc : Xm[(xr + 1) * W + col];
-                double xb = (gkm == 0) ? -xc : Xmm[xr * W + col];
-                double xt = (gkm == g.gnz - 1) ? -xc : Xk[xr * W + col];
-                double bnew = gs_update(xc, xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3],
-                                        rb[4], rb[5], rb[6], rb[7], rb[8], a, bh2);
-                double2 o = bsel ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
-                *(double2*)(xo + (long)(p - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
-                            SF_OX + gxa) = o;
+#pragma unroll
+                for (int r = 0; r < RPW; r++) {
+                    double2 o = (sel == 0)
+                                    ? black_pair<0>(s, xoff[r], lane, gxa, gyr[r], g, gkm, a, bh2, rb[r])
+                                    : black_pair<1>(s, xoff[r], lane, gxa, gyr[r], g, gkm, a, bh2, rb[r]);
+                    *(double2*)(xo + (long)(p - 1 + SF_GZ) * g.ks + (long)(gyr[r] + SF_GY) * g.js +
+                                SF_OX + gxa) = o;
+                }
             }
 #pragma unroll
-            for (int i = 0; i < 9; i++) rb[i] = nb[i];
+            for (int r = 0; r < RPW; r++)
+#pragma unroll
+                for (int i = 0; i < 9; i++) rb[r][i] = nb[r][i];
+            // rotate slots
+            ixmm = ixm; ixm = ix; ix = ixp; ixp = (ixp + 1 == NXS) ? 0 : ixp + 1;
+            ic = (ic + 1 == NCS) ? 0 : ic + 1;
+            iklo = ikhi; ikhi = (ikhi + 1 == NKS) ? 0 : ikhi + 1;
         }
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
@@ -347,8 +443,8 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
     SF_TRY(get_encoder());
     static bool attr = false;
     if (!attr) {
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)SMEM));
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<1>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
         SF_CUDA(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
@@ -383,8 +479,8 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
         int grid = std::min(items, G);
-        gsrb_pair_tma_kernel<<<grid, NT, SMEM, L->stream>>>(mp, g, v.f[xout], a, bh2, depth, ntx,
-                                                            tiles, items);
+        gsrb_pair_tma_kernel<1><<<grid, NT, SMEM, L->stream>>>(mp, g, v.f[xout], a, bh2, depth,
+                                                               ntx, tiles, items);
         SF_LAUNCHED();
     }
     return sf_check_launch("gsrb_pair_tma");
