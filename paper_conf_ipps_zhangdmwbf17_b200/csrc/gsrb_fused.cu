@@ -46,7 +46,7 @@ constexpr int NT = 32 * TY;            // 256 threads
 constexpr int W = TX + 4;              // smem row: gx in [x0-2, x0+TX+2)
 constexpr int XH = TY + 4;             // x rows:   gy in [y0-2, y0+TY+2)
 constexpr int CHH = TY + 3;            // coef rows: gy in [y0-1, y0+TY+2)
-constexpr int NXS = 6, NCS = 4, NKS = 5, NMB = 4;  // slot counts
+constexpr int NXS = 7, NCS = 3, NKS = 4, NMB = 4;  // slot counts
 constexpr int NCA = 5;                 // staged coefficient arrays per plane (beta_k separate)
 constexpr int XSLOT = XH * W;          // doubles (6528 B = 51 x 128)
 constexpr int CARR = 752;              // 11*68 = 748 doubles padded to 128 B
@@ -176,8 +176,8 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     return r;
 }
 
-// B(p-1) for the pair; the black cell of plane p-1 sits at the same pair
-// position as the red cell of plane p (SEL).  Returns the output pair.
+// B for the pair; SEL = position (0: even x, 1: odd x) of the black cell in
+// the pair.  Returns the output pair (red-new, black-new in place).
 template <int SEL>
 __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int lane, int gx, int gy,
                                               const Geo& g, int gkm, double a, double bh2,
@@ -223,12 +223,17 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
                      a, bh2);
 }
 
-template <int RPW>
-__global__ void __launch_bounds__(32 * TY / RPW, 1)
+// Step t of the software pipeline: R(t+1) and B(t-1) are independent (R(t+1)
+// reads black-OLD cells of planes t..t+2, B(t-1) reads red-NEW cells of
+// planes t-2..t and writes only global memory), so each thread runs both
+// chains together (ILP 2) between two consecutive barriers.  The black cell's
+// coefficients of plane q are taken from the smem slot by R(q) at step q-1
+// and kept in registers until B(q) at step q+1 (stash alternates by step).
+__global__ void __launch_bounds__(NT, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems) {
-    constexpr int NWARP = TY / RPW;
-    constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;
+    constexpr int NWARP = TY;
+    constexpr int RING_PER_WARP = NRING / NWARP;   // 9
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
     double* Cs = Xs + NXS * XSLOT;                    // [NCS][NCA][CHH][W]
@@ -249,21 +254,21 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         const int z0 = chunk * depth, z1 = min(z0 + depth, g.nz);
         const int cx = SF_OX + x0 - 2;        // TMA x coordinate of the box
         const int cyx = y0, cyc = y0 + 1;     // TMA y coordinates (x box, coef box)
-        const unsigned seq0 = seq;            // pre-bundle; bundle p -> seq0 + 2 + p - z0
+        const unsigned seq0 = seq;            // pre-bundle; bundle q -> seq0 + 2 + q - z0
 
-        // bundle p: x(p+1), alpha/Dinv/rhs/beta_i/beta_j (p), beta_k(p+1)
-        auto issue = [&](int p) {
-            unsigned sq = seq0 + 2 + (p - z0);
+        // bundle q: x(q+1), alpha/Dinv/rhs/beta_i/beta_j (q), beta_k(q+1); needed by R(q)
+        auto issue = [&](int q) {
+            unsigned sq = seq0 + 2 + (q - z0);
             unsigned long long* b = &mbar[sq % NMB];
             mbar_expect(b, BUNDLE_BYTES);
-            tma3(Xs + md(p + 1, NXS) * XSLOT, &mp.x, cx, cyx, p + 1 + SF_GZ, b);
-            double* c = Cs + md(p, NCS) * CSLOT;
-            tma3(c + CA_AL * CARR, &mp.al, cx, cyc, p + SF_GZ, b);
-            tma3(c + CA_DV * CARR, &mp.dv, cx, cyc, p + SF_GZ, b);
-            tma3(c + CA_RH * CARR, &mp.rh, cx, cyc, p + SF_GZ, b);
-            tma3(c + CA_BI * CARR, &mp.bi, cx, cyc, p + SF_GZ, b);
-            tma3(c + CA_BJ * CARR, &mp.bj, cx, cyc, p + SF_GZ, b);
-            tma3(Ks + md(p + 1, NKS) * CARR, &mp.bk, cx, cyc, p + 1 + SF_GZ, b);
+            tma3(Xs + md(q + 1, NXS) * XSLOT, &mp.x, cx, cyx, q + 1 + SF_GZ, b);
+            double* c = Cs + md(q, NCS) * CSLOT;
+            tma3(c + CA_AL * CARR, &mp.al, cx, cyc, q + SF_GZ, b);
+            tma3(c + CA_DV * CARR, &mp.dv, cx, cyc, q + SF_GZ, b);
+            tma3(c + CA_RH * CARR, &mp.rh, cx, cyc, q + SF_GZ, b);
+            tma3(c + CA_BI * CARR, &mp.bi, cx, cyc, q + SF_GZ, b);
+            tma3(c + CA_BJ * CARR, &mp.bj, cx, cyc, q + SF_GZ, b);
+            tma3(Ks + md(q + 1, NKS) * CARR, &mp.bk, cx, cyc, q + 1 + SF_GZ, b);
         };
         if (tid == 0) {
             fence_proxy_async();  // generic smem writes of the previous item before TMA reuse
@@ -272,21 +277,14 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 2 + SF_GZ, b);
             tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 1 + SF_GZ, b);
             tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, z0 - 1 + SF_GZ, b);
-            issue(z0 - 1);
-            if (z0 <= z1) issue(z0);
+            for (int q = z0 - 1; q <= min(z0, z1); q++) issue(q);   // step t issues t+3
         }
 
-        // this thread's pairs: rows y0 + w + r*NWARP, cells gxa (even) and gxa+1
-        const int gxa = x0 + 2 * lane;
-        int xoff[RPW], coff[RPW], gyr[RPW];
-#pragma unroll
-        for (int r = 0; r < RPW; r++) {
-            int row = w + r * NWARP;
-            gyr[r] = y0 + row;
-            xoff[r] = (row + 2) * W + 2 * lane + 2;
-            coff[r] = (row + 1) * W + 2 * lane + 2;
-        }
-        // ring cell of this thread for both parities of gk (offsets + BC flags)
+        // this thread's pair: row gy, cells gxa (even) and gxa+1
+        const int gxa = x0 + 2 * lane, gy = y0 + w;
+        const int xoff = (w + 2) * W + 2 * lane + 2;
+        const int coff = (w + 1) * W + 2 * lane + 2;
+        // ring cell of this thread for both parities of the plane (offsets + BC flags)
         int rxo[2], rco[2], rfl[2];
         bool rok[2];
         {
@@ -294,7 +292,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
 #pragma unroll
             for (int par = 0; par < 2; par++) {
                 int rgx = 0, rgy = 0;
-                bool ok = lane < RING_PER_WARP && rt < NRING;
+                bool ok = lane < RING_PER_WARP;
                 if (rt < TX) {
                     int pp = rt % (TX / 2);
                     rgy = (rt < TX / 2) ? y0 - 1 : y0 + TY;
@@ -314,88 +312,81 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                            ((rgy == g.ny - 1) << 3);
             }
         }
-        double rb[RPW][9];
+        double stA[9], stB[9];
 #pragma unroll
-        for (int r = 0; r < RPW; r++)
-#pragma unroll
-            for (int i = 0; i < 9; i++) rb[r][i] = 0.0;
+        for (int i = 0; i < 9; i++) stA[i] = stB[i] = 0.0;
 
-        // rotating slot indices (no modulo in the loop)
-        int ixmm = md(z0 - 3, NXS), ixm = md(z0 - 2, NXS), ix = md(z0 - 1, NXS),
-            ixp = md(z0, NXS);
-        int ic = md(z0 - 1, NCS);
-        int iklo = md(z0 - 1, NKS), ikhi = md(z0, NKS);
+        // rotating slot indices for step t = z0-2: R(z0-1) / B(z0-3)
+        // x slots: x(t-2) .. x(t+2)
+        int ix_m2 = md(z0 - 4, NXS), ix_m1 = md(z0 - 3, NXS), ix_0 = md(z0 - 2, NXS),
+            ix_p1 = md(z0 - 1, NXS), ix_p2 = md(z0, NXS);
+        int ic = md(z0 - 1, NCS);                       // coef(t+1)
+        int ik1 = md(z0 - 1, NKS), ik2 = md(z0, NKS);   // beta_k(t+1), beta_k(t+2)
         mbar_wait(&mbar[seq0 % NMB], (seq0 / NMB) & 1);
 
-        for (int p = z0 - 1; p <= z1; p++) {
-            const unsigned sq = seq0 + 2 + (p - z0);
-            mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
-            const int gk = g.z0 + p;
-            const bool kin = gk >= 0 && gk < g.gnz;
-            const bool zlo = gk == 0, zhi = gk == g.gnz - 1;
-            StepCtx s;
-            s.Xk = Xs + ix * XSLOT;
-            s.Xm = Xs + ixm * XSLOT;
-            s.Xp = Xs + ixp * XSLOT;
-            s.Xmm = Xs + ixmm * XSLOT;
-            s.C = Cs + ic * CSLOT;
-            s.Klo = Ks + iklo * CARR;
-            s.Khi = Ks + ikhi * CARR;
-            double* Xkw = Xs + ix * XSLOT;
-            const int par = gk & 1;
-            const int sel = (y0 + w + gk) & 1;  // same for all RPW rows (rows differ by NWARP, even)
-
-            double nb[RPW][9];
-            if (kin) {
-                double rn[RPW];
-                if (sel == 0) {
-#pragma unroll
-                    for (int r = 0; r < RPW; r++)
-                        rn[r] = red_pair<0>(s, xoff[r], coff[r], lane, gxa, gyr[r], g, zlo, zhi,
-                                            a, bh2, nb[r]);
-                } else {
-#pragma unroll
-                    for (int r = 0; r < RPW; r++)
-                        rn[r] = red_pair<1>(s, xoff[r], coff[r], lane, gxa, gyr[r], g, zlo, zhi,
-                                            a, bh2, nb[r]);
-                }
-                double rr = 0.0;
-                const bool ring = par ? rok[1] : rok[0];
-                const int ro = par ? rxo[1] : rxo[0];
-                if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], a, bh2,
-                                        zlo, zhi);
-                // R(p) reads only black cells of plane p (and cells of planes
-                // p+-1 that are black there): writing red cells now is safe.
-#pragma unroll
-                for (int r = 0; r < RPW; r++) Xkw[xoff[r] + sel] = rn[r];
-                if (ring) Xkw[ro] = rr;
+        auto step = [&](int t, double* stash) {
+            // --- wait for bundle t+1 (R(t+1) operands)
+            const int q = t + 1;
+            if (q <= z1) {
+                const unsigned sq = seq0 + 2 + (q - z0);
+                mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
             }
+            const int gkr = g.z0 + q;                    // plane of R
+            const bool rin = q <= z1 && gkr >= 0 && gkr < g.gnz;
+            const bool bin = t - 1 >= z0;                // B(t-1) on the tile
+            const int sel = (y0 + w + gkr) & 1;          // same pair position for R and B
+            StepCtx s;                                   // centred on plane q = t+1 for R
+            s.Xk = Xs + ix_p1 * XSLOT;
+            s.Xm = Xs + ix_0 * XSLOT;
+            s.Xp = Xs + ix_p2 * XSLOT;
+            s.C = Cs + ic * CSLOT;
+            s.Klo = Ks + ik1 * CARR;
+            s.Khi = Ks + ik2 * CARR;
+            StepCtx sb;                                  // centred on plane t-1 for B
+            sb.Xk = Xs + ix_0 * XSLOT;                   // x(t)   (top neighbour)
+            sb.Xm = Xs + ix_m1 * XSLOT;                  // x(t-1) (the plane)
+            sb.Xmm = Xs + ix_m2 * XSLOT;                 // x(t-2) (bottom neighbour)
+            double nb[9];
+            double rn = 0.0;
+            double2 o = make_double2(0.0, 0.0);
+            const bool zlo = gkr == 0, zhi = gkr == g.gnz - 1;
+            const int gkm = g.z0 + t - 1;
+            // planes t+1 and t-1 have the same parity: the black cell of
+            // plane t-1 is the pair's other cell (position 1-sel)
+            if (sel == 0) {
+                if (rin) rn = red_pair<0>(s, xoff, coff, lane, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (bin) o = black_pair<1>(sb, xoff, lane, gxa, gy, g, gkm, a, bh2, stash);
+            } else {
+                if (rin) rn = red_pair<1>(s, xoff, coff, lane, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (bin) o = black_pair<0>(sb, xoff, lane, gxa, gy, g, gkm, a, bh2, stash);
+            }
+            const int par = gkr & 1;
+            const bool ring = rin && (par ? rok[1] : rok[0]);
+            const int ro = par ? rxo[1] : rxo[0];
+            double rr = 0.0;
+            if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], a, bh2, zlo, zhi);
+            double* Xw = Xs + ix_p1 * XSLOT;
+            if (rin) Xw[xoff + sel] = rn;
+            if (ring) Xw[ro] = rr;
+            if (bin)
+                *(double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
+                            SF_OX + gxa) = o;
+#pragma unroll
+            for (int i = 0; i < 9; i++) stash[i] = nb[i];
             fence_proxy_async();
             __syncthreads();
-
-            // refill: bundle p+2 (its slots were last read by B(p-2), before this barrier)
-            if (tid == 0 && p + 2 <= z1) issue(p + 2);
-
-            // ------------------------------------------------ B(p-1)
-            if (p - 1 >= z0) {
-                const int gkm = gk - 1;
-#pragma unroll
-                for (int r = 0; r < RPW; r++) {
-                    double2 o = (sel == 0)
-                                    ? black_pair<0>(s, xoff[r], lane, gxa, gyr[r], g, gkm, a, bh2, rb[r])
-                                    : black_pair<1>(s, xoff[r], lane, gxa, gyr[r], g, gkm, a, bh2, rb[r]);
-                    *(double2*)(xo + (long)(p - 1 + SF_GZ) * g.ks + (long)(gyr[r] + SF_GY) * g.js +
-                                SF_OX + gxa) = o;
-                }
-            }
-#pragma unroll
-            for (int r = 0; r < RPW; r++)
-#pragma unroll
-                for (int i = 0; i < 9; i++) rb[r][i] = nb[r][i];
+            // refill bundle t+3 (its slots were last read before this barrier)
+            if (tid == 0 && t + 3 <= z1) issue(t + 3);
             // rotate slots
-            ixmm = ixm; ixm = ix; ix = ixp; ixp = (ixp + 1 == NXS) ? 0 : ixp + 1;
+            ix_m2 = ix_m1; ix_m1 = ix_0; ix_0 = ix_p1; ix_p1 = ix_p2;
+            ix_p2 = (ix_p2 + 1 == NXS) ? 0 : ix_p2 + 1;
             ic = (ic + 1 == NCS) ? 0 : ic + 1;
-            iklo = ikhi; ikhi = (ikhi + 1 == NKS) ? 0 : ikhi + 1;
+            ik1 = ik2; ik2 = (ik2 + 1 == NKS) ? 0 : ik2 + 1;
+        };
+        // steps t = z0-2 .. z1; B(t-1) consumes the stash R(t-1) filled at step t-2
+        for (int t = z0 - 2; t <= z1; t += 2) {
+            step(t, stA);
+            if (t + 1 <= z1) step(t + 1, stB);
         }
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
@@ -443,7 +434,7 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
     SF_TRY(get_encoder());
     static bool attr = false;
     if (!attr) {
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<1>,
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
@@ -479,7 +470,7 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
         int grid = std::min(items, G);
-        gsrb_pair_tma_kernel<1><<<grid, NT, SMEM, L->stream>>>(mp, g, v.f[xout], a, bh2, depth,
+        gsrb_pair_tma_kernel<<<grid, NT, SMEM, L->stream>>>(mp, g, v.f[xout], a, bh2, depth,
                                                                ntx, tiles, items);
         SF_LAUNCHED();
     }
