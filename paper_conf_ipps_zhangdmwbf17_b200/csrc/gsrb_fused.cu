@@ -46,7 +46,8 @@ constexpr int NT = 32 * TY;            // 256 threads
 constexpr int W = TX + 4;              // smem row: gx in [x0-2, x0+TX+2)
 constexpr int XH = TY + 4;             // x rows:   gy in [y0-2, y0+TY+2)
 constexpr int CHH = TY + 3;            // coef rows: gy in [y0-1, y0+TY+2)
-constexpr int NXS = 7, NCS = 3, NKS = 4, NMB = 4;  // slot counts
+constexpr int PF = 3;                  // bundles in flight ahead of the one being consumed
+constexpr int NXS = 5 + PF, NCS = 1 + PF, NKS = 2 + PF, NMB = PF + 2;  // slot counts
 constexpr int NCA = 5;                 // staged coefficient arrays per plane (beta_k separate)
 constexpr int XSLOT = XH * W;          // doubles (6528 B = 51 x 128)
 constexpr int CARR = 752;              // 11*68 = 748 doubles padded to 128 B
@@ -277,7 +278,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 2 + SF_GZ, b);
             tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 1 + SF_GZ, b);
             tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, z0 - 1 + SF_GZ, b);
-            for (int q = z0 - 1; q <= min(z0, z1); q++) issue(q);   // step t issues t+3
+            for (int q = z0 - 1; q <= min(z0 + PF - 2, z1); q++) issue(q);  // step t: t+PF+1
         }
 
         // this thread's pair: row gy, cells gxa (even) and gxa+1
@@ -375,8 +376,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             for (int i = 0; i < 9; i++) stash[i] = nb[i];
             fence_proxy_async();
             __syncthreads();
-            // refill bundle t+3 (its slots were last read before this barrier)
-            if (tid == 0 && t + 3 <= z1) issue(t + 3);
+            // refill bundle t+PF+1 (its slots were last read before this barrier)
+            if (tid == 0 && t + PF + 1 <= z1) issue(t + PF + 1);
             // rotate slots
             ix_m2 = ix_m1; ix_m1 = ix_0; ix_0 = ix_p1; ix_p1 = ix_p2;
             ix_p2 = (ix_p2 + 1 == NXS) ? 0 : ix_p2 + 1;
