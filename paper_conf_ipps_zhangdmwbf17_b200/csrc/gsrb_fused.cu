@@ -456,6 +456,8 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
         double cost = rounds * (d + 3.0);
         if (cost < best - 1e-9) { best = cost; best_d = d; }
     }
+    const char* ed = getenv("SF_GSRB_DEPTH");   // tuning override
+    if (ed && atoi(ed) > 0) best_d = std::min(L->lnz, atoi(ed));
     const int depth = best_d, nch = (L->lnz + depth - 1) / depth;
     const int items = tiles * nch;
     const double bh2 = b / (L->h * L->h);
