@@ -18,7 +18,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 BUILD = os.path.join(PKG, "_build")
 LIB = os.path.join(PKG, "libsf.so")
-SOURCES = ["level.cu", "kernels.cu", "gsrb_fused.cu", "comm.cu", "mg.cu"]
+SOURCES = ["level.cu", "kernels.cu", "kernels_pair.cu", "gsrb_fused.cu", "comm.cu", "mg.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xptxas", "-v",

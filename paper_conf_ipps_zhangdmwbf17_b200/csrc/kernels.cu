@@ -382,6 +382,7 @@ sf_status k_apply_op(sf_level* L, int out, int x, double a, double b) {
 }
 
 sf_status k_residual(sf_level* L, int res, int x, int rhs, double a, double b) {
+    if (pair_ok(L)) return k_residual_pair(L, res, x, rhs, a, b, nullptr);
     double bh2 = b / (L->h * L->h);
     SF_TRY(sf_halo(L, x, 1));
     for (int p = 0; p < L->nlocal; p++) {
@@ -458,6 +459,7 @@ sf_status k_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind) {
 }
 
 sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind) {
+    if (kind == SF_INTERP_P0 && pair_ok(F)) return k_interp_p0_pair(F, ff, s, C, cf);
     bool rep = replicated_below(C, F);
     if (kind == SF_INTERP_PL) SF_TRY(k_bc(C, cf));
     for (int p = 0; p < F->nlocal; p++) {
@@ -476,6 +478,7 @@ sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind)
 }
 
 sf_status k_norm(sf_level* L, int field, int kind, double* dst) {
+    if (pair_ok(L)) return k_norm_pair(L, field, kind, dst);
     zero_scalar_kernel<<<1, 1, 0, L->stream>>>(dst);
     SF_LAUNCHED();
     for (int p = 0; p < L->nlocal; p++) {

@@ -1,0 +1,264 @@
+// Bandwidth-shaped per-level kernels (sm_100a, fp64): each thread owns a PAIR
+// of x-adjacent cells (16-byte loads/stores along the unit-stride axis) and
+// streams a chunk of z-planes, so a block issues one atomic per launch-chunk
+// instead of one per cell.  Rows A6 (+A10, +A7) and A8 of DESIGN.md.
+//
+//   residual_pair<WRITE, NORM>  res = rhs - A x; optionally
+//                               writes res and/or reduces max|res| (A10, the
+//                               convergence check of reading R-9) in the same
+//                               pass (48 B/cell when only the norm is needed)
+//   residual_restrict           coarse rhs = R_cell(rhs - A x) (A6 + A7 fused,
+//                               49 B per fine cell): the V-cycle's residual
+//                               never goes to HBM
+//   interp_p0_pair              fine += P0(coarse) (A8, V-cycle)
+//   norm_pair                   max|x| / sum x^2 of a field (A10)
+//
+// The operator is evaluated in exactly the term order of op_at (kernels.cu)
+// and the oracle; the Dirichlet fold reads -x(c) across global faces.
+#include "sf_internal.h"
+
+namespace {
+
+constexpr int PX = 32, PY = 4;  // threads per block: 32 pairs (64 cells) x 4 rows
+
+__device__ __forceinline__ double2 ld2(const double* p) { return *(const double2*)p; }
+
+// A x at the pair (i, i+1) of row j, plane k; c = sf_ix(i, j, k), i even.
+__device__ __forceinline__ void op_pair(const PV& v, const double* __restrict__ x, int i, int j,
+                                        int gk, long c, double a, double bh2, double& axa,
+                                        double& axb) {
+    const double2 xc = ld2(x + c);
+    double xw = (i == 0) ? -xc.x : x[c - 1];
+    double xe = (i + 1 == v.nx - 1) ? -xc.y : x[c + 2];
+    double2 xs = ld2(x + c - v.js), xn = ld2(x + c + v.js);
+    double2 xb = ld2(x + c - v.ks), xt = ld2(x + c + v.ks);
+    if (j == 0) xs = make_double2(-xc.x, -xc.y);
+    if (j == v.ny - 1) xn = make_double2(-xc.x, -xc.y);
+    if (gk == 0) xb = make_double2(-xc.x, -xc.y);
+    if (gk == v.gnz - 1) xt = make_double2(-xc.x, -xc.y);
+    const double2 bi = ld2(v.f[SF_BETA_I] + c);
+    const double bie = v.f[SF_BETA_I][c + 2];
+    const double2 bjs = ld2(v.f[SF_BETA_J] + c), bjn = ld2(v.f[SF_BETA_J] + c + v.js);
+    const double2 bkb = ld2(v.f[SF_BETA_K] + c), bkt = ld2(v.f[SF_BETA_K] + c + v.ks);
+    const double2 al = ld2(v.f[SF_ALPHA] + c);
+    double fa = bi.y * (xc.y - xc.x);
+    fa += bi.x * (xw - xc.x);
+    fa += bjn.x * (xn.x - xc.x);
+    fa += bjs.x * (xs.x - xc.x);
+    fa += bkt.x * (xt.x - xc.x);
+    fa += bkb.x * (xb.x - xc.x);
+    double fb = bie * (xe - xc.y);
+    fb += bi.y * (xc.x - xc.y);
+    fb += bjn.y * (xn.y - xc.y);
+    fb += bjs.y * (xs.y - xc.y);
+    fb += bkt.y * (xt.y - xc.y);
+    fb += bkb.y * (xb.y - xc.y);
+    axa = a * al.x * xc.x - bh2 * fa;
+    axb = a * al.y * xc.y - bh2 * fb;
+}
+
+__device__ __forceinline__ unsigned long long umax64(unsigned long long a, unsigned long long b) {
+    return a > b ? a : b;
+}
+
+// block-wide max of non-negative doubles via their bit patterns (NaN wins)
+__device__ __forceinline__ void block_max_atomic(unsigned long long m, double* out) {
+    __shared__ unsigned long long red[PX * PY / 32];
+    for (int o = 16; o > 0; o >>= 1) m = umax64(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const int t = threadIdx.y * PX + threadIdx.x;
+    if ((t & 31) == 0) red[t >> 5] = m;
+    __syncthreads();
+    if (t == 0) {
+        for (int wq = 1; wq < PX * PY / 32; wq++) m = umax64(m, red[wq]);
+        atomicMax((unsigned long long*)out, m);
+    }
+}
+
+__device__ __forceinline__ unsigned long long abits(double v) {
+    return (unsigned long long)__double_as_longlong(fabs(v));
+}
+
+template <bool WRITE, bool NORM>
+__global__ void __launch_bounds__(PX* PY) residual_pair_kernel(PV v, double* __restrict__ res,
+                                                                const double* __restrict__ x,
+                                                                const double* __restrict__ rhs,
+                                                                double a, double bh2, int depth,
+                                                                double* nout) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    unsigned long long m = 0ull;
+    if (i < v.nx && j < v.ny) {
+        for (int k = k0; k < k1; k++) {
+            const long c = sf_ix(v, i, j, k);
+            double axa, axb;
+            op_pair(v, x, i, j, v.z0 + k, c, a, bh2, axa, axb);
+            const double2 f = ld2(rhs + c);
+            const double ra = f.x - axa, rb = f.y - axb;
+            if (WRITE) *(double2*)(res + c) = make_double2(ra, rb);
+            if (NORM) m = umax64(m, umax64(abits(ra), abits(rb)));
+        }
+    }
+    if (NORM) block_max_atomic(m, nout);
+}
+
+// coarse(I,J,K) = 1/8 sum over the 8 children of (rhs - A x); thread per (I,J)
+__global__ void __launch_bounds__(PX* PY) residual_restrict_kernel(PV f, const double* __restrict__ x,
+                                                                    const double* __restrict__ rhs,
+                                                                    double a, double bh2, PV c,
+                                                                    double* __restrict__ cx,
+                                                                    int zoff, int depth) {
+    const int I = blockIdx.x * PX + threadIdx.x, J = blockIdx.y * PY + threadIdx.y;
+    const int K0 = blockIdx.z * depth, K1 = min(K0 + depth, f.nz / 2);
+    if (2 * I >= f.nx || 2 * J >= f.ny) return;
+    for (int K = K0; K < K1; K++) {
+        double s = 0.0;
+#pragma unroll
+        for (int d = 0; d < 2; d++)
+#pragma unroll
+            for (int bb = 0; bb < 2; bb++) {
+                const int j = 2 * J + bb, k = 2 * K + d;
+                const long q = sf_ix(f, 2 * I, j, k);
+                double axa, axb;
+                op_pair(f, x, 2 * I, j, f.z0 + k, q, a, bh2, axa, axb);
+                const double2 r = ld2(rhs + q);
+                s += r.x - axa;
+                s += r.y - axb;
+            }
+        cx[sf_ix(c, I, J, K + zoff)] = s / 8.0;
+    }
+}
+
+// fine pair (2I', 2I'+1) shares its coarse parent
+__global__ void __launch_bounds__(PX* PY) interp_p0_pair_kernel(PV f, double* __restrict__ y, double s,
+                                                                 PV c, const double* __restrict__ x,
+                                                                 int zoff, int depth) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, f.nz);
+    if (i >= f.nx || j >= f.ny) return;
+    for (int k = k0; k < k1; k++) {
+        const long q = sf_ix(f, i, j, k);
+        const double p = x[sf_ix(c, i >> 1, j >> 1, (k >> 1) + zoff)];
+        double2 u = ld2(y + q);
+        if (s == 0.0) {
+            u.x = p;
+            u.y = p;
+        } else {
+            u.x = s * u.x + p;
+            u.y = s * u.y + p;
+        }
+        *(double2*)(y + q) = u;
+    }
+}
+
+__global__ void __launch_bounds__(PX* PY) norm_pair_kernel(PV v, const double* __restrict__ x,
+                                                            int kind, int depth, double* out) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    unsigned long long m = 0ull;
+    double acc = 0.0;
+    if (i < v.nx && j < v.ny)
+        for (int k = k0; k < k1; k++) {
+            const double2 u = ld2(x + sf_ix(v, i, j, k));
+            m = umax64(m, umax64(abits(u.x), abits(u.y)));
+            acc += u.x * u.x;
+            acc += u.y * u.y;
+        }
+    if (kind == SF_NORM_MAX) {
+        block_max_atomic(m, out);
+    } else {
+        __shared__ double rs[PX * PY / 32];
+        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+        const int t = threadIdx.y * PX + threadIdx.x;
+        if ((t & 31) == 0) rs[t >> 5] = acc;
+        __syncthreads();
+        if (t == 0) {
+            for (int wq = 1; wq < PX * PY / 32; wq++) acc += rs[wq];
+            atomicAdd(out, acc);
+        }
+    }
+}
+
+__global__ void zero_scalar(double* p) { *p = 0.0; }
+
+// grid over pairs: (ceil(nx/64), ceil(ny/4), z-chunks) with ~16 blocks per SM
+inline dim3 pair_grid(int nx, int ny, int nz, int* depth) {
+    const int gx = (nx / 2 + PX - 1) / PX, gy = (ny + PY - 1) / PY;
+    const long want = 148L * 16;
+    int zc = (int)std::max(1L, std::min((long)nz, (want + (long)gx * gy - 1) / ((long)gx * gy)));
+    *depth = (nz + zc - 1) / zc;
+    zc = (nz + *depth - 1) / *depth;
+    return dim3(gx, gy, zc);
+}
+
+}  // namespace
+
+bool pair_ok(const sf_level* L) { return L->nx % 2 == 0; }
+
+sf_status k_residual_pair(sf_level* L, int res, int x, int rhs, double a, double b, double* nout) {
+    const double bh2 = b / (L->h * L->h);
+    SF_TRY(sf_halo(L, x, 1));
+    if (nout) {
+        zero_scalar<<<1, 1, 0, L->stream>>>(nout);
+        SF_LAUNCHED();
+    }
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        double* r = res >= 0 ? v.f[res] : nullptr;
+        if (r && nout)
+            residual_pair_kernel<true, true><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+        else if (r)
+            residual_pair_kernel<true, false><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+        else
+            residual_pair_kernel<false, true><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("residual_pair");
+}
+
+sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf) {
+    const double bh2 = b / (F->h * F->h);
+    const bool rep = C->nparts == 1 && F->nparts > 1;
+    SF_TRY(sf_halo(F, x, 1));
+    for (int p = 0; p < F->nlocal; p++) {
+        PV f = sf_view(F, p);
+        PV c = sf_view(C, rep ? 0 : p);
+        int depth;
+        dim3 g = pair_grid(f.nx, f.ny / 2, f.nz / 2, &depth);  // thread per coarse (I,J)
+        residual_restrict_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[x], f.f[rhs], a, bh2, c,
+                                                                    c.f[cf], rep ? f.z0 / 2 : 0,
+                                                                    depth);
+        SF_LAUNCHED();
+    }
+    SF_TRY(sf_check_launch("residual_restrict"));
+    if (rep) SF_TRY(sf_agglomerate(C, cf, F->nparts, F->lnz / 2));
+    return SF_OK;
+}
+
+sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf) {
+    const bool rep = C->nparts == 1 && F->nparts > 1;
+    for (int p = 0; p < F->nlocal; p++) {
+        PV f = sf_view(F, p);
+        PV c = sf_view(C, rep ? 0 : p);
+        int depth;
+        dim3 g = pair_grid(f.nx, f.ny, f.nz, &depth);
+        interp_p0_pair_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[ff], s, c, c.f[cf],
+                                                                 rep ? f.z0 / 2 : 0, depth);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("interp_p0_pair");
+}
+
+sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst) {
+    zero_scalar<<<1, 1, 0, L->stream>>>(dst);
+    SF_LAUNCHED();
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        norm_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[field], kind, depth, dst);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("norm_pair");
+}

@@ -151,8 +151,12 @@ static sf_status vcyc(sf_mg* m, int l) {
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     sf_level* C = m->lv[l + 1];
     SF_TRY(smooth(m, L, m->o.pre_pairs));
-    SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
-    SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
+    if (pair_ok(L)) {  // residual never stored: A6 + A7 in one pass
+        SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F));
+    } else {
+        SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
+        SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
+    }
     SF_TRY(k_zero(C, SF_U));
     SF_TRY(vcyc(m, l + 1));
     SF_TRY(k_interp(L, SF_U, 1.0, C, SF_U, m->o.vcycle_interp));
@@ -175,8 +179,14 @@ static sf_status fcyc(sf_mg* m) {
 // residual of the finest level and its max norm into dscratch[0] + pinned copy
 static sf_status check(sf_mg* m) {
     sf_level* L = m->lv[0];
-    SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
-    SF_TRY(sf_norm_async(L, SF_R, SF_NORM_MAX, L->dscratch));
+    if (pair_ok(L)) {  // max|f - Au| reduced in the residual pass, nothing stored
+        SF_TRY(k_residual_pair(L, -1, SF_U, SF_F, m->a, m->b, L->dscratch));
+        if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+            SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
+    } else {
+        SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
+        SF_TRY(sf_norm_async(L, SF_R, SF_NORM_MAX, L->dscratch));
+    }
     SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
                             L->stream));
     return SF_OK;

@@ -102,6 +102,14 @@ sf_status k_init_problem(sf_level* L, int problem, double a, double b, int want_
 sf_status k_bottom_setup(sf_level* L, double a, double b, double* ainv);
 sf_status k_bottom_solve(sf_level* L, int x, int rhs, const double* ainv);
 
+// pair-per-thread bandwidth kernels (kernels_pair.cu); need even nx
+bool pair_ok(const sf_level* L);
+sf_status k_residual_pair(sf_level* L, int res /* -1: do not write */, int x, int rhs, double a,
+                          double b, double* max_out /* NULL: no norm */);
+sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf);
+sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf);
+sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
+
 // fused colour pair (gsrb_fused.cu)
 bool gsrb_fused_supported(const sf_level* L);
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b);

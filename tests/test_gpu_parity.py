@@ -36,7 +36,7 @@ def make_level(sf, shape, coeffs, parts=1, h=None):
     return L
 
 
-SHAPES = [(16, 16, 16), (8, 6, 10), (20, 64, 64), (32, 24, 128), (40, 16, 192)]
+SHAPES = [(16, 16, 16), (8, 6, 10), (6, 5, 9), (20, 64, 64), (32, 24, 128), (40, 16, 192)]
 
 
 @pytest.mark.parametrize("shape", SHAPES)
