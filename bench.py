@@ -169,9 +169,7 @@ def run_reference(args):
     tv = sum(steps) / len(steps)
     cyc = solve_cycles_guess()
     t_solve = tv * (F_OVER_V + cyc)
-    dof = nx * ny * nz * args.gpus
-    val = dof / (t_solve * args.gpus) * args.gpus if args.gpus else dof / t_solve
-    val = (nx * ny * nz) / t_solve
+    val = (nx * ny * nz) / t_solve          # per-GPU-equivalent workload, one host
     sample = (f"{desc}{'' if scale == 1 else f' scaled x{scale:g} to {nx}^3'}; solve = 1 F-cycle "
               f"(= {F_OVER_V:.3f} V) + {cyc} V-cycles, per GPU-equivalent workload")
     line = {"impl": "reference", "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
@@ -244,12 +242,17 @@ def main():
     sf.sf_launch_count(reset=True)
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    prof = os.environ.get("SF_PROFILE_TIMED") == "1"   # ncu --profile-from-start off
     with ClockSampler(local) as clk:
+        if prof:
+            torch.cuda.cudart().cudaProfilerStart()
         e0.record(stream)
         for _ in range(args.steps):
             st, cyc, hist = step()
         e1.record(stream)
         barrier()
+        if prof:
+            torch.cuda.cudart().cudaProfilerStop()
     launches = sf.sf_launch_count(reset=True)
     t = max_over_ranks(e0.elapsed_time(e1) / 1e3)
     value = dof_local * world * args.steps / t

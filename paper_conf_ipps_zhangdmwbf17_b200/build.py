@@ -18,7 +18,14 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 BUILD = os.path.join(PKG, "_build")
 LIB = os.path.join(PKG, "libsf.so")
-SOURCES = ["level.cu", "kernels.cu", "kernels_pair.cu", "gsrb_fused.cu", "comm.cu", "mg.cu"]
+# (source, object, extra flags): the fused GSRB source is built for two tile shapes
+SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
+           ("kernels_pair.cu", "kernels_pair.o", []),
+           ("gsrb_fused.cu", "gsrb_fused_t32.o",
+            ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t32"]),
+           ("gsrb_fused.cu", "gsrb_fused_t64.o",
+            ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=3", "-DSF_GSRB_SUFFIX=_t64"]),
+           ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
@@ -32,13 +39,14 @@ def _needs(obj, deps):
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def _compile(src, force):
+def _compile(spec, force):
+    src, obj, extra = spec
     s = os.path.join(CSRC, src)
-    o = os.path.join(BUILD, src.replace(".cu", ".o"))
+    o = os.path.join(BUILD, obj)
     deps = [s, os.path.join(CSRC, "sf_internal.h"), os.path.join(INCLUDE, "sf.h")]
     if not force and not _needs(o, deps):
         return o, ""
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", s, "-o", o]
+    cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", s, "-o", o]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")

@@ -40,23 +40,43 @@
 
 namespace {
 
-constexpr int TX = 64;                 // tile width  = 32 lanes x 2 cells
-constexpr int TY = 8;                  // tile height = 8 warps
-constexpr int NT = 32 * TY;            // 256 threads
+// Tile = 512 cells handled by 8 warps, one red/black pair per thread.  32x16
+// (default) carries ~22% less halo per cell than 64x8 and 48 instead of 72
+// redundant ring cells; its smaller bundle leaves room for 4-deep prefetch.
+// Compiled twice by build.py: 32x16 with 4-deep prefetch (suffix _t32) and
+// 64x8 with 3-deep prefetch (_t64, used when ny % 16 != 0).
+#ifndef SF_GSRB_TX
+#define SF_GSRB_TX 32
+#endif
+#ifndef SF_GSRB_PF
+#define SF_GSRB_PF 4
+#endif
+#ifndef SF_GSRB_SUFFIX
+#define SF_GSRB_SUFFIX _t32
+#endif
+#define SF_CAT2(a, b) a##b
+#define SF_CAT(a, b) SF_CAT2(a, b)
+constexpr int TX = SF_GSRB_TX;         // tile width (cells)
+constexpr int PPR = TX / 2;            // pairs per row = lanes per row segment
+constexpr int NWARP = 8;
+constexpr int TY = NWARP * 32 / PPR;   // tile height (rows): 16 for TX = 32
+constexpr int NT = 32 * NWARP;         // 256 threads
 constexpr int W = TX + 4;              // smem row: gx in [x0-2, x0+TX+2)
 constexpr int XH = TY + 4;             // x rows:   gy in [y0-2, y0+TY+2)
 constexpr int CHH = TY + 3;            // coef rows: gy in [y0-1, y0+TY+2)
-constexpr int PF = 3;                  // bundles in flight ahead of the one being consumed
+constexpr int PF = SF_GSRB_PF;         // bundles in flight ahead of the one being consumed
 constexpr int NXS = 5 + PF, NCS = 1 + PF, NKS = 2 + PF, NMB = PF + 2;  // slot counts
 constexpr int NCA = 5;                 // staged coefficient arrays per plane (beta_k separate)
-constexpr int XSLOT = XH * W;          // doubles (6528 B = 51 x 128)
-constexpr int CARR = 752;              // 11*68 = 748 doubles padded to 128 B
+constexpr int XSLOT = (XH * W + 15) / 16 * 16;   // doubles, 128-byte multiple
+constexpr int CARR = (CHH * W + 15) / 16 * 16;
 constexpr int CSLOT = NCA * CARR;
 constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8;
 constexpr int BUNDLE_BYTES = XBYTES + (NCA + 1) * CBYTES;
 constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR) + 64;
+static_assert(SMEM <= 232448, "shared memory budget");
+static_assert(TX % 2 == 0 && 32 % PPR == 0, "tile shape");
 enum { CA_AL = 0, CA_DV = 1, CA_RH = 2, CA_BI = 3, CA_BJ = 4 };
-constexpr int NRING = TX + TX + TY / 2 + TY / 2;   // red ring cells per plane (72)
+constexpr int NRING = TX + TY;         // red ring cells per plane (half of the 1-ring)
 
 struct Maps {
     CUtensorMap x, al, dv, rh, bi, bj, bk;
@@ -142,16 +162,16 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
     double2 bkl = *(const double2*)&s.Klo[co_];
     double2 bkh = *(const double2*)&s.Khi[co_];
-    double bie = __shfl_down_sync(0xffffffffu, bi2.x, 1);
-    if (lane == 31) bie = s.C[CA_BI * CARR + co_ + 2];
+    double bie = __shfl_down_sync(0xffffffffu, bi2.x, 1, PPR);
+    if (lane == PPR - 1) bie = s.C[CA_BI * CARR + co_ + 2];
     double xc, xw, xe;
     if (SEL == 0) {
-        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1);
+        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1, PPR);
         if (lane == 0) xl = s.Xk[xo_ - 1];
         xc = xp2.x; xw = xl; xe = xp2.y;
     } else {
-        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1);
-        if (lane == 31) xr = s.Xk[xo_ + 2];
+        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1, PPR);
+        if (lane == PPR - 1) xr = s.Xk[xo_ + 2];
         xc = xp2.y; xw = xp2.x; xe = xr;
     }
     const int gxr = gx + SEL;
@@ -186,12 +206,12 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int lan
     double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
     double xc, xw, xe;
     if (SEL == 0) {
-        double ql = __shfl_up_sync(0xffffffffu, q2.y, 1);
+        double ql = __shfl_up_sync(0xffffffffu, q2.y, 1, PPR);
         if (lane == 0) ql = s.Xm[xo_ - 1];
         xc = q2.x; xw = ql; xe = q2.y;
     } else {
-        double qr = __shfl_down_sync(0xffffffffu, q2.x, 1);
-        if (lane == 31) qr = s.Xm[xo_ + 2];
+        double qr = __shfl_down_sync(0xffffffffu, q2.x, 1, PPR);
+        if (lane == PPR - 1) qr = s.Xm[xo_ + 2];
         xc = q2.y; xw = q2.x; xe = qr;
     }
     const int gxb = gx + SEL;
@@ -233,8 +253,7 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
 __global__ void __launch_bounds__(NT, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems) {
-    constexpr int NWARP = TY;
-    constexpr int RING_PER_WARP = NRING / NWARP;   // 9
+    constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
     double* Cs = Xs + NXS * XSLOT;                    // [NCS][NCA][CHH][W]
@@ -282,9 +301,11 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
 
         // this thread's pair: row gy, cells gxa (even) and gxa+1
-        const int gxa = x0 + 2 * lane, gy = y0 + w;
-        const int xoff = (w + 2) * W + 2 * lane + 2;
-        const int coff = (w + 1) * W + 2 * lane + 2;
+        // lanes [seg*PPR, (seg+1)*PPR) of warp w own row w + NWARP*seg (same parity)
+        const int hl = lane % PPR, row = w + NWARP * (lane / PPR);
+        const int gxa = x0 + 2 * hl, gy = y0 + row;
+        const int xoff = (row + 2) * W + 2 * hl + 2;
+        const int coff = (row + 1) * W + 2 * hl + 2;
         // ring cell of this thread for both parities of the plane (offsets + BC flags)
         int rxo[2], rco[2], rfl[2];
         bool rok[2];
@@ -293,7 +314,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
 #pragma unroll
             for (int par = 0; par < 2; par++) {
                 int rgx = 0, rgy = 0;
-                bool ok = lane < RING_PER_WARP;
+                bool ok = lane < RING_PER_WARP && rt < NRING;
                 if (rt < TX) {
                     int pp = rt % (TX / 2);
                     rgy = (rt < TX / 2) ? y0 - 1 : y0 + TY;
@@ -335,7 +356,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const int gkr = g.z0 + q;                    // plane of R
             const bool rin = q <= z1 && gkr >= 0 && gkr < g.gnz;
             const bool bin = t - 1 >= z0;                // B(t-1) on the tile
-            const int sel = (y0 + w + gkr) & 1;          // same pair position for R and B
+            const int sel = (y0 + w + gkr) & 1;          // same for both row segments
             StepCtx s;                                   // centred on plane q = t+1 for R
             s.Xk = Xs + ix_p1 * XSLOT;
             s.Xm = Xs + ix_0 * XSLOT;
@@ -355,11 +376,11 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             // planes t+1 and t-1 have the same parity: the black cell of
             // plane t-1 is the pair's other cell (position 1-sel)
             if (sel == 0) {
-                if (rin) rn = red_pair<0>(s, xoff, coff, lane, gxa, gy, g, zlo, zhi, a, bh2, nb);
-                if (bin) o = black_pair<1>(sb, xoff, lane, gxa, gy, g, gkm, a, bh2, stash);
+                if (rin) rn = red_pair<0>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (bin) o = black_pair<1>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
             } else {
-                if (rin) rn = red_pair<1>(s, xoff, coff, lane, gxa, gy, g, zlo, zhi, a, bh2, nb);
-                if (bin) o = black_pair<0>(sb, xoff, lane, gxa, gy, g, gkm, a, bh2, stash);
+                if (rin) rn = red_pair<1>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (bin) o = black_pair<0>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
             }
             const int par = gkr & 1;
             const bool ring = rin && (par ? rok[1] : rok[0]);
@@ -369,9 +390,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             double* Xw = Xs + ix_p1 * XSLOT;
             if (rin) Xw[xoff + sel] = rn;
             if (ring) Xw[ro] = rr;
-            if (bin)
-                *(double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
-                            SF_OX + gxa) = o;
+            if (bin)   // streaming store: do not evict halo lines other tiles still need
+                __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
+                                  SF_OX + gxa), o);
 #pragma unroll
             for (int i = 0; i < 9; i++) stash[i] = nb[i];
             fence_proxy_async();
@@ -426,12 +447,13 @@ int g_num_sms = 0;
 
 }  // namespace
 
-bool gsrb_fused_supported(const sf_level* L) {
+bool SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(const sf_level* L) {
     return L->nx % TX == 0 && L->ny % TY == 0 && L->lnz >= 1;
 }
 
-sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b) {
-    if (!gsrb_fused_supported(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%64==0, ny%%8==0");
+sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
+                                                    double b) {
+    if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
     SF_TRY(get_encoder());
     static bool attr = false;
     if (!attr) {

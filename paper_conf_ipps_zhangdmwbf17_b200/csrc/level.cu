@@ -269,6 +269,15 @@ extern "C" sf_status sf_residual(sf_level* L, int res, int x, int rhs, double a,
     return k_residual(L, res, x, rhs, a, b);
 }
 
+bool gsrb_fused_supported(const sf_level* L) {
+    return gsrb_fused_supported_t32(L) || gsrb_fused_supported_t64(L);
+}
+
+sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b) {
+    if (gsrb_fused_supported_t32(L)) return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b);
+    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b);
+}
+
 static void swap_fields(sf_level* L, int f1, int f2) {
     for (auto& P : L->parts) std::swap(P.f[f1], P.f[f2]);
 }

@@ -110,7 +110,11 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
 sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf);
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
 
-// fused colour pair (gsrb_fused.cu)
+// fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
+bool gsrb_fused_supported_t32(const sf_level* L);
+bool gsrb_fused_supported_t64(const sf_level* L);
+sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b);
+sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b);
 bool gsrb_fused_supported(const sf_level* L);
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b);
 

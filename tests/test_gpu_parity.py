@@ -92,13 +92,13 @@ def test_dinv(sf, oracle, shape):
     assert rel(L.download(sf.SF_DINV), P.dinv()) < 1e-14
 
 
-@pytest.mark.parametrize("shape", SHAPES + [(64, 64, 64), (24, 8, 64)])
+@pytest.mark.parametrize("shape", SHAPES + [(64, 64, 64), (24, 8, 64), (12, 16, 32), (8, 16, 96)])
 @pytest.mark.parametrize("kind", ["colour", "fused"])
 def test_gsrb_per_pair(sf, oracle, shape, kind):
     """Each RB pair (BC, red, BC, black) matches the oracle to 1e-12."""
     nz, ny, nx = shape
-    if kind == "fused" and (nx % 64 or ny % 8):
-        pytest.skip("fused kernel needs nx%64==0, ny%8==0")
+    if kind == "fused" and not ((nx % 32 == 0 and ny % 16 == 0) or (nx % 64 == 0 and ny % 8 == 0)):
+        pytest.skip("fused kernel needs (nx%32, ny%16) or (nx%64, ny%8) == 0")
     a, b = 1.0, 1.0
     h = I.level_h(nx, ny, nz)
     coeffs = I.hpgmg_coeffs(nx, ny, nz) if nx >= 64 else I.random_coeffs(nx, ny, nz, 5)
