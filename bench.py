@@ -33,8 +33,6 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 GSRB_BYTES_PER_CELL = 64      # PAPER.md:669-672 (x r+w, rhs, alpha, beta x3, lambda)
-WEAK_SHAPES = {1: (512, 512, 512), 2: (512, 512, 1024), 4: (512, 1024, 1024),
-               8: (1024, 1024, 1024)}   # (nx, ny, nz)
 F_OVER_V = 8.0 / 7.0          # F-cycle cost in finest-level V-cycles (sum over levels)
 
 
@@ -52,9 +50,8 @@ def parse():
 
 
 def dims_for(n, gpus):
-    if n == 512 and gpus in WEAK_SHAPES:
-        return WEAK_SHAPES[gpus]
-    return (n, n, n * gpus)
+    from paper_conf_ipps_zhangdmwbf17_b200.parallel import weak_dims
+    return weak_dims(n, gpus)
 
 
 # ------------------------------------------------------------------ clocks
@@ -218,12 +215,10 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
+    from paper_conf_ipps_zhangdmwbf17_b200.parallel import max_over_ranks as _mor
+
     def max_over_ranks(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return _mor(x, device=dev)
 
     nx, ny, nz = dims_for(args.n, world)
     comm = sf.Comm.nccl() if world > 1 else None

@@ -100,7 +100,7 @@ typedef struct {
     double rtol;            /* ||f-Au||inf/||f||inf target (1e-10, reading R-9) */
 } sf_mg_opts;
 
-/* Default options (pre=post=2, P0/PL, agglomerate below 8 planes, 50 cycles,
+/* Default options (pre=post=2, P0/PL, agglomerate below 16 planes, 50 cycles,
  * graphs on, AUTO smoother, rtol 1e-10). */
 void sf_mg_opts_default(sf_mg_opts* o);
 
@@ -195,6 +195,15 @@ sf_status sf_sync(sf_level* level);
  *   max_cycles+1 doubles); syncs.
  */
 sf_status sf_mg_create(sf_mg** out, sf_level* finest, double a, double b, const sf_mg_opts* opts);
+/* Host-only (no device needed): the hierarchy sf_mg_create builds for a
+ * gnx x gny x gnz level split into nparts z-slabs -- coarsen while every dim is
+ * even and the min dim > 2; a level stays decomposed while its slabs keep >=
+ * agglom_min_planes planes (and it is not the bottom), else it and all coarser
+ * levels are replicated (agglomerated).  Fills up to max_levels entries of
+ * dims[3*l .. 3*l+2] and distributed[l]; *nlevels = levels.  SF_ERR_SHAPE if the
+ * bottom would exceed 64 cells or slabs cannot be halved. */
+sf_status sf_mg_plan(int gnx, int gny, int gnz, int nparts, int agglom_min_planes, int max_levels,
+                     int* nlevels, int* dims, int* distributed);
 sf_status sf_mg_num_levels(const sf_mg* mg, int* n);
 sf_status sf_mg_level(sf_mg* mg, int l, sf_level** out);
 sf_status sf_vcycle(sf_mg* mg, int l);

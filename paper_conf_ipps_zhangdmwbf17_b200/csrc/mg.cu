@@ -30,7 +30,7 @@ extern "C" void sf_mg_opts_default(sf_mg_opts* o) {
     o->post_pairs = 2;
     o->vcycle_interp = SF_INTERP_P0;
     o->fcycle_interp = SF_INTERP_PL;
-    o->agglom_min_planes = 8;
+    o->agglom_min_planes = 16;
     o->max_cycles = 50;
     o->use_graph = 1;
     o->smoother = SF_SMOOTH_AUTO;
@@ -55,6 +55,51 @@ extern "C" sf_status sf_mg_destroy(sf_mg* m) {
     return SF_OK;
 }
 
+// Hierarchy plan shared by sf_mg_create and the host-side tests.
+struct LevelPlan {
+    int nx, ny, nz;
+    bool distributed;
+};
+
+static sf_status plan_levels(int gnx, int gny, int gnz, int nparts, int amin,
+                             std::vector<LevelPlan>& out) {
+    out.clear();
+    if (gnx < 2 || gny < 2 || gnz < 2 || nparts < 1 || amin < 2)
+        return sf_fail(SF_ERR_INVALID, "bad plan arguments");
+    if (gnz % nparts) return sf_fail(SF_ERR_SHAPE, "gnz=%d not divisible by %d parts", gnz, nparts);
+    out.push_back({gnx, gny, gnz, nparts > 1});
+    for (;;) {
+        const LevelPlan F = out.back();
+        int mn = std::min(F.nx, std::min(F.ny, F.nz));
+        if (mn <= 2 || (F.nx | F.ny | F.nz) & 1) break;
+        int cx = F.nx / 2, cy = F.ny / 2, cz = F.nz / 2;
+        if (F.distributed && (F.nz / nparts) % 2 != 0)
+            return sf_fail(SF_ERR_SHAPE, "odd planes per part (%d) cannot coarsen", F.nz / nparts);
+        bool last = std::min(cx, std::min(cy, cz)) <= 2 || ((cx | cy | cz) & 1);
+        bool dist = F.distributed && !last && (F.nz / nparts) / 2 >= amin;
+        out.push_back({cx, cy, cz, dist});
+    }
+    const LevelPlan B = out.back();
+    if (B.distributed || (long)B.nx * B.ny * B.nz > 64)
+        return sf_fail(SF_ERR_SHAPE, "coarsest level %dx%dx%d is not a <=64-cell replicated box",
+                       B.nx, B.ny, B.nz);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_mg_plan(int gnx, int gny, int gnz, int nparts, int amin, int max_levels,
+                                int* nlevels, int* dims, int* distributed) {
+    std::vector<LevelPlan> P;
+    SF_TRY(plan_levels(gnx, gny, gnz, nparts, amin, P));
+    if (nlevels) *nlevels = (int)P.size();
+    for (int l = 0; l < (int)P.size() && l < max_levels; l++) {
+        if (dims) {
+            dims[3 * l] = P[l].nx; dims[3 * l + 1] = P[l].ny; dims[3 * l + 2] = P[l].nz;
+        }
+        if (distributed) distributed[l] = P[l].distributed ? 1 : 0;
+    }
+    return SF_OK;
+}
+
 extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double b,
                                   const sf_mg_opts* opts) {
     if (!out || !fine) return sf_fail(SF_ERR_INVALID, "NULL argument");
@@ -67,38 +112,32 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
         delete m;
         return sf_fail(SF_ERR_INVALID, "bad mg options");
     }
+    std::vector<LevelPlan> plan;
+    {
+        sf_status ps = plan_levels(fine->gnx, fine->gny, fine->gnz, fine->nparts,
+                                   m->o.agglom_min_planes, plan);
+        if (ps != SF_OK) {
+            delete m;
+            return ps;
+        }
+    }
     m->lv.push_back(fine);
     m->own.push_back(false);
-    // coarsen while every dim is even and the min dim is > 2
-    for (;;) {
+    for (size_t l = 1; l < plan.size(); l++) {
         sf_level* F = m->lv.back();
-        int mn = std::min(F->gnx, std::min(F->gny, F->gnz));
-        if (mn <= 2 || (F->gnx | F->gny | F->gnz) & 1) break;
-        int cx = F->gnx / 2, cy = F->gny / 2, cz = F->gnz / 2;
-        bool last = std::min(cx, std::min(cy, cz)) <= 2 || ((cx | cy | cz) & 1);
-        bool distributed = F->nparts > 1 && F->comm && !last &&
-                           F->lnz / 2 >= m->o.agglom_min_planes && F->lnz % 2 == 0;
-        if (F->nparts > 1 && F->lnz % 2 != 0) {
-            sf_mg_destroy(m);
-            return sf_fail(SF_ERR_SHAPE, "odd planes per part (%d) cannot coarsen", F->lnz);
-        }
+        const LevelPlan& P = plan[l];
         sf_level* C = nullptr;
-        sf_status s = sf_level_create(&C, cx, cy, cz, 2.0 * F->h, distributed ? F->comm : nullptr,
-                                      F->stream, nullptr, 0);
+        sf_status s = sf_level_create(&C, P.nx, P.ny, P.nz, 2.0 * F->h,
+                                      P.distributed ? F->comm : nullptr, F->stream, nullptr, 0);
         if (s != SF_OK) {
             sf_mg_destroy(m);
             return s;
         }
-        if (!distributed) C->rep_comm = F->comm ? F->comm : F->rep_comm;
+        if (!P.distributed) C->rep_comm = F->comm ? F->comm : F->rep_comm;
         m->lv.push_back(C);
         m->own.push_back(true);
     }
     sf_level* B = m->lv.back();
-    if (B->nparts != 1 || (long)B->gnx * B->gny * B->gnz > 64) {
-        sf_mg_destroy(m);
-        return sf_fail(SF_ERR_SHAPE, "coarsest level %dx%dx%d is not a <=64-cell replicated box",
-                       B->gnx, B->gny, B->gnz);
-    }
     // operator on every level: restrict coefficients (A7), rebuild Dinv (A4)
     sf_status s = sf_rebuild_operator(fine, a, b);
     for (size_t l = 1; l < m->lv.size() && s == SF_OK; l++) {

@@ -40,7 +40,7 @@ EXPORTS = [
     "sf_level_download", "sf_level_field_ptr", "sf_init_problem", "sf_rebuild_operator",
     "sf_apply_bc", "sf_apply_op", "sf_smooth_gsrb", "sf_residual", "sf_restrict",
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
-    "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count",
+    "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
 ]
 
 
@@ -104,6 +104,7 @@ def lib():
         "sf_solve": (_i, [_vp, _i, _d, _i, C.POINTER(_i), _P]),
         "sf_mg_destroy": (_i, [_vp]),
         "sf_launch_count": (_i, [C.POINTER(C.c_longlong), _i]),
+        "sf_mg_plan": (_i, [_i, _i, _i, _i, _i, _i, C.POINTER(_i), C.POINTER(_i), C.POINTER(_i)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -266,6 +267,17 @@ def sf_mg_destroy(mg):
     _check(lib().sf_mg_destroy(mg))
 
 
+def sf_mg_plan(gnx, gny, gnz, nparts=1, agglom_min_planes=8, max_levels=32):
+    """Host-only hierarchy plan: [((nx, ny, nz), distributed), ...] finest first."""
+    n = _i()
+    dims = (_i * (3 * max_levels))()
+    dist = (_i * max_levels)()
+    _check(lib().sf_mg_plan(gnx, gny, gnz, nparts, agglom_min_planes, max_levels, C.byref(n),
+                            dims, dist))
+    return [((dims[3 * l], dims[3 * l + 1], dims[3 * l + 2]), bool(dist[l]))
+            for l in range(min(n.value, max_levels))]
+
+
 def sf_launch_count(reset=False):
     n = C.c_longlong()
     _check(lib().sf_launch_count(C.byref(n), int(reset)))
@@ -291,13 +303,9 @@ class Comm:
     @classmethod
     def nccl(cls, group=None):
         """One part per rank of the default (or given) torch.distributed group."""
-        import torch
-        import torch.distributed as dist
-        rank, world = dist.get_rank(group), dist.get_world_size(group)
-        uid = [sf_get_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0, group=group)
-        torch.cuda.synchronize()
-        return cls(sf_comm_create_nccl(uid[0], world, rank), world, 1, rank)
+        from . import parallel
+        uid, rank, world = parallel.broadcast_unique_id(group)
+        return cls(sf_comm_create_nccl(uid, world, rank), world, 1, rank)
 
     def close(self):
         if self.h:
