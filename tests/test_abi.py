@@ -78,5 +78,5 @@ def test_product_does_not_import_oracle():
         for f in fs:
             if f.endswith((".py", ".cu", ".h", ".cpp")):
                 txt = open(os.path.join(dp, f)).read()
-                assert not re.search(r"(^\s*(from|import)\s+oracle)|liboracle|or_[a-z_]+\(", txt,
+                assert not re.search(r"(^\s*(from|import)\s+oracle)|liboracle|\bor_[a-z_]+\(", txt,
                                      flags=re.M), f
