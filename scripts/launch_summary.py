@@ -9,10 +9,13 @@ def summarise(path):
     i = [k for k, r in enumerate(rows) if r and r[0] == "ID"][0]
     hdr, data = rows[i], rows[i + 1:]
     kn, mn, mv, idc = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("ID")
+    mu = hdr.index("Metric Unit")
+    scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1.0, "us": 1e3, "ms": 1e6,
+             "usecond": 1e3, "nsecond": 1.0, "msecond": 1e6}
     per = collections.defaultdict(dict)
     names = {}
     for r in data:
-        per[r[idc]][r[mn]] = float(r[mv].replace(",", ""))
+        per[r[idc]][r[mn]] = float(r[mv].replace(",", "")) * scale.get(r[mu], 1.0)
         names[r[idc]] = r[kn].split("(")[0].split("::")[-1].replace("void ", "")
     agg = collections.defaultdict(lambda: [0, 0.0, 0.0])
     for lid, m in per.items():
