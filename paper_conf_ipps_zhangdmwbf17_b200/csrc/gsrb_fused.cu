@@ -130,6 +130,24 @@ __device__ __forceinline__ double gs_update(double xc, double xw, double xe, dou
     return xc + dv * (rh - ax);
 }
 
+// A x at one cell (op_at term order); used for the fused input residual
+__device__ __forceinline__ double ax_at(double xc, double xw, double xe, double xs, double xn,
+                                       double xb, double xt, double bw, double be, double bs,
+                                       double bn, double bb, double bt, double al, double a,
+                                       double bh2) {
+    double flux = be * (xe - xc);
+    flux += bw * (xw - xc);
+    flux += bn * (xn - xc);
+    flux += bs * (xs - xc);
+    flux += bt * (xt - xc);
+    flux += bb * (xb - xc);
+    return a * al * xc - bh2 * flux;
+}
+
+__device__ __forceinline__ unsigned long long abits(double v) {
+    return (unsigned long long)__double_as_longlong(fabs(v));
+}
+
 struct Geo {
     int nx, ny, nz, z0, gnz;
     long js, ks;
@@ -149,10 +167,11 @@ struct StepCtx {
 // R(p) for the pair at smem offsets (xo_: x box, co_: coef box).  SEL = 1 if
 // the odd cell of the pair is red at this plane (warp-uniform).  Returns the
 // red-new value; leaves the black cell's coefficients of plane p in nb.
-template <int SEL>
+template <int SEL, bool RESID>
 __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
                                            int gy, const Geo& g, bool zlo, bool zhi, double a,
-                                           double bh2, double* nb) {
+                                           double bh2, double* nb, double& rres, double& rold,
+                                           double2& xpair) {
     double2 xp2 = *(const double2*)&s.Xk[xo_];
     double2 al2 = *(const double2*)&s.C[CA_AL * CARR + co_];
     double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
@@ -184,17 +203,64 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     double xt = zhi ? -xc : s.Xp[col];
     double r;
     if (SEL == 0) {
-        r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x, al2.x,
-                      dv2.x, rh2.x, a, bh2);
+        if (RESID) {
+            double ax = ax_at(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x,
+                              bkh.x, al2.x, a, bh2);
+            rres = rh2.x - ax;
+            r = xc + dv2.x * rres;
+        } else {
+            r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x,
+                          al2.x, dv2.x, rh2.x, a, bh2);
+        }
         nb[0] = bi2.y; nb[1] = bie; nb[2] = bjl.y; nb[3] = bjh.y; nb[4] = bkl.y; nb[5] = bkh.y;
         nb[6] = al2.y; nb[7] = dv2.y; nb[8] = rh2.y;
     } else {
-        r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y, al2.y,
-                      dv2.y, rh2.y, a, bh2);
+        if (RESID) {
+            double ax = ax_at(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y,
+                              al2.y, a, bh2);
+            rres = rh2.y - ax;
+            r = xc + dv2.y * rres;
+        } else {
+            r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y,
+                          al2.y, dv2.y, rh2.y, a, bh2);
+        }
         nb[0] = bi2.x; nb[1] = bi2.y; nb[2] = bjl.x; nb[3] = bjh.x; nb[4] = bkl.x; nb[5] = bkh.x;
         nb[6] = al2.x; nb[7] = dv2.x; nb[8] = rh2.x;
     }
+    rold = xc;
+    xpair = xp2;
     return r;
+}
+
+// Residual rhs - A x of the INPUT iterate at the black cell (position BS) of
+// plane q, computed during R(q) before any red write: in-plane red neighbours
+// are still old in smem, the red cell below (same column, plane q-1) is this
+// thread's red-old value of the previous plane, the one above is untouched.
+template <int BS>
+__device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int lane, int gx, int gy,
+                                              const Geo& g, bool zlo, bool zhi, double a,
+                                              double bh2, const double* nb, double rold_below,
+                                              double2 xp2) {
+    double xc, xw, xe;
+    if (BS == 1) {
+        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1, PPR);
+        if (lane == PPR - 1) xr = s.Xk[xo_ + 2];
+        xc = xp2.y; xw = xp2.x; xe = xr;
+    } else {
+        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1, PPR);
+        if (lane == 0) xl = s.Xk[xo_ - 1];
+        xc = xp2.x; xw = xl; xe = xp2.y;
+    }
+    const int gxb = gx + BS;
+    if (gxb == 0) xw = -xc;
+    if (gxb == g.nx - 1) xe = -xc;
+    const int col = xo_ + BS;
+    double xs = (gy == 0) ? -xc : s.Xk[col - W];
+    double xn = (gy == g.ny - 1) ? -xc : s.Xk[col + W];
+    double xb = zlo ? -xc : rold_below;
+    double xt = zhi ? -xc : s.Xp[col];
+    return nb[8] - ax_at(xc, xw, xe, xs, xn, xb, xt, nb[0], nb[1], nb[2], nb[3], nb[4], nb[5],
+                         nb[6], a, bh2);
 }
 
 // B for the pair; SEL = position (0: even x, 1: odd x) of the black cell in
@@ -250,9 +316,10 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
 // chains together (ILP 2) between two consecutive barriers.  The black cell's
 // coefficients of plane q are taken from the smem slot by R(q) at step q-1
 // and kept in registers until B(q) at step q+1 (stash alternates by step).
+template <bool RESID>
 __global__ void __launch_bounds__(NT, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
-                     double bh2, int depth, int ntx, int ntiles, int nitems) {
+                     double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax) {
     constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
@@ -267,6 +334,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
     }
     __syncthreads();
 
+    unsigned long long rbits = 0ull;  // RESID: max |rhs - A x_in| of this thread's cells
     unsigned seq = 0;  // bundles issued by this CTA so far (all threads track it)
     for (int item = blockIdx.x; item < nitems; item += gridDim.x) {
         const int chunk = item / ntiles, tile = item - chunk * ntiles;
@@ -334,6 +402,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                            ((rgy == g.ny - 1) << 3);
             }
         }
+        double rold = 0.0;  // RESID: red-old value of the previous plane (this pair)
         double stA[9], stB[9];
 #pragma unroll
         for (int i = 0; i < 9; i++) stA[i] = stB[i] = 0.0;
@@ -375,18 +444,34 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const int gkm = g.z0 + t - 1;
             // planes t+1 and t-1 have the same parity: the black cell of
             // plane t-1 is the pair's other cell (position 1-sel)
+            double rres = 0.0, rold_new = 0.0, bres = 0.0;
+            double2 xpair = make_double2(0.0, 0.0);
             if (sel == 0) {
-                if (rin) rn = red_pair<0>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb,
+                                                 rres, rold_new, xpair);
                 if (bin) o = black_pair<1>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
+                if (RESID && rin)
+                    bres = black_resid<1>(s, xoff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb, rold, xpair);
             } else {
-                if (rin) rn = red_pair<1>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb);
+                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb,
+                                                 rres, rold_new, xpair);
                 if (bin) o = black_pair<0>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
+                if (RESID && rin)
+                    bres = black_resid<0>(s, xoff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb, rold, xpair);
+            }
+            if (RESID) {
+                if (rin && q >= z0 && q < z1) {   // this item's planes only
+                    unsigned long long m2 = abits(rres) > abits(bres) ? abits(rres) : abits(bres);
+                    rbits = m2 > rbits ? m2 : rbits;
+                }
+                rold = rold_new;
             }
             const int par = gkr & 1;
             const bool ring = rin && (par ? rok[1] : rok[0]);
             const int ro = par ? rxo[1] : rxo[0];
             double rr = 0.0;
             if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], a, bh2, zlo, zhi);
+            if (RESID) __syncthreads();   // black residuals read red-OLD cells of plane q
             double* Xw = Xs + ix_p1 * XSLOT;
             if (rin) Xw[xoff + sel] = rn;
             if (ring) Xw[ro] = rr;
@@ -412,6 +497,19 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
+    }
+    if (RESID) {   // CTA max -> one atomic (bit order = numeric order for |r|; NaN wins)
+        __shared__ unsigned long long wmax[NWARP];
+        for (int o2 = 16; o2 > 0; o2 >>= 1) {
+            unsigned long long v = __shfl_xor_sync(0xffffffffu, rbits, o2);
+            rbits = v > rbits ? v : rbits;
+        }
+        if (lane == 0) wmax[w] = rbits;
+        __syncthreads();
+        if (tid == 0) {
+            for (int i = 1; i < NWARP; i++) rbits = wmax[i] > rbits ? wmax[i] : rbits;
+            atomicMax((unsigned long long*)rmax, rbits);
+        }
     }
 }
 
@@ -451,13 +549,19 @@ bool SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(const sf_level* L) {
     return L->nx % TX == 0 && L->ny % TY == 0 && L->lnz >= 1;
 }
 
+static __global__ void zero_bits(double* p) { *p = 0.0; }
+
+// rmax != NULL: also reduce max |rhs - A x_in| of the INPUT iterate into *rmax
+// (device scalar; the caller all-reduces across ranks).
 sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
-                                                    double b) {
+                                                    double b, double* rmax) {
     if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
     SF_TRY(get_encoder());
     static bool attr = false;
     if (!attr) {
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel,
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<true>,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
@@ -495,8 +599,17 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
         int grid = std::min(items, G);
-        gsrb_pair_tma_kernel<<<grid, NT, SMEM, L->stream>>>(mp, g, v.f[xout], a, bh2, depth,
-                                                               ntx, tiles, items);
+        if (rmax) {
+            if (p == 0) {
+                zero_bits<<<1, 1, 0, L->stream>>>(rmax);
+                SF_LAUNCHED();
+            }
+            gsrb_pair_tma_kernel<true><<<grid, NT, SMEM, L->stream>>>(
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax);
+        } else {
+            gsrb_pair_tma_kernel<false><<<grid, NT, SMEM, L->stream>>>(
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr);
+        }
         SF_LAUNCHED();
     }
     return sf_check_launch("gsrb_pair_tma");

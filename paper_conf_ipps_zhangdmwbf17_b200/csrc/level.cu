@@ -273,12 +273,13 @@ bool gsrb_fused_supported(const sf_level* L) {
     return gsrb_fused_supported_t32(L) || gsrb_fused_supported_t64(L);
 }
 
-sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b) {
-    if (gsrb_fused_supported_t32(L)) return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b);
-    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b);
+sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
+                            double* rmax) {
+    if (gsrb_fused_supported_t32(L)) return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax);
+    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b, rmax);
 }
 
-static void swap_fields(sf_level* L, int f1, int f2) {
+void sf_swap_fields(sf_level* L, int f1, int f2) {
     for (auto& P : L->parts) std::swap(P.f[f1], P.f[f2]);
 }
 
@@ -302,7 +303,7 @@ extern "C" sf_status sf_smooth_gsrb(sf_level* L, int x, int rhs, double a, doubl
         for (int p = 0; p < rb_pairs; p++) {
             SF_TRY(sf_halo(L, x, 2));
             SF_TRY(k_gsrb_pair_fused(L, x, other, rhs, a, b));
-            swap_fields(L, x, other);  // result now lives under the id `x`
+            sf_swap_fields(L, x, other);  // result now lives under the id `x`
         }
         return SF_OK;
     }

@@ -19,8 +19,8 @@ struct sf_mg {
     double a, b;
     sf_mg_opts o;
     double* ainv = nullptr;
-    cudaGraphExec_t gexec[2] = {nullptr, nullptr};  // [0] V-cycle+check, [1] F-cycle+check
-    long long gnodes[2] = {0, 0};
+    cudaGraphExec_t gexec[5] = {};  // V+check, F+check, F, first pair+check, rest of V
+    long long gnodes[5] = {};
     bool graph_failed = false;
 };
 
@@ -184,12 +184,13 @@ static sf_status smooth(sf_mg* m, sf_level* L, int pairs) {
     return sf_smooth_gsrb(L, SF_U, SF_F, m->a, m->b, pairs, m->o.smoother);
 }
 
-// V(l): smooth, residual, restrict, zero e_{l+1}, V(l+1), e_l += P0 e_{l+1}, smooth
-static sf_status vcyc(sf_mg* m, int l) {
+// V(l): smooth, residual, restrict, zero e_{l+1}, V(l+1), e_l += P0 e_{l+1}, smooth.
+// skip_first: the first pre-smoothing pair was already run (fused check, below).
+static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     sf_level* L = m->lv[l];
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     sf_level* C = m->lv[l + 1];
-    SF_TRY(smooth(m, L, m->o.pre_pairs));
+    SF_TRY(smooth(m, L, m->o.pre_pairs - (skip_first ? 1 : 0)));
     if (pair_ok(L)) {  // residual never stored: A6 + A7 in one pass
         SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F));
     } else {
@@ -215,7 +216,13 @@ static sf_status fcyc(sf_mg* m) {
     return SF_OK;
 }
 
-// residual of the finest level and its max norm into dscratch[0] + pinned copy
+static sf_status to_host(sf_level* L) {
+    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
+                            L->stream));
+    return SF_OK;
+}
+
+// separate convergence check: max|F - A U| of the finest level (A6 + A10)
 static sf_status check(sf_mg* m) {
     sf_level* L = m->lv[0];
     if (pair_ok(L)) {  // max|f - Au| reduced in the residual pass, nothing stored
@@ -226,63 +233,104 @@ static sf_status check(sf_mg* m) {
         SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
         SF_TRY(sf_norm_async(L, SF_R, SF_NORM_MAX, L->dscratch));
     }
-    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
-                            L->stream));
-    return SF_OK;
+    return to_host(L);
+}
+
+// The convergence check fused into the next cycle's first pre-smoothing pair:
+// the colour-fused pair streams every operand anyway and reduces
+// max|F - A U_in| of its INPUT while it writes the smoothed iterate to TMP.
+// If that says "converged", U (the previous cycle's result) is untouched.
+static bool fused_check_ok(const sf_mg* m) {
+    return m->lv.size() > 1 && m->o.pre_pairs >= 1 && m->o.smoother != SF_SMOOTH_COLOUR &&
+           gsrb_fused_supported(m->lv[0]) && (m->o.pre_pairs + m->o.post_pairs) % 2 == 0;
+}
+
+static sf_status first_pair_check(sf_mg* m) {
+    sf_level* L = m->lv[0];
+    SF_TRY(sf_halo(L, SF_F, 1));
+    SF_TRY(sf_halo(L, SF_U, 2));
+    SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
+    sf_swap_fields(L, SF_U, SF_TMP);
+    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+        SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
+    return to_host(L);
 }
 
 static bool graphs_allowed(const sf_mg* m) {
     if (!m->o.use_graph || m->graph_failed) return false;
     if (m->lv[0]->stream == nullptr) return false;  // legacy stream cannot be captured
-    // the fused smoother swaps U/TMP per pair; only an even count per smooth
-    // leaves the host-side mapping unchanged across a captured cycle
+    // the fused smoother swaps U/TMP per pair; only an even count per captured
+    // sequence leaves the host-side mapping unchanged for replays
     return (m->o.pre_pairs % 2 == 0 && m->o.post_pairs % 2 == 0) ||
            m->o.smoother == SF_SMOOTH_COLOUR;
 }
 
-// run cycle kind (0 = V on level 0, 1 = F) followed by the check
-static sf_status run_cycle(sf_mg* m, int kind) {
-    sf_level* L = m->lv[0];
-    auto body = [&]() -> sf_status {
-        if (kind == 0) SF_TRY(vcyc(m, 0)); else SF_TRY(fcyc(m));
-        return check(m);
-    };
-    if (!graphs_allowed(m)) return body();
-    if (!m->gexec[kind]) {
-        long long before, after;
-        sf_launch_count(&before, 0);
-        if (cudaStreamBeginCapture(L->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
-            cudaGetLastError();
-            m->graph_failed = true;
-            return body();
-        }
-        sf_status s = body();
-        cudaGraph_t g = nullptr;
-        cudaError_t e = cudaStreamEndCapture(L->stream, &g);
-        if (s != SF_OK) {
-            if (g) cudaGraphDestroy(g);
-            return s;
-        }
-        if (e != cudaSuccess || !g) {
-            cudaGetLastError();
-            m->graph_failed = true;
-            return body();
-        }
-        e = cudaGraphInstantiate(&m->gexec[kind], g, 0);
-        cudaGraphDestroy(g);
-        if (e != cudaSuccess) {
-            cudaGetLastError();
-            m->gexec[kind] = nullptr;
-            m->graph_failed = true;
-            return body();
-        }
-        sf_launch_count(&after, 0);
-        m->gnodes[kind] = after - before;
-        sf_count_launch(-(after - before));  // captured, not launched
+enum { G_VCHECK = 0, G_FCHECK = 1, G_F = 2, G_FIRST = 3, G_REST = 4 };
+
+static sf_status body_of(sf_mg* m, int kind) {
+    switch (kind) {
+        case G_VCHECK: SF_TRY(vcyc(m, 0)); return check(m);
+        case G_FCHECK: SF_TRY(fcyc(m)); return check(m);
+        case G_F: return fcyc(m);
+        case G_FIRST: return first_pair_check(m);
+        default: return vcyc(m, 0, true);
     }
-    SF_CUDA(cudaGraphLaunch(m->gexec[kind], L->stream));
-    sf_count_launch(m->gnodes[kind]);
+}
+
+static sf_status capture(sf_mg* m, int kind) {
+    sf_level* L = m->lv[0];
+    long long before, after;
+    sf_launch_count(&before, 0);
+    if (cudaStreamBeginCapture(L->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        cudaGetLastError();
+        m->graph_failed = true;
+        return SF_OK;
+    }
+    sf_status s = body_of(m, kind);
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(L->stream, &g);
+    sf_launch_count(&after, 0);
+    sf_count_launch(-(after - before));  // captured, not launched
+    if (s != SF_OK) {
+        if (g) cudaGraphDestroy(g);
+        return s;
+    }
+    if (e != cudaSuccess || !g) {
+        cudaGetLastError();
+        m->graph_failed = true;
+        return SF_OK;
+    }
+    e = cudaGraphInstantiate(&m->gexec[kind], g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        m->gexec[kind] = nullptr;
+        m->graph_failed = true;
+        return SF_OK;
+    }
+    m->gnodes[kind] = after - before;
     return SF_OK;
+}
+
+// enqueue cycle piece `kind` (graph replay when possible)
+static sf_status run(sf_mg* m, int kind) {
+    sf_level* L = m->lv[0];
+    if (graphs_allowed(m) && !m->gexec[kind]) {
+        if (kind == G_FIRST || kind == G_REST) {
+            // capture both halves back to back: together they hold an even
+            // number of U/TMP swaps, so the host mapping is restored
+            SF_TRY(capture(m, G_FIRST));
+            SF_TRY(capture(m, G_REST));
+        } else {
+            SF_TRY(capture(m, kind));
+        }
+    }
+    if (graphs_allowed(m) && m->gexec[kind]) {
+        SF_CUDA(cudaGraphLaunch(m->gexec[kind], L->stream));
+        sf_count_launch(m->gnodes[kind]);
+        return SF_OK;
+    }
+    return body_of(m, kind);
 }
 
 extern "C" sf_status sf_vcycle(sf_mg* m, int l) {
@@ -310,18 +358,47 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
         SF_TRY(k_zero(L, SF_U));
         return sf_sync(L);
     }
-    int c = 0;
-    bool first = true;
-    while (c < max_cycles) {
-        SF_TRY(run_cycle(m, (fcycle && first) ? 1 : 0));
-        first = false;
-        SF_CUDA(cudaStreamSynchronize(L->stream));
-        double rel = L->hscratch[0] / fn;
-        if (hist) hist[c] = rel;
-        c++;
+    const bool fused = fused_check_ok(m);
+    auto fin = [&](double rel, int c) -> int {  // 0 continue, 1 converged, -1 numeric error
+        if (hist) hist[c - 1] = rel;
         if (cycles) *cycles = c;
-        if (!(rel == rel) || std::isinf(rel)) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
-        if (rel < rtol) return SF_OK;
+        if (!(rel == rel) || std::isinf(rel)) return -1;
+        return rel < rtol ? 1 : 0;
+    };
+    if (!fused) {
+        for (int c = 1; c <= max_cycles; c++) {
+            SF_TRY(run(m, (fcycle && c == 1) ? G_FCHECK : G_VCHECK));
+            SF_CUDA(cudaStreamSynchronize(L->stream));
+            int r = fin(L->hscratch[0] / fn, c);
+            if (r < 0) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
+            if (r > 0) return SF_OK;
+        }
+        return sf_fail(SF_ERR_NOT_CONVERGED, "no convergence to %g in %d cycles", rtol, max_cycles);
     }
-    return sf_fail(SF_ERR_NOT_CONVERGED, "no convergence to %g in %d cycles", rtol, max_cycles);
+    int done = 0;
+    if (fcycle) {
+        SF_TRY(run(m, G_F));
+        done = 1;
+    }
+    for (;;) {
+        // first pair of the next V-cycle + max|F - A U| of the iterate after `done` cycles
+        const double* u0 = L->parts[0].f[SF_U];
+        SF_TRY(run(m, G_FIRST));
+        SF_CUDA(cudaStreamSynchronize(L->stream));
+        if (done >= 1) {
+            int r = fin(L->hscratch[0] / fn, done);
+            if (r != 0 || done >= max_cycles) {
+                // discard the speculative pair: the iterate of cycle `done` is
+                // the buffer U named before it (a graph replay leaves the
+                // host-side mapping as it was; an eager run swapped it)
+                if (L->parts[0].f[SF_U] != u0) sf_swap_fields(L, SF_U, SF_TMP);
+                if (r < 0) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
+                if (r > 0) return SF_OK;
+                return sf_fail(SF_ERR_NOT_CONVERGED, "no convergence to %g in %d cycles", rtol,
+                               max_cycles);
+            }
+        }
+        SF_TRY(run(m, G_REST));
+        done++;
+    }
 }

@@ -67,6 +67,7 @@ __host__ __device__ __forceinline__ long sf_ix(const PV& v, int i, int j, int k)
 }
 
 PV sf_view(const sf_level* L, int p);
+void sf_swap_fields(sf_level* L, int f1, int f2);   // host-side id <-> buffer mapping
 
 sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst);
 
@@ -113,10 +114,14 @@ sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
 // fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
 bool gsrb_fused_supported_t32(const sf_level* L);
 bool gsrb_fused_supported_t64(const sf_level* L);
-sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b);
-sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b);
+sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b,
+                                double* rmax);
+sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
+                                double* rmax);
 bool gsrb_fused_supported(const sf_level* L);
-sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b);
+// rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax
+sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
+                            double* rmax = nullptr);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.

@@ -329,3 +329,38 @@ def test_c3_full_size_gsrb_pair(sf, oracle):
     got = L.download(sf.SF_U)
     P = oracle.Problem(oracle.Grid(n, n, n, 1.0 / n), 1.0, 1.0, *coeffs)
     assert rel(got, P.smooth(x, f, 1)) < TOL
+
+
+@pytest.mark.parametrize("fcycle", [False, True])
+def test_solve_eager_equals_graph(sf, oracle, fcycle):
+    """The fused convergence check (first pre-smoothing pair reduces the input
+    residual) gives the same iterate and cycle count with and without CUDA
+    graph replay."""
+    n = 32
+    out = {}
+    for g in (0, 1):
+        L, M, O = mg_pair(sf, oracle, n, use_graph=g)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        st, cyc, hist = M.solve(fcycle=fcycle, rtol=1e-10)
+        out[g] = (L.download(sf.SF_U), cyc, hist)
+    assert out[0][1] == out[1][1]
+    assert np.array_equal(out[0][0], out[1][0])
+    assert np.allclose(out[0][2], out[1][2], rtol=1e-12, atol=0)
+
+
+@pytest.mark.parametrize("use_graph", [0, 1])
+def test_solve_max_cycles_keeps_last_cycle(sf, oracle, use_graph):
+    """Stopping at max_cycles discards the speculative first pair of the next
+    cycle: U equals the oracle's iterate after exactly max_cycles cycles."""
+    n = 64
+    L, M, O = mg_pair(sf, oracle, n, use_graph=use_graph)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, max_cycles=3, raise_on_error=False)
+    assert st == sf.SF_ERR_NOT_CONVERGED and cyc == 3
+    u = O.fcycle(f)
+    for _ in range(2):
+        u = O.vcycle(u, f)
+    assert rel(L.download(sf.SF_U), u) < 1e-11
+    assert abs(hist[-1] / O.relres(u, f) - 1) < 1e-6
