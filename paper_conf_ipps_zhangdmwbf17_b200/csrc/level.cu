@@ -274,9 +274,10 @@ bool gsrb_fused_supported(const sf_level* L) {
 }
 
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                            double* rmax) {
-    if (gsrb_fused_supported_t32(L)) return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax);
-    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b, rmax);
+                            double* rmax, sf_level* C, int cf) {
+    if (gsrb_fused_supported_t32(L))
+        return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax, C, cf);
+    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b, rmax, C, cf);
 }
 
 void sf_swap_fields(sf_level* L, int f1, int f2) {

@@ -199,6 +199,17 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     }
     SF_TRY(k_zero(C, SF_U));
     SF_TRY(vcyc(m, l + 1));
+    if (m->o.vcycle_interp == SF_INTERP_P0 && m->o.post_pairs >= 1 &&
+        m->o.smoother != SF_SMOOTH_COLOUR && gsrb_fused_supported(L)) {
+        // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
+        SF_TRY(sf_halo(C, SF_U, 1));
+        SF_TRY(sf_halo(L, SF_F, 1));
+        SF_TRY(sf_halo(L, SF_U, 2));
+        SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, nullptr, C, SF_U));
+        sf_swap_fields(L, SF_U, SF_TMP);
+        SF_TRY(smooth(m, L, m->o.post_pairs - 1));
+        return SF_OK;
+    }
     SF_TRY(k_interp(L, SF_U, 1.0, C, SF_U, m->o.vcycle_interp));
     SF_TRY(smooth(m, L, m->o.post_pairs));
     return SF_OK;

@@ -115,13 +115,14 @@ sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
 bool gsrb_fused_supported_t32(const sf_level* L);
 bool gsrb_fused_supported_t64(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                                double* rmax);
+                                double* rmax, sf_level* C, int cf);
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                                double* rmax);
+                                double* rmax, sf_level* C, int cf);
 bool gsrb_fused_supported(const sf_level* L);
-// rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax
+// rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax;
+// C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                            double* rmax = nullptr);
+                            double* rmax = nullptr, sf_level* C = nullptr, int cf = 0);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.
