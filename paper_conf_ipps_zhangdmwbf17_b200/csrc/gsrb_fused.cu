@@ -73,20 +73,23 @@ constexpr int CSLOT = NCA * CARR;
 constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8;
 constexpr int BUNDLE_BYTES = XBYTES + (NCA + 1) * CBYTES;
 constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR) + 64;
-// fused P0 interpolation (INTERP): coarse parents of an x box, one per x plane
-constexpr int CW = W / 2, CHX = XH / 2;            // coarse box (x0-2)/2.. x (y0-2)/2..
-constexpr int CBOX = (CW * CHX + 15) / 16 * 16;     // doubles, 128-byte multiple
-constexpr int CBOX_BYTES = CW * CHX * 8;
-constexpr int NES = PF + 2;                         // coarse box slots (x-plane ring)
-constexpr size_t SMEM_INTERP = SMEM + 64 + sizeof(double) * NES * CBOX;
-static_assert(SMEM_INTERP <= 232448, "shared memory budget");
+// fused P0 interpolation (INTERP): each x-box pair (2 cells, one parent) is
+// corrected in smem; a thread owns pairs tid and tid+NT of the box
+constexpr int XPAIRS = XH * (W / 2);
+static_assert(XPAIRS <= 2 * NT, "two correction pairs per thread");
 static_assert(TX % 2 == 0 && 32 % PPR == 0, "tile shape");
 enum { CA_AL = 0, CA_DV = 1, CA_RH = 2, CA_BI = 3, CA_BJ = 4 };
 constexpr int NRING = TX + TY;         // red ring cells per plane (half of the 1-ring)
 
 struct Maps {
     CUtensorMap x, al, dv, rh, bi, bj, bk;
-    CUtensorMap ec;   // INTERP: coarse correction field (box CW x CHX)
+};
+
+// INTERP: coarse correction field e_c (read through L2, it is 1/8 of the fine level)
+struct CoarseView {
+    const double* e;
+    long js, ks;
+    int zoff;   // coarse plane of fine plane 0 inside a replicated coarse part
 };
 
 __device__ __forceinline__ unsigned smem_u32(const void* p) {
@@ -327,14 +330,13 @@ template <bool RESID, bool INTERP>
 __global__ void __launch_bounds__(NT, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
-                     int czoff) {
+                     CoarseView cv) {
     constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
     double* Cs = Xs + NXS * XSLOT;                    // [NCS][NCA][CHH][W]
     double* Ks = Cs + NCS * CSLOT;                    // [NKS][CHH][W]
     unsigned long long* mbar = (unsigned long long*)(Ks + NKS * CARR);
-    double* Es = (double*)(mbar + 16);                // INTERP: [NES][CHX][CW], 128-B aligned
 
     const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
     if (tid == 0) {
@@ -352,19 +354,13 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         const int cx = SF_OX + x0 - 2;        // TMA x coordinate of the box
         const int cyx = y0, cyc = y0 + 1;     // TMA y coordinates (x box, coef box)
         const unsigned seq0 = seq;            // pre-bundle; bundle q -> seq0 + 2 + q - z0
-        const int ccx = SF_OX + x0 / 2 - 1, ccy = SF_GY + y0 / 2 - 1;  // coarse box origin
-        // INTERP: the coarse parents of x plane p travel with it (plane p>>1 of the coarse part)
-        auto issue_e = [&](int p, unsigned long long* b) {
-            if (INTERP) tma3(Es + md(p, NES) * CBOX, &mp.ec, ccx, ccy, (p >> 1) + czoff + SF_GZ, b);
-        };
 
         // bundle q: x(q+1), alpha/Dinv/rhs/beta_i/beta_j (q), beta_k(q+1); needed by R(q)
         auto issue = [&](int q) {
             unsigned sq = seq0 + 2 + (q - z0);
             unsigned long long* b = &mbar[sq % NMB];
-            mbar_expect(b, BUNDLE_BYTES + (INTERP ? CBOX_BYTES : 0));
+            mbar_expect(b, BUNDLE_BYTES);
             tma3(Xs + md(q + 1, NXS) * XSLOT, &mp.x, cx, cyx, q + 1 + SF_GZ, b);
-            issue_e(q + 1, b);
             double* c = Cs + md(q, NCS) * CSLOT;
             tma3(c + CA_AL * CARR, &mp.al, cx, cyc, q + SF_GZ, b);
             tma3(c + CA_DV * CARR, &mp.dv, cx, cyc, q + SF_GZ, b);
@@ -376,11 +372,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         if (tid == 0) {
             fence_proxy_async();  // generic smem writes of the previous item before TMA reuse
             unsigned long long* b = &mbar[seq0 % NMB];
-            mbar_expect(b, 2 * XBYTES + CBYTES + (INTERP ? 2 * CBOX_BYTES : 0));
+            mbar_expect(b, 2 * XBYTES + CBYTES);
             tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 2 + SF_GZ, b);
             tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 1 + SF_GZ, b);
-            issue_e(z0 - 2, b);
-            issue_e(z0 - 1, b);
             tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, z0 - 1 + SF_GZ, b);
             for (int q = z0 - 1; q <= min(z0 + PF - 2, z1); q++) issue(q);  // step t: t+PF+1
         }
@@ -431,25 +425,41 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         int ic = md(z0 - 1, NCS);                       // coef(t+1)
         int ik1 = md(z0 - 1, NKS), ik2 = md(z0, NKS);   // beta_k(t+1), beta_k(t+2)
         mbar_wait(&mbar[seq0 % NMB], (seq0 / NMB) & 1);
-        // INTERP (A8 P0 fused): x(p) += e_c(parent) in smem, once per plane,
-        // one step before its first read (pairs of x share a parent)
-        auto correct = [&](int p) {
+        // INTERP (A8 P0 fused): x(p) += e_c(parent) in smem, once per plane, one
+        // step before its first read; the two parents a thread needs for plane
+        // p are loaded (L2) one step earlier still.
+        const int ep0 = tid, ep1 = tid + NT;   // x-box pairs of this thread
+        auto e_addr = [&](int pr, int p) -> long {
+            const int r = pr / (W / 2), c2 = pr - r * (W / 2);
+            const int I = x0 / 2 - 1 + c2, J = y0 / 2 - 1 + (r >> 1), K = (p >> 1) + cv.zoff;
+            return (long)(K + SF_GZ) * cv.ks + (long)(J + SF_GY) * cv.js + SF_OX + I;
+        };
+        auto load_e = [&](int p, double& e0, double& e1) {
+            e0 = __ldg(cv.e + e_addr(ep0, p));
+            e1 = (ep1 < XPAIRS) ? __ldg(cv.e + e_addr(ep1, p)) : 0.0;
+        };
+        auto correct = [&](int p, double e0, double e1) {
             double* X = Xs + md(p, NXS) * XSLOT;
-            const double* E = Es + md(p, NES) * CBOX;
-            for (int i = tid; i < XH * (W / 2); i += NT) {
-                const int r = i / (W / 2), c2 = i - r * (W / 2);
-                const double e = E[(r >> 1) * CW + c2];
-                double2 v = *(double2*)&X[r * W + 2 * c2];
-                v.x = v.x + e;
-                v.y = v.y + e;
-                *(double2*)&X[r * W + 2 * c2] = v;
+            double2 v = *(double2*)&X[2 * ep0];
+            v.x = v.x + e0;
+            v.y = v.y + e0;
+            *(double2*)&X[2 * ep0] = v;
+            if (ep1 < XPAIRS) {
+                double2 u = *(double2*)&X[2 * ep1];
+                u.x = u.x + e1;
+                u.y = u.y + e1;
+                *(double2*)&X[2 * ep1] = u;
             }
         };
+        double ce0 = 0.0, ce1 = 0.0;   // parents for the next plane to correct
         if (INTERP) {
             mbar_wait(&mbar[(seq0 + 1) % NMB], ((seq0 + 1) / NMB) & 1);   // bundle z0-1: x(z0)
-            correct(z0 - 2);
-            correct(z0 - 1);
-            correct(z0);
+            for (int p = z0 - 2; p <= z0; p++) {
+                double e0, e1;
+                load_e(p, e0, e1);
+                correct(p, e0, e1);
+            }
+            if (z0 + 1 <= z1 + 1) load_e(z0 + 1, ce0, ce1);
             __syncthreads();
         }
 
@@ -463,7 +473,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             if (INTERP && q + 1 <= z1) {   // bundle t+2 (x(t+3)) one step early, corrected now
                 const unsigned sq = seq0 + 2 + (q + 1 - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
-                correct(t + 3);
+                correct(t + 3, ce0, ce1);
+                if (t + 4 <= z1 + 1) load_e(t + 4, ce0, ce1);
             }
             const int gkr = g.z0 + q;                    // plane of R
             const bool rin = q <= z1 && gkr >= 0 && gkr < g.gnz;
@@ -608,8 +619,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<true, false>,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, true>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)SMEM_INTERP));
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
         SF_CUDA(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
@@ -646,23 +656,11 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
         int grid = std::min(items, G);
-        int czoff = 0;
+        CoarseView cvw{nullptr, 0, 0, 0};
         if (C) {
             const bool rep = C->nparts == 1 && L->nparts > 1;
-            PV cv = sf_view(C, rep ? 0 : p);
-            czoff = rep ? v.z0 / 2 : 0;
-            cuuint64_t dims[3] = {(cuuint64_t)C->js, (cuuint64_t)(C->ny + 2 * SF_GY),
-                                  (cuuint64_t)(C->lnz + 2 * SF_GZ)};
-            cuuint64_t strides[2] = {(cuuint64_t)C->js * 8, (cuuint64_t)C->ks * 8};
-            cuuint32_t box[3] = {(cuuint32_t)CW, (cuuint32_t)CHX, 1};
-            cuuint32_t es[3] = {1, 1, 1};
-            CUresult r = g_encode(&mp.ec, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)cv.f[cf], dims,
-                                  strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                  CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-            if (r != CUDA_SUCCESS) return sf_fail(SF_ERR_CUDA, "coarse tensor map (%d)", (int)r);
-        } else {
-            mp.ec = mp.x;
+            PV c = sf_view(C, rep ? 0 : p);
+            cvw = CoarseView{c.f[cf], C->js, C->ks, rep ? v.z0 / 2 : 0};
         }
         if (rmax) {
             if (p == 0) {
@@ -670,13 +668,13 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
                 SF_LAUNCHED();
             }
             gsrb_pair_tma_kernel<true, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax, 0);
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax, cvw);
         } else if (C) {
-            gsrb_pair_tma_kernel<false, true><<<grid, NT, SMEM_INTERP, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, czoff);
+            gsrb_pair_tma_kernel<false, true><<<grid, NT, SMEM, L->stream>>>(
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw);
         } else {
             gsrb_pair_tma_kernel<false, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, 0);
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw);
         }
         SF_LAUNCHED();
     }
