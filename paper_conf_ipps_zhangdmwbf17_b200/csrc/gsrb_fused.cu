@@ -125,33 +125,33 @@ __device__ __forceinline__ void fence_proxy_async() {
 
 __device__ __forceinline__ int md(int k, int m) { return ((k % m) + m) % m; }
 
-// x <- x + Dinv (rhs - Ax); operator in the term order of op_at (kernels.cu)
+// x <- x + Dinv (rhs - Ax).  The six face fluxes are summed as a tree (depth 4
+// instead of 7 dependent FP64 ops: this kernel is latency-bound per plane
+// step); the result differs from op_at's sequential order only in rounding.
+__device__ __forceinline__ double flux6(double xc, double xw, double xe, double xs, double xn,
+                                       double xb, double xt, double bw, double be, double bs,
+                                       double bn, double bb, double bt) {
+    const double fx = be * (xe - xc) + bw * (xw - xc);
+    const double fy = bn * (xn - xc) + bs * (xs - xc);
+    const double fz = bt * (xt - xc) + bb * (xb - xc);
+    return (fx + fy) + fz;
+}
+
 __device__ __forceinline__ double gs_update(double xc, double xw, double xe, double xs, double xn,
                                             double xb, double xt, double bw, double be, double bs,
                                             double bn, double bb, double bt, double al, double dv,
                                             double rh, double a, double bh2) {
-    double flux = be * (xe - xc);
-    flux += bw * (xw - xc);
-    flux += bn * (xn - xc);
-    flux += bs * (xs - xc);
-    flux += bt * (xt - xc);
-    flux += bb * (xb - xc);
-    double ax = a * al * xc - bh2 * flux;
+    const double flux = flux6(xc, xw, xe, xs, xn, xb, xt, bw, be, bs, bn, bb, bt);
+    const double ax = a * al * xc - bh2 * flux;
     return xc + dv * (rh - ax);
 }
 
-// A x at one cell (op_at term order); used for the fused input residual
+// A x at one cell (same tree as gs_update); used for the fused input residual
 __device__ __forceinline__ double ax_at(double xc, double xw, double xe, double xs, double xn,
                                        double xb, double xt, double bw, double be, double bs,
                                        double bn, double bb, double bt, double al, double a,
                                        double bh2) {
-    double flux = be * (xe - xc);
-    flux += bw * (xw - xc);
-    flux += bn * (xn - xc);
-    flux += bs * (xs - xc);
-    flux += bt * (xt - xc);
-    flux += bb * (xb - xc);
-    return a * al * xc - bh2 * flux;
+    return a * al * xc - bh2 * flux6(xc, xw, xe, xs, xn, xb, xt, bw, be, bs, bn, bb, bt);
 }
 
 __device__ __forceinline__ unsigned long long abits(double v) {
@@ -191,17 +191,12 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
     double2 bkl = *(const double2*)&s.Klo[co_];
     double2 bkh = *(const double2*)&s.Khi[co_];
-    double bie = __shfl_down_sync(0xffffffffu, bi2.x, 1, PPR);
-    if (lane == PPR - 1) bie = s.C[CA_BI * CARR + co_ + 2];
+    const double bie = s.C[CA_BI * CARR + co_ + 2];   // east face of the odd cell
     double xc, xw, xe;
     if (SEL == 0) {
-        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1, PPR);
-        if (lane == 0) xl = s.Xk[xo_ - 1];
-        xc = xp2.x; xw = xl; xe = xp2.y;
+        xc = xp2.x; xw = s.Xk[xo_ - 1]; xe = xp2.y;
     } else {
-        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1, PPR);
-        if (lane == PPR - 1) xr = s.Xk[xo_ + 2];
-        xc = xp2.y; xw = xp2.x; xe = xr;
+        xc = xp2.y; xw = xp2.x; xe = s.Xk[xo_ + 2];
     }
     const int gxr = gx + SEL;
     if (gxr == 0) xw = -xc;
@@ -253,13 +248,9 @@ __device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int lan
                                               double2 xp2) {
     double xc, xw, xe;
     if (BS == 1) {
-        double xr = __shfl_down_sync(0xffffffffu, xp2.x, 1, PPR);
-        if (lane == PPR - 1) xr = s.Xk[xo_ + 2];
-        xc = xp2.y; xw = xp2.x; xe = xr;
+        xc = xp2.y; xw = xp2.x; xe = s.Xk[xo_ + 2];
     } else {
-        double xl = __shfl_up_sync(0xffffffffu, xp2.y, 1, PPR);
-        if (lane == 0) xl = s.Xk[xo_ - 1];
-        xc = xp2.x; xw = xl; xe = xp2.y;
+        xc = xp2.x; xw = s.Xk[xo_ - 1]; xe = xp2.y;
     }
     const int gxb = gx + BS;
     if (gxb == 0) xw = -xc;
@@ -282,13 +273,9 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int lan
     double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
     double xc, xw, xe;
     if (SEL == 0) {
-        double ql = __shfl_up_sync(0xffffffffu, q2.y, 1, PPR);
-        if (lane == 0) ql = s.Xm[xo_ - 1];
-        xc = q2.x; xw = ql; xe = q2.y;
+        xc = q2.x; xw = s.Xm[xo_ - 1]; xe = q2.y;
     } else {
-        double qr = __shfl_down_sync(0xffffffffu, q2.x, 1, PPR);
-        if (lane == PPR - 1) qr = s.Xm[xo_ + 2];
-        xc = q2.y; xw = q2.x; xe = qr;
+        xc = q2.y; xw = q2.x; xe = s.Xm[xo_ + 2];
     }
     const int gxb = gx + SEL;
     if (gxb == 0) xw = -xc;

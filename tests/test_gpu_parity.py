@@ -128,7 +128,7 @@ def test_fused_equals_colour(sf):
         L.upload(sf.SF_F, I.random_field(shape, 1))
         sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, k)
         outs.append(L.download(sf.SF_U))
-    assert rel(outs[1], outs[0]) < 1e-14
+    assert rel(outs[1], outs[0]) < 1e-13   # fused sums the fluxes as a tree
 
 
 def test_c1_config(sf, oracle):
