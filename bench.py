@@ -298,7 +298,7 @@ def main():
             "roofline": roof,
         }
         line.update({k: v for k, v in side.items() if k in ("e2e", "gsrb_c3", "vcycle",
-                                                             "cpu_baseline")})
+                                                             "cpu_baseline", "fig7_256")})
         print(json.dumps(line), flush=True)
     M.close()
     L.close()
@@ -394,6 +394,31 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
         b.record(s)
         s.synchronize()
         msc = a.elapsed_time(b) / 20
+        # Fig 7 analogue: the paper's three operators at 256^3,
+        # GPU algorithmic bytes (no write-allocate): CC 7pt 16 B, CC Jacobi 24 B,
+        # VC GSRB 64 B per cell per RB pair (paper's write-allocate counts: 24/40/64)
+        def per_call(fn, reps=50):
+            for _ in range(5):
+                fn()
+            s.synchronize()
+            a.record(s)
+            for _ in range(reps):
+                fn()
+            b.record(s)
+            s.synchronize()
+            return a.elapsed_time(b) / reps
+        fig7 = {}
+        for name, fn, bpc in (
+                ("cc_7pt_laplacian", lambda: sf.sf_apply_laplacian(G.handle, sf.SF_R, sf.SF_U), 16),
+                ("cc_jacobi_w2/3", lambda: sf.sf_jacobi(G.handle, sf.SF_R, sf.SF_U, sf.SF_F,
+                                                         2.0 / 3.0), 24)):
+            m_ = per_call(fn)
+            fig7[name] = {"ms": m_, "gstencil_s": cells / (m_ / 1e3) / 1e9,
+                          "alg_gbs": bpc * cells / (m_ / 1e3) / 1e9,
+                          "frac_of_peak": bpc * cells / (m_ / 1e3) / 1e9 / pk, "bytes_per_cell": bpc}
+        fig7["vc_gsrb_pair"] = {"ms": ms, "gstencil_s": cells / (ms / 1e3) / 1e9, "alg_gbs": gbs,
+                                "frac_of_peak": gbs / pk, "bytes_per_cell": 64}
+        out["fig7_256"] = fig7
         out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms, "gstencil_s": 2 * cells / 2 / (ms / 1e3) / 1e9,
                           "point_updates_per_s": cells / (ms / 1e3),
                           "alg_gbs": gbs, "frac_of_peak": gbs / pk,

@@ -178,6 +178,15 @@ sf_status sf_restrict(sf_level* coarse, int c_field, sf_level* fine, int f_field
  * coarse field's ghosts (A2) first. */
 sf_status sf_interpolate(sf_level* fine, int f_field, double prescale,
                          sf_level* coarse, int c_field, int kind);
+/* NEXT-2, the other two operators of the paper's Fig 7:
+ * sf_apply_laplacian: out = L x, the canonical constant-coefficient 7-point
+ *   Laplacian h^-2 * sum_n (x(c) - x(n)) with the Dirichlet fold (A3 with a = 0,
+ *   b = 1, beta = 1, but no coefficient array is read).  out != x.
+ * sf_jacobi: out = x + omega * D^-1 (f - L x), D = diag(L) with the fold
+ *   (reading R-11: omega = 2/3 in the paper).  Out of place: out != x, f.
+ * Both need an even gnx (SF_ERR_SHAPE otherwise). */
+sf_status sf_apply_laplacian(sf_level* level, int out, int x);
+sf_status sf_jacobi(sf_level* level, int out, int x, int f, double omega);
 /* A10: norm of the interior over all parts/ranks; syncs. */
 sf_status sf_norm(sf_level* level, int field, int kind, double* out);
 sf_status sf_sync(sf_level* level);

@@ -524,3 +524,45 @@ void or_gsrb_pair_points(const or_grid* g, double a, double b, const double* alp
             if (in[d]) x[at[d]] = ov[d];
     }
 }
+
+/* ------------------------------------------------------------------------ */
+/* NEXT-2 (Fig 7's other two operators, Sec. V.A):         */
+/* the canonical 7-point constant-coefficient Laplacian                      */
+/*   L x(c) = h^-2 * sum_{6 neighbours n} (x(c) - x(n))                      */
+/* (A3 with a = 0, b = 1, beta = 1; ghosts from A2), and the weighted Jacobi */
+/* smoother x <- x + (2/3) D^-1 (f - L x) (garbled "2/3 D^-1", reading R-11),*/
+/* D = diag(L) with the Dirichlet fold (a boundary face adds 2/h^2).         */
+/* ------------------------------------------------------------------------ */
+static double lap_at(const or_grid* g, const double* x, int i, int j, int k) {
+    double hm2 = 1.0 / (g->h * g->h);
+    double xc = x[OIDX(g, i, j, k)];
+    double s = 0.0;
+    s += xc - x[OIDX(g, i + 1, j, k)];
+    s += xc - x[OIDX(g, i - 1, j, k)];
+    s += xc - x[OIDX(g, i, j + 1, k)];
+    s += xc - x[OIDX(g, i, j - 1, k)];
+    s += xc - x[OIDX(g, i, j, k + 1)];
+    s += xc - x[OIDX(g, i, j, k - 1)];
+    return hm2 * s;
+}
+
+void or_laplacian_cc(const or_grid* g, double* x, double* out) {
+    or_apply_bc(g, x);
+    for (int k = 0; k < g->nz; k++)
+        for (int j = 0; j < g->ny; j++)
+            for (int i = 0; i < g->nx; i++) out[OIDX(g, i, j, k)] = lap_at(g, x, i, j, k);
+}
+
+void or_jacobi_cc(const or_grid* g, double omega, double* x, const double* f, double* out) {
+    double hm2 = 1.0 / (g->h * g->h);
+    or_apply_bc(g, x);
+    for (int k = 0; k < g->nz; k++)
+        for (int j = 0; j < g->ny; j++)
+            for (int i = 0; i < g->nx; i++) {
+                int nb = (i == 0) + (i == g->nx - 1) + (j == 0) + (j == g->ny - 1) + (k == 0) +
+                         (k == g->nz - 1);
+                double d = hm2 * (6.0 + nb);
+                size_t c = OIDX(g, i, j, k);
+                out[c] = x[c] + omega * (f[c] - lap_at(g, x, i, j, k)) / d;
+            }
+}

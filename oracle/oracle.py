@@ -72,6 +72,8 @@ def lib():
             "or_mg_fcycle": (C.c_int, [C.c_void_p, _P, _P]),
             "or_mg_relres": (d, [C.c_void_p, _P, _P]),
             "or_mg_solve": (C.c_int, [C.c_void_p, _P, _P, C.c_int, d, C.c_int, _P]),
+            "or_laplacian_cc": (None, [G, _P, _P]),
+            "or_jacobi_cc": (None, [G, d, _P, _P, _P]),
             "or_residual_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP, _IP,
                                           _P]),
             "or_gsrb_pair_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP,
@@ -230,6 +232,24 @@ def interpolate(fine, coarse, prescale, kind="p0"):
     fn = lib().or_interp_p0 if kind == "p0" else lib().or_interp_pl
     fn(gf.ref, _ptr(fp), float(prescale), gc.ref, _ptr(cp))
     return interior(fp)
+
+
+def laplacian_cc(x, h):
+    """NEXT-2: constant-coefficient 7-point Laplacian (Fig 7)."""
+    nz, ny, nx = x.shape
+    g = Grid(nx, ny, nz, h)
+    xp, out = pad(x), np.zeros((nz + 2, ny + 2, nx + 2))
+    lib().or_laplacian_cc(g.ref, _ptr(xp), _ptr(out))
+    return interior(out)
+
+
+def jacobi_cc(x, f, h, omega=2.0 / 3.0):
+    """NEXT-2: weighted Jacobi x + omega D^-1 (f - L x) (R-11)."""
+    nz, ny, nx = x.shape
+    g = Grid(nx, ny, nz, h)
+    xp, fp, out = pad(x), pad(f), np.zeros((nz + 2, ny + 2, nx + 2))
+    lib().or_jacobi_cc(g.ref, float(omega), _ptr(xp), _ptr(fp), _ptr(out))
+    return interior(out)
 
 
 def norm(x, kind="max"):

@@ -178,6 +178,58 @@ __global__ void __launch_bounds__(PX* PY) norm_pair_kernel(PV v, const double* _
     }
 }
 
+// NEXT-2 (Fig 7): constant-coefficient 7-point Laplacian
+// L x = h^-2 sum_n (x_c - x_n) (Dirichlet fold: a boundary neighbour is -x_c),
+// and weighted Jacobi out = x + w D^-1 (f - L x), D^-1 = h^2 / (6 + boundary
+// faces) computed on the fly.  Streams x only (Laplacian: 16 B/cell) or x, f
+// (Jacobi: 24 B/cell); no coefficient arrays.
+template <bool JACOBI>
+__global__ void __launch_bounds__(PX* PY) cc_pair_kernel(PV v, double* __restrict__ out,
+                                                          const double* __restrict__ x,
+                                                          const double* __restrict__ f,
+                                                          double hm2, double h2w, int depth) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    if (i >= v.nx || j >= v.ny) return;
+    for (int k = k0; k < k1; k++) {
+        const long c = sf_ix(v, i, j, k);
+        const int gk = v.z0 + k;
+        const double2 xc = ld2(x + c);
+        double xw = (i == 0) ? -xc.x : x[c - 1];
+        double xe = (i + 1 == v.nx - 1) ? -xc.y : x[c + 2];
+        double2 xs = ld2(x + c - v.js), xn = ld2(x + c + v.js);
+        double2 xb = ld2(x + c - v.ks), xt = ld2(x + c + v.ks);
+        if (j == 0) xs = make_double2(-xc.x, -xc.y);
+        if (j == v.ny - 1) xn = make_double2(-xc.x, -xc.y);
+        if (gk == 0) xb = make_double2(-xc.x, -xc.y);
+        if (gk == v.gnz - 1) xt = make_double2(-xc.x, -xc.y);
+        double sa = xc.x - xc.y;
+        sa += xc.x - xw;
+        sa += xc.x - xn.x;
+        sa += xc.x - xs.x;
+        sa += xc.x - xt.x;
+        sa += xc.x - xb.x;
+        double sb = xc.y - xe;
+        sb += xc.y - xc.x;
+        sb += xc.y - xn.y;
+        sb += xc.y - xs.y;
+        sb += xc.y - xt.y;
+        sb += xc.y - xb.y;
+        double2 o;
+        if (JACOBI) {
+            const int nyz = (j == 0) + (j == v.ny - 1) + (gk == 0) + (gk == v.gnz - 1);
+            const double2 fv = ld2(f + c);
+            const double da = 6.0 + nyz + (i == 0), db = 6.0 + nyz + (i + 1 == v.nx - 1);
+            o.x = xc.x + h2w * (fv.x - hm2 * sa) / da;
+            o.y = xc.y + h2w * (fv.y - hm2 * sb) / db;
+        } else {
+            o.x = hm2 * sa;
+            o.y = hm2 * sb;
+        }
+        *(double2*)(out + c) = o;
+    }
+}
+
 __global__ void zero_scalar(double* p) { *p = 0.0; }
 
 // grid over pairs: (ceil(nx/64), ceil(ny/4), z-chunks) with ~16 blocks per SM
@@ -248,6 +300,25 @@ sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf) {
         SF_LAUNCHED();
     }
     return sf_check_launch("interp_p0_pair");
+}
+
+sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi) {
+    if (!pair_ok(L)) return sf_fail(SF_ERR_SHAPE, "CC kernels need an even nx");
+    SF_TRY(sf_halo(L, x, 1));
+    const double hm2 = 1.0 / (L->h * L->h), h2w = omega * L->h * L->h;
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        if (jacobi)
+            cc_pair_kernel<true><<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], v.f[f], hm2,
+                                                                     h2w, depth);
+        else
+            cc_pair_kernel<false><<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], nullptr,
+                                                                      hm2, h2w, depth);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("cc_pair");
 }
 
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst) {

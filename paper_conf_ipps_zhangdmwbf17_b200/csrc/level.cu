@@ -260,6 +260,23 @@ extern "C" sf_status sf_apply_op(sf_level* L, int out, int x, double a, double b
     return k_apply_op(L, out, x, a, b);
 }
 
+extern "C" sf_status sf_apply_laplacian(sf_level* L, int out, int x) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(out));
+    SF_TRY(check_field(x));
+    if (out == x) return sf_fail(SF_ERR_INVALID, "out must differ from x");
+    return k_cc(L, out, x, -1, 0.0, false);
+}
+
+extern "C" sf_status sf_jacobi(sf_level* L, int out, int x, int f, double omega) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(out));
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(f));
+    if (out == x || out == f) return sf_fail(SF_ERR_INVALID, "out must differ from x and f");
+    return k_cc(L, out, x, f, omega, true);
+}
+
 extern "C" sf_status sf_residual(sf_level* L, int res, int x, int rhs, double a, double b) {
     if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
     SF_TRY(check_field(res));

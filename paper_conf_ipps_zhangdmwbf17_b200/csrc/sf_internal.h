@@ -110,6 +110,7 @@ sf_status k_residual_pair(sf_level* L, int res /* -1: do not write */, int x, in
 sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf);
 sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf);
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
+sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi);  // NEXT-2
 
 // fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
 bool gsrb_fused_supported_t32(const sf_level* L);

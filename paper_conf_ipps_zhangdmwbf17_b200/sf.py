@@ -41,6 +41,7 @@ EXPORTS = [
     "sf_apply_bc", "sf_apply_op", "sf_smooth_gsrb", "sf_residual", "sf_restrict",
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
+    "sf_apply_laplacian", "sf_jacobi",
 ]
 
 
@@ -92,6 +93,8 @@ def lib():
         "sf_apply_op": (_i, [_vp, _i, _i, _d, _d]),
         "sf_smooth_gsrb": (_i, [_vp, _i, _i, _d, _d, _i, _i]),
         "sf_residual": (_i, [_vp, _i, _i, _i, _d, _d]),
+        "sf_apply_laplacian": (_i, [_vp, _i, _i]),
+        "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
         "sf_restrict": (_i, [_vp, _i, _vp, _i, _i]),
         "sf_interpolate": (_i, [_vp, _i, _d, _vp, _i, _i]),
         "sf_norm": (_i, [_vp, _i, _i, _P]),
@@ -202,6 +205,14 @@ def sf_apply_op(level, out, x, a, b):
 
 def sf_smooth_gsrb(level, x, rhs, a, b, rb_pairs, kind=SF_SMOOTH_AUTO):
     _check(lib().sf_smooth_gsrb(level, x, rhs, float(a), float(b), int(rb_pairs), int(kind)))
+
+
+def sf_apply_laplacian(level, out, x):
+    _check(lib().sf_apply_laplacian(level, out, x))
+
+
+def sf_jacobi(level, out, x, f, omega=2.0 / 3.0):
+    _check(lib().sf_jacobi(level, out, x, f, float(omega)))
 
 
 def sf_residual(level, res, x, rhs, a, b):

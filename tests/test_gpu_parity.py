@@ -364,3 +364,33 @@ def test_solve_max_cycles_keeps_last_cycle(sf, oracle, use_graph):
         u = O.vcycle(u, f)
     assert rel(L.download(sf.SF_U), u) < 1e-11
     assert abs(hist[-1] / O.relres(u, f) - 1) < 1e-6
+
+
+# ------------------------------------------------------- NEXT-2 (Fig 7 operators)
+@pytest.mark.parametrize("shape", [(16, 16, 16), (8, 6, 10), (20, 64, 64), (33, 12, 40)])
+def test_cc_laplacian_and_jacobi(sf, oracle, shape):
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    L = sf.Level(nx, ny, nz, h)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    sf.sf_apply_laplacian(L.handle, sf.SF_R, sf.SF_U)
+    assert rel(L.download(sf.SF_R), oracle.laplacian_cc(x, h)) < TOL
+    sf.sf_jacobi(L.handle, sf.SF_TMP, sf.SF_U, sf.SF_F, 2.0 / 3.0)
+    assert rel(L.download(sf.SF_TMP), oracle.jacobi_cc(x, f, h)) < TOL
+
+
+def test_cc_decomposition_invariance(sf):
+    shape = (32, 16, 32)
+    nz, ny, nx = shape
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    outs = []
+    for P in (1, 4):
+        comm = sf.Comm.local(P) if P > 1 else None
+        L = sf.Level(nx, ny, nz, comm=comm)
+        L.upload(sf.SF_U, x)
+        L.upload(sf.SF_F, f)
+        sf.sf_jacobi(L.handle, sf.SF_TMP, sf.SF_U, sf.SF_F, 2.0 / 3.0)
+        outs.append(L.download(sf.SF_TMP))
+    assert np.array_equal(outs[0], outs[1])

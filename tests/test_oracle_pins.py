@@ -412,3 +412,37 @@ def test_point_evaluations_match_whole_grid(oracle):
     assert np.array_equal(P.residual_points(x, f, pts), r[pts[2], pts[1], pts[0]])
     s = P.smooth(x, f, 1)
     assert np.array_equal(P.gsrb_pair_points(x, f, pts), s[pts[2], pts[1], pts[0]])
+
+
+# ------------------------------------------------------- NEXT-2 (Fig 7 operators)
+def _kron_laplacian(nx, ny, nz, h):
+    def T(n):
+        t = (2 * np.eye(n) - np.eye(n, k=1) - np.eye(n, k=-1))
+        t[0, 0] = t[-1, -1] = 3
+        return t / h**2
+    return (np.kron(np.eye(nz), np.kron(np.eye(ny), T(nx)))
+            + np.kron(np.eye(nz), np.kron(T(ny), np.eye(nx)))
+            + np.kron(T(nz), np.kron(np.eye(ny), np.eye(nx))))
+
+
+def test_cc_laplacian_is_textbook_matrix(oracle):
+    """The CC 7-point Laplacian with the Dirichlet fold is the Kronecker sum of
+    tridiag(-1,2,-1)/h^2 with end diagonals 3/h^2."""
+    nz, ny, nx, h = 5, 3, 4, 0.25
+    K = _kron_laplacian(nx, ny, nz, h)
+    x = I.random_field((nz, ny, nx), 4)
+    got = oracle.laplacian_cc(x, h)
+    assert np.abs(got.ravel() - K @ x.ravel()).max() < 1e-12 * np.abs(K @ x.ravel()).max()
+
+
+def test_cc_jacobi_brute_force(oracle):
+    """x + (2/3) D^-1 (f - L x) with dense L and D = diag(L) (reading R-11)."""
+    nz, ny, nx, h = 4, 5, 6, 0.2
+    K = _kron_laplacian(nx, ny, nz, h)
+    x, f = I.random_field((nz, ny, nx), 0), I.random_field((nz, ny, nx), 1)
+    exp = x.ravel() + (2.0 / 3.0) * (f.ravel() - K @ x.ravel()) / np.diag(K)
+    got = oracle.jacobi_cc(x, f, h)
+    assert np.abs(got.ravel() - exp).max() < 1e-12 * np.abs(exp).max()
+    # the damped Jacobi iteration converges (spectral radius < 1 for SPD L, omega 2/3)
+    Jm = np.eye(K.shape[0]) - (2.0 / 3.0) * K / np.diag(K)[:, None]
+    assert np.abs(np.linalg.eigvals(Jm)).max() < 1.0
