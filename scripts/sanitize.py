@@ -1,0 +1,24 @@
+"""Small end-to-end workload for compute-sanitizer: fused pair variants (plain,
+check-fused, P0-fused), colour sweeps, residual/restriction, CC kernels, and a
+32^3 / 64^3 solve (graphs off so every launch is visible)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I, sf  # noqa: E402
+
+for n, parts in ((32, 1), (64, 1), (64, 2)):
+    comm = sf.Comm.local(parts) if parts > 1 else None
+    L = sf.Level(n, n, n, 1.0 / n, comm=comm)
+    sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
+    M = sf.MG(L, 1.0, 1.0, use_graph=0, agglom_min_planes=4)
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, max_cycles=3, raise_on_error=False)
+    sf.sf_apply_laplacian(L.handle, sf.SF_R, sf.SF_U)
+    sf.sf_jacobi(L.handle, sf.SF_TMP, sf.SF_U, sf.SF_F)
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_COLOUR)
+    sf.sf_apply_bc(L.handle, sf.SF_U)
+    sf.sf_sync(L.handle)
+    print("ok", n, parts, cyc, flush=True)
+    M.close(); L.close()
+    if comm:
+        comm.close()
