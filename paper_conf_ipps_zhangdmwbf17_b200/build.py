@@ -22,9 +22,9 @@ LIB = os.path.join(PKG, "libsf.so")
 SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            ("kernels_pair.cu", "kernels_pair.o", []),
            ("gsrb_fused.cu", "gsrb_fused_t32.o",
-            ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t32"]),
+            ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=5", "-DSF_GSRB_SUFFIX=_t32"]),
            ("gsrb_fused.cu", "gsrb_fused_t64.o",
-            ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=3", "-DSF_GSRB_SUFFIX=_t64"]),
+            ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t64"]),
            ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

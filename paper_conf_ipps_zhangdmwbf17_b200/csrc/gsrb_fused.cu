@@ -49,7 +49,7 @@ namespace {
 #define SF_GSRB_TX 32
 #endif
 #ifndef SF_GSRB_PF
-#define SF_GSRB_PF 4
+#define SF_GSRB_PF 5
 #endif
 #ifndef SF_GSRB_SUFFIX
 #define SF_GSRB_SUFFIX _t32
@@ -66,7 +66,7 @@ constexpr int XH = TY + 4;             // x rows:   gy in [y0-2, y0+TY+2)
 constexpr int CHH = TY + 3;            // coef rows: gy in [y0-1, y0+TY+2)
 constexpr int PF = SF_GSRB_PF;         // bundles in flight ahead of the one being consumed
 constexpr int NXS = 5 + PF, NCS = 1 + PF, NKS = 2 + PF, NMB = PF + 2;  // slot counts
-constexpr int NCA = 5;                 // staged coefficient arrays per plane (beta_k separate)
+constexpr int NCA = 4;                 // staged coefficient arrays per plane (beta_k separate)
 constexpr int XSLOT = (XH * W + 15) / 16 * 16;   // doubles, 128-byte multiple
 constexpr int CARR = (CHH * W + 15) / 16 * 16;
 constexpr int CSLOT = NCA * CARR;
@@ -78,11 +78,11 @@ constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR
 constexpr int XPAIRS = XH * (W / 2);
 static_assert(XPAIRS <= 2 * NT, "two correction pairs per thread");
 static_assert(TX % 2 == 0 && 32 % PPR == 0, "tile shape");
-enum { CA_AL = 0, CA_DV = 1, CA_RH = 2, CA_BI = 3, CA_BJ = 4 };
+enum { CA_DV = 0, CA_RH = 1, CA_BI = 2, CA_BJ = 3 };
 constexpr int NRING = TX + TY;         // red ring cells per plane (half of the 1-ring)
 
 struct Maps {
-    CUtensorMap x, al, dv, rh, bi, bj, bk;
+    CUtensorMap x, dv, rh, bi, bj, bk;
 };
 
 // INTERP: coarse correction field e_c (read through L2, it is 1/8 of the fine level)
@@ -125,33 +125,21 @@ __device__ __forceinline__ void fence_proxy_async() {
 
 __device__ __forceinline__ int md(int k, int m) { return ((k % m) + m) % m; }
 
-// x <- x + Dinv (rhs - Ax).  The six face fluxes are summed as a tree (depth 4
-// instead of 7 dependent FP64 ops: this kernel is latency-bound per plane
-// step); the result differs from op_at's sequential order only in rounding.
-__device__ __forceinline__ double flux6(double xc, double xw, double xe, double xs, double xn,
-                                       double xb, double xt, double bw, double be, double bs,
-                                       double bn, double bb, double bt) {
-    const double fx = be * (xe - xc) + bw * (xw - xc);
-    const double fy = bn * (xn - xc) + bs * (xs - xc);
-    const double fz = bt * (xt - xc) + bb * (xb - xc);
-    return (fx + fy) + fz;
-}
-
-__device__ __forceinline__ double gs_update(double xc, double xw, double xe, double xs, double xn,
-                                            double xb, double xt, double bw, double be, double bs,
-                                            double bn, double bb, double bt, double al, double dv,
-                                            double rh, double a, double bh2) {
-    const double flux = flux6(xc, xw, xe, xs, xn, xb, xt, bw, be, bs, bn, bb, bt);
-    const double ax = a * al * xc - bh2 * flux;
-    return xc + dv * (rh - ax);
-}
-
-// A x at one cell (same tree as gs_update); used for the fused input residual
-__device__ __forceinline__ double ax_at(double xc, double xw, double xe, double xs, double xn,
-                                       double xb, double xt, double bw, double be, double bs,
-                                       double bn, double bb, double bt, double al, double a,
-                                       double bh2) {
-    return a * al * xc - bh2 * flux6(xc, xw, xe, xs, xn, xb, xt, bw, be, bs, bn, bb, bt);
+// Gauss-Seidel update in lambda-form.  With lambda = Dinv the EXACT inverse
+// diagonal of A including the Dirichlet fold (reading R-4),
+//     x + lambda (rhs - A x)  ==  lambda (rhs + b h^-2 S),
+//     S = sum over the cell's interior faces of beta_f * x(nbr_f),
+// because A x = D x(c) - b h^-2 S (a boundary face's ghost term -2 beta x(c)
+// is part of D).  The smoother therefore never reads alpha: 56 instead of the
+// 64 compulsory bytes of PAPER.md:669-672.  Boundary neighbours enter S as 0.
+// S is summed as a tree (depth 3): the per-plane step is latency-bound.
+__device__ __forceinline__ double sum6(double xw, double xe, double xs, double xn, double xb,
+                                      double xt, double bw, double be, double bs, double bn,
+                                      double bb, double bt) {
+    const double sx = be * xe + bw * xw;
+    const double sy = bn * xn + bs * xs;
+    const double sz = bt * xt + bb * xb;
+    return (sx + sy) + sz;
 }
 
 __device__ __forceinline__ unsigned long long abits(double v) {
@@ -177,62 +165,55 @@ struct StepCtx {
 // R(p) for the pair at smem offsets (xo_: x box, co_: coef box).  SEL = 1 if
 // the odd cell of the pair is red at this plane (warp-uniform).  Returns the
 // red-new value; leaves the black cell's coefficients of plane p in nb.
+// R for the pair at smem offsets (xo_: x box, co_: coef box).  SEL = 1 if
+// the odd cell of the pair is red at this plane (warp-uniform).  Returns the
+// red-new value; leaves the black cell's coefficients of the plane in nb
+// (bw, be, bs, bn, bb, bt, dinv, rhs).  RESID: rres = rhs - A x_in at the red
+// cell (A x = x(c)/dinv - b h^-2 S), rold = its old value, xpair = old pair.
 template <int SEL, bool RESID>
 __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
-                                           int gy, const Geo& g, bool zlo, bool zhi, double a,
-                                           double bh2, double* nb, double& rres, double& rold,
-                                           double2& xpair) {
-    double2 xp2 = *(const double2*)&s.Xk[xo_];
-    double2 al2 = *(const double2*)&s.C[CA_AL * CARR + co_];
-    double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
-    double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
-    double2 bi2 = *(const double2*)&s.C[CA_BI * CARR + co_];
-    double2 bjl = *(const double2*)&s.C[CA_BJ * CARR + co_];
-    double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
-    double2 bkl = *(const double2*)&s.Klo[co_];
-    double2 bkh = *(const double2*)&s.Khi[co_];
+                                           int gy, const Geo& g, bool zlo, bool zhi, double bh2,
+                                           double* nb, double& rres, double& rold, double2& xpair) {
+    const double2 xp2 = *(const double2*)&s.Xk[xo_];
+    const double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
+    const double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
+    const double2 bi2 = *(const double2*)&s.C[CA_BI * CARR + co_];
+    const double2 bjl = *(const double2*)&s.C[CA_BJ * CARR + co_];
+    const double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
+    const double2 bkl = *(const double2*)&s.Klo[co_];
+    const double2 bkh = *(const double2*)&s.Khi[co_];
     const double bie = s.C[CA_BI * CARR + co_ + 2];   // east face of the odd cell
-    double xc, xw, xe;
+    const int col = xo_ + SEL;
+    double xw, xe;
     if (SEL == 0) {
-        xc = xp2.x; xw = s.Xk[xo_ - 1]; xe = xp2.y;
+        xw = s.Xk[xo_ - 1]; xe = xp2.y;
     } else {
-        xc = xp2.y; xw = xp2.x; xe = s.Xk[xo_ + 2];
+        xw = xp2.x; xe = s.Xk[xo_ + 2];
     }
     const int gxr = gx + SEL;
-    if (gxr == 0) xw = -xc;
-    if (gxr == g.nx - 1) xe = -xc;
-    const int col = xo_ + SEL;
-    double xs = (gy == 0) ? -xc : s.Xk[col - W];
-    double xn = (gy == g.ny - 1) ? -xc : s.Xk[col + W];
-    double xb = zlo ? -xc : s.Xm[col];
-    double xt = zhi ? -xc : s.Xp[col];
-    double r;
+    if (gxr == 0) xw = 0.0;
+    if (gxr == g.nx - 1) xe = 0.0;
+    const double xs = (gy == 0) ? 0.0 : s.Xk[col - W];
+    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
+    const double xb = zlo ? 0.0 : s.Xm[col];
+    const double xt = zhi ? 0.0 : s.Xp[col];
+    double r, S;
     if (SEL == 0) {
-        if (RESID) {
-            double ax = ax_at(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x,
-                              bkh.x, al2.x, a, bh2);
-            rres = rh2.x - ax;
-            r = xc + dv2.x * rres;
-        } else {
-            r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x,
-                          al2.x, dv2.x, rh2.x, a, bh2);
-        }
+        S = sum6(xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x);
+        const double q = rh2.x + bh2 * S;
+        r = dv2.x * q;
+        if (RESID) rres = q - xp2.x / dv2.x;
         nb[0] = bi2.y; nb[1] = bie; nb[2] = bjl.y; nb[3] = bjh.y; nb[4] = bkl.y; nb[5] = bkh.y;
-        nb[6] = al2.y; nb[7] = dv2.y; nb[8] = rh2.y;
+        nb[6] = dv2.y; nb[7] = rh2.y;
     } else {
-        if (RESID) {
-            double ax = ax_at(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y,
-                              al2.y, a, bh2);
-            rres = rh2.y - ax;
-            r = xc + dv2.y * rres;
-        } else {
-            r = gs_update(xc, xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y,
-                          al2.y, dv2.y, rh2.y, a, bh2);
-        }
+        S = sum6(xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y);
+        const double q = rh2.y + bh2 * S;
+        r = dv2.y * q;
+        if (RESID) rres = q - xp2.y / dv2.y;
         nb[0] = bi2.x; nb[1] = bi2.y; nb[2] = bjl.x; nb[3] = bjh.x; nb[4] = bkl.x; nb[5] = bkh.x;
-        nb[6] = al2.x; nb[7] = dv2.x; nb[8] = rh2.x;
+        nb[6] = dv2.x; nb[7] = rh2.x;
     }
-    rold = xc;
+    rold = SEL ? xp2.y : xp2.x;
     xpair = xp2;
     return r;
 }
@@ -242,77 +223,68 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
 // are still old in smem, the red cell below (same column, plane q-1) is this
 // thread's red-old value of the previous plane, the one above is untouched.
 template <int BS>
-__device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int lane, int gx, int gy,
-                                              const Geo& g, bool zlo, bool zhi, double a,
-                                              double bh2, const double* nb, double rold_below,
-                                              double2 xp2) {
-    double xc, xw, xe;
+__device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int gx, int gy,
+                                              const Geo& g, bool zlo, bool zhi, double bh2,
+                                              const double* nb, double rold_below, double2 xp2) {
+    double xw, xe;
     if (BS == 1) {
-        xc = xp2.y; xw = xp2.x; xe = s.Xk[xo_ + 2];
+        xw = xp2.x; xe = s.Xk[xo_ + 2];
     } else {
-        xc = xp2.x; xw = s.Xk[xo_ - 1]; xe = xp2.y;
+        xw = s.Xk[xo_ - 1]; xe = xp2.y;
     }
+    const double xc = BS ? xp2.y : xp2.x;
     const int gxb = gx + BS;
-    if (gxb == 0) xw = -xc;
-    if (gxb == g.nx - 1) xe = -xc;
+    if (gxb == 0) xw = 0.0;
+    if (gxb == g.nx - 1) xe = 0.0;
     const int col = xo_ + BS;
-    double xs = (gy == 0) ? -xc : s.Xk[col - W];
-    double xn = (gy == g.ny - 1) ? -xc : s.Xk[col + W];
-    double xb = zlo ? -xc : rold_below;
-    double xt = zhi ? -xc : s.Xp[col];
-    return nb[8] - ax_at(xc, xw, xe, xs, xn, xb, xt, nb[0], nb[1], nb[2], nb[3], nb[4], nb[5],
-                         nb[6], a, bh2);
+    const double xs = (gy == 0) ? 0.0 : s.Xk[col - W];
+    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
+    const double xb = zlo ? 0.0 : rold_below;
+    const double xt = zhi ? 0.0 : s.Xp[col];
+    const double S = sum6(xw, xe, xs, xn, xb, xt, nb[0], nb[1], nb[2], nb[3], nb[4], nb[5]);
+    return (nb[7] + bh2 * S) - xc / nb[6];
 }
 
 // B for the pair; SEL = position (0: even x, 1: odd x) of the black cell in
 // the pair.  Returns the output pair (red-new, black-new in place).
 template <int SEL>
-__device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int lane, int gx, int gy,
-                                              const Geo& g, int gkm, double a, double bh2,
-                                              const double* rb) {
-    double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
-    double xc, xw, xe;
+__device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx, int gy,
+                                              const Geo& g, int gkm, double bh2, const double* rb) {
+    const double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
+    double xw, xe;
     if (SEL == 0) {
-        xc = q2.x; xw = s.Xm[xo_ - 1]; xe = q2.y;
+        xw = s.Xm[xo_ - 1]; xe = q2.y;
     } else {
-        xc = q2.y; xw = q2.x; xe = s.Xm[xo_ + 2];
+        xw = q2.x; xe = s.Xm[xo_ + 2];
     }
     const int gxb = gx + SEL;
-    if (gxb == 0) xw = -xc;
-    if (gxb == g.nx - 1) xe = -xc;
+    if (gxb == 0) xw = 0.0;
+    if (gxb == g.nx - 1) xe = 0.0;
     const int col = xo_ + SEL;
-    double xs = (gy == 0) ? -xc : s.Xm[col - W];
-    double xn = (gy == g.ny - 1) ? -xc : s.Xm[col + W];
-    double xb = (gkm == 0) ? -xc : s.Xmm[col];
-    double xt = (gkm == g.gnz - 1) ? -xc : s.Xk[col];
-    double bnew = gs_update(xc, xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5],
-                            rb[6], rb[7], rb[8], a, bh2);
+    const double xs = (gy == 0) ? 0.0 : s.Xm[col - W];
+    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
+    const double xb = (gkm == 0) ? 0.0 : s.Xmm[col];
+    const double xt = (gkm == g.gnz - 1) ? 0.0 : s.Xk[col];
+    const double bnew =
+        rb[6] * (rb[7] + bh2 * sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
     return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
 }
 
 // Ring red cell at smem offsets (xo_, co_) (scalar loads; bounds in flags)
-__device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, int flags, double a,
-                                           double bh2, bool zlo, bool zhi) {
-    double xc = s.Xk[xo_];
-    double xw = (flags & 1) ? -xc : s.Xk[xo_ - 1];
-    double xe = (flags & 2) ? -xc : s.Xk[xo_ + 1];
-    double xs = (flags & 4) ? -xc : s.Xk[xo_ - W];
-    double xn = (flags & 8) ? -xc : s.Xk[xo_ + W];
-    double xb = zlo ? -xc : s.Xm[xo_];
-    double xt = zhi ? -xc : s.Xp[xo_];
-    return gs_update(xc, xw, xe, xs, xn, xb, xt, s.C[CA_BI * CARR + co_],
-                     s.C[CA_BI * CARR + co_ + 1], s.C[CA_BJ * CARR + co_],
-                     s.C[CA_BJ * CARR + co_ + W], s.Klo[co_], s.Khi[co_],
-                     s.C[CA_AL * CARR + co_], s.C[CA_DV * CARR + co_], s.C[CA_RH * CARR + co_],
-                     a, bh2);
+__device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, int flags, double bh2,
+                                           bool zlo, bool zhi) {
+    const double xw = (flags & 1) ? 0.0 : s.Xk[xo_ - 1];
+    const double xe = (flags & 2) ? 0.0 : s.Xk[xo_ + 1];
+    const double xs = (flags & 4) ? 0.0 : s.Xk[xo_ - W];
+    const double xn = (flags & 8) ? 0.0 : s.Xk[xo_ + W];
+    const double xb = zlo ? 0.0 : s.Xm[xo_];
+    const double xt = zhi ? 0.0 : s.Xp[xo_];
+    const double S = sum6(xw, xe, xs, xn, xb, xt, s.C[CA_BI * CARR + co_],
+                          s.C[CA_BI * CARR + co_ + 1], s.C[CA_BJ * CARR + co_],
+                          s.C[CA_BJ * CARR + co_ + W], s.Klo[co_], s.Khi[co_]);
+    return s.C[CA_DV * CARR + co_] * (s.C[CA_RH * CARR + co_] + bh2 * S);
 }
 
-// Step t of the software pipeline: R(t+1) and B(t-1) are independent (R(t+1)
-// reads black-OLD cells of planes t..t+2, B(t-1) reads red-NEW cells of
-// planes t-2..t and writes only global memory), so each thread runs both
-// chains together (ILP 2) between two consecutive barriers.  The black cell's
-// coefficients of plane q are taken from the smem slot by R(q) at step q-1
-// and kept in registers until B(q) at step q+1 (stash alternates by step).
 template <bool RESID, bool INTERP>
 __global__ void __launch_bounds__(NT, 1)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
@@ -349,7 +321,6 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             mbar_expect(b, BUNDLE_BYTES);
             tma3(Xs + md(q + 1, NXS) * XSLOT, &mp.x, cx, cyx, q + 1 + SF_GZ, b);
             double* c = Cs + md(q, NCS) * CSLOT;
-            tma3(c + CA_AL * CARR, &mp.al, cx, cyc, q + SF_GZ, b);
             tma3(c + CA_DV * CARR, &mp.dv, cx, cyc, q + SF_GZ, b);
             tma3(c + CA_RH * CARR, &mp.rh, cx, cyc, q + SF_GZ, b);
             tma3(c + CA_BI * CARR, &mp.bi, cx, cyc, q + SF_GZ, b);
@@ -401,9 +372,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             }
         }
         double rold = 0.0;  // RESID: red-old value of the previous plane (this pair)
-        double stA[9], stB[9];
+        double stA[8], stB[8];
 #pragma unroll
-        for (int i = 0; i < 9; i++) stA[i] = stB[i] = 0.0;
+        for (int i = 0; i < 8; i++) stA[i] = stB[i] = 0.0;
 
         // rotating slot indices for step t = z0-2: R(z0-1) / B(z0-3)
         // x slots: x(t-2) .. x(t+2)
@@ -478,7 +449,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             sb.Xk = Xs + ix_0 * XSLOT;                   // x(t)   (top neighbour)
             sb.Xm = Xs + ix_m1 * XSLOT;                  // x(t-1) (the plane)
             sb.Xmm = Xs + ix_m2 * XSLOT;                 // x(t-2) (bottom neighbour)
-            double nb[9];
+            double nb[8];
             double rn = 0.0;
             double2 o = make_double2(0.0, 0.0);
             const bool zlo = gkr == 0, zhi = gkr == g.gnz - 1;
@@ -488,17 +459,17 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             double rres = 0.0, rold_new = 0.0, bres = 0.0;
             double2 xpair = make_double2(0.0, 0.0);
             if (sel == 0) {
-                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb,
+                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
                                                  rres, rold_new, xpair);
-                if (bin) o = black_pair<1>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
+                if (bin) o = black_pair<1>(sb, xoff, gxa, gy, g, gkm, bh2, stash);
                 if (RESID && rin)
-                    bres = black_resid<1>(s, xoff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb, rold, xpair);
+                    bres = black_resid<1>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
             } else {
-                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb,
+                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
                                                  rres, rold_new, xpair);
-                if (bin) o = black_pair<0>(sb, xoff, hl, gxa, gy, g, gkm, a, bh2, stash);
+                if (bin) o = black_pair<0>(sb, xoff, gxa, gy, g, gkm, bh2, stash);
                 if (RESID && rin)
-                    bres = black_resid<0>(s, xoff, hl, gxa, gy, g, zlo, zhi, a, bh2, nb, rold, xpair);
+                    bres = black_resid<0>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
             }
             if (RESID) {
                 if (rin && q >= z0 && q < z1) {   // this item's planes only
@@ -511,7 +482,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const bool ring = rin && (par ? rok[1] : rok[0]);
             const int ro = par ? rxo[1] : rxo[0];
             double rr = 0.0;
-            if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], a, bh2, zlo, zhi);
+            if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], bh2, zlo, zhi);
             if (RESID) __syncthreads();   // black residuals read red-OLD cells of plane q
             double* Xw = Xs + ix_p1 * XSLOT;
             if (rin) Xw[xoff + sel] = rn;
@@ -520,7 +491,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
 #pragma unroll
-            for (int i = 0; i < 9; i++) stash[i] = nb[i];
+            for (int i = 0; i < 8; i++) stash[i] = nb[i];
             fence_proxy_async();
             __syncthreads();
             // refill bundle t+PF+1 (its slots were last read before this barrier)
@@ -635,7 +606,6 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         PV v = sf_view(L, p);
         Maps mp;
         SF_TRY(encode(&mp.x, L, v.f[xin], XH));
-        SF_TRY(encode(&mp.al, L, v.f[SF_ALPHA], CHH));
         SF_TRY(encode(&mp.dv, L, v.f[SF_DINV], CHH));
         SF_TRY(encode(&mp.rh, L, v.f[rhs], CHH));
         SF_TRY(encode(&mp.bi, L, v.f[SF_BETA_I], CHH));
