@@ -33,6 +33,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 GSRB_BYTES_PER_CELL = 64      # PAPER.md:669-672 (x r+w, rhs, alpha, beta x3, lambda)
+GSRB_KERNEL_BYTES_PER_CELL = 56   # lambda-form smoother never reads alpha
 F_OVER_V = 8.0 / 7.0          # F-cycle cost in finest-level V-cycles (sum over levels)
 
 
@@ -276,11 +277,17 @@ def main():
             alg = GSRB_BYTES_PER_CELL * dof_local
             ach = alg / (fine_pair / 1e3) / 1e9
             tr = ncu_traffic().get(f"{nx}x{ny}x{nz // world}")
+            kb = GSRB_KERNEL_BYTES_PER_CELL * dof_local
             roof = {"bound": "hbm", "achieved": ach, "peak": pk, "unit": "GB/s",
                     "frac": ach / pk, "traffic": tr,
-                    "kernel": "gsrb_pair_kernel (colour-fused RB pair, finest level)",
-                    "algorithmic_bytes_per_launch": alg, "launch_ms": fine_pair,
-                    "peak_source": pk_src,
+                    "kernel": "gsrb_pair_tma_kernel (colour-fused RB pair, finest level)",
+                    "algorithmic_bytes_per_launch": alg,
+                    "algorithmic_basis": "64 B/cell per RB pair (PAPER.md:669-672, SURVEY 8d)",
+                    "kernel_compulsory_bytes_per_launch": kb,
+                    "frac_of_kernel_compulsory": kb / (fine_pair / 1e3) / 1e9 / pk,
+                    "note": "lambda-form update reads 56 of the paper's 64 B/cell (alpha enters "
+                            "only through lambda = 1/diag(A)); traffic = ncu DRAM bytes per launch",
+                    "launch_ms": fine_pair, "peak_source": pk_src,
                     "share_of_step": side.get("fine_pair_share")}
         line = {
             "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
@@ -419,7 +426,10 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
         fig7["vc_gsrb_pair"] = {"ms": ms, "gstencil_s": cells / (ms / 1e3) / 1e9, "alg_gbs": gbs,
                                 "frac_of_peak": gbs / pk, "bytes_per_cell": 64}
         out["fig7_256"] = fig7
-        out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms, "gstencil_s": 2 * cells / 2 / (ms / 1e3) / 1e9,
+        out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms,
+                          "frac_of_kernel_compulsory": GSRB_KERNEL_BYTES_PER_CELL * cells / (ms / 1e3)
+                          / 1e9 / pk,
+                          "gstencil_s": 2 * cells / 2 / (ms / 1e3) / 1e9,
                           "point_updates_per_s": cells / (ms / 1e3),
                           "alg_gbs": gbs, "frac_of_peak": gbs / pk,
                           "colour_sweeps_ms_per_rb_pair": msc,
