@@ -288,13 +288,28 @@ static sf_status body_of(sf_mg* m, int kind) {
     }
 }
 
+// Capture cycle piece `kind` into a graph.  Any failure during capture (e.g. a
+// collective that refuses capture) leaves graphs off for this hierarchy and
+// restores every level's field mapping, so the caller falls back to eager
+// enqueueing; only errors of the eager path are reported.
 static sf_status capture(sf_mg* m, int kind) {
     sf_level* L = m->lv[0];
+    std::vector<std::vector<SfPart>> saved;
+    for (sf_level* lv : m->lv) saved.push_back(lv->parts);
     long long before, after;
     sf_launch_count(&before, 0);
-    if (cudaStreamBeginCapture(L->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+    auto give_up = [&]() {
         cudaGetLastError();
+        for (size_t i = 0; i < m->lv.size(); i++) m->lv[i]->parts = saved[i];
         m->graph_failed = true;
+        for (auto& g : m->gexec)
+            if (g) {
+                cudaGraphExecDestroy(g);
+                g = nullptr;
+            }
+    };
+    if (cudaStreamBeginCapture(L->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        give_up();
         return SF_OK;
     }
     sf_status s = body_of(m, kind);
@@ -302,21 +317,16 @@ static sf_status capture(sf_mg* m, int kind) {
     cudaError_t e = cudaStreamEndCapture(L->stream, &g);
     sf_launch_count(&after, 0);
     sf_count_launch(-(after - before));  // captured, not launched
-    if (s != SF_OK) {
+    if (s != SF_OK || e != cudaSuccess || !g) {
         if (g) cudaGraphDestroy(g);
-        return s;
-    }
-    if (e != cudaSuccess || !g) {
-        cudaGetLastError();
-        m->graph_failed = true;
+        give_up();
         return SF_OK;
     }
     e = cudaGraphInstantiate(&m->gexec[kind], g, 0);
     cudaGraphDestroy(g);
     if (e != cudaSuccess) {
-        cudaGetLastError();
         m->gexec[kind] = nullptr;
-        m->graph_failed = true;
+        give_up();
         return SF_OK;
     }
     m->gnodes[kind] = after - before;
@@ -331,7 +341,7 @@ static sf_status run(sf_mg* m, int kind) {
             // capture both halves back to back: together they hold an even
             // number of U/TMP swaps, so the host mapping is restored
             SF_TRY(capture(m, G_FIRST));
-            SF_TRY(capture(m, G_REST));
+            if (!m->graph_failed) SF_TRY(capture(m, G_REST));
         } else {
             SF_TRY(capture(m, kind));
         }
