@@ -340,8 +340,12 @@ static sf_status run(sf_mg* m, int kind) {
         if (kind == G_FIRST || kind == G_REST) {
             // capture both halves back to back: together they hold an even
             // number of U/TMP swaps, so the host mapping is restored
+            std::vector<std::vector<SfPart>> saved;
+            for (sf_level* lv : m->lv) saved.push_back(lv->parts);
             SF_TRY(capture(m, G_FIRST));
             if (!m->graph_failed) SF_TRY(capture(m, G_REST));
+            if (m->graph_failed)
+                for (size_t i = 0; i < m->lv.size(); i++) m->lv[i]->parts = saved[i];
         } else {
             SF_TRY(capture(m, kind));
         }
