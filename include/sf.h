@@ -82,7 +82,8 @@ enum sf_interp_kind { SF_INTERP_P0 = 0 /* piecewise constant */,
 enum sf_norm_kind { SF_NORM_MAX = 0, SF_NORM_L2 = 1 };
 enum sf_smoother_kind { SF_SMOOTH_AUTO = 0,     /* fused when the shape allows */
                         SF_SMOOTH_COLOUR = 1,   /* one kernel per colour sweep  */
-                        SF_SMOOTH_FUSED = 2 };  /* colour-fused RB pair         */
+                        SF_SMOOTH_FUSED = 2,    /* colour-fused RB pair         */
+                        SF_SMOOTH_CHEBY = 3 };  /* NEXT-3 Chebyshev (mg option) */
 
 typedef struct sf_comm sf_comm;
 typedef struct sf_level sf_level;
@@ -98,6 +99,7 @@ typedef struct {
     int use_graph;          /* capture V-cycles as CUDA graphs (1) */
     int smoother;           /* enum sf_smoother_kind */
     double rtol;            /* ||f-Au||inf/||f||inf target (1e-10, reading R-9) */
+    int cheby_degree;       /* SF_SMOOTH_CHEBY: steps per pair count (2: pre=post=2 -> 4 steps) */
 } sf_mg_opts;
 
 /* Default options (pre=post=2, P0/PL, agglomerate below 16 planes, 50 cycles,
@@ -187,6 +189,19 @@ sf_status sf_interpolate(sf_level* fine, int f_field, double prescale,
  * Both need an even gnx (SF_ERR_SHAPE otherwise). */
 sf_status sf_apply_laplacian(sf_level* level, int out, int x);
 sf_status sf_jacobi(sf_level* level, int out, int x, int f, double omega);
+/* NEXT-3, the Chebyshev smoother the paper names as an in-place technique
+ * (formula = reading R-16, Saad Alg. 12.1 with the Jacobi
+ * preconditioner D = diag(A)):
+ * sf_smooth_chebyshev: `degree` steps damping the eigenvalues of D^-1 A in
+ *   [lo, hi] (0 < lo < hi), in place on x; uses TMP and R as scratch (x, rhs
+ *   must be other fields).  Field ids of TMP/R may be permuted afterwards.
+ * sf_lambda_max: power iteration estimate of lambda_max(D^-1 A): `iters` (>= 2)
+ *   steps v <- D^-1 A v / ||.||_2 from the current v, or from the start vector
+ *   v = 1 + ((7i + 13j + 29k) mod 17)/17 if start != 0; uses R; syncs. */
+sf_status sf_smooth_chebyshev(sf_level* level, int x, int rhs, double a, double b, int degree,
+                              double lo, double hi);
+sf_status sf_lambda_max(sf_level* level, int v, double a, double b, int iters, int start,
+                        double* out);
 /* A10: norm of the interior over all parts/ranks; syncs. */
 sf_status sf_norm(sf_level* level, int field, int kind, double* out);
 sf_status sf_sync(sf_level* level);

@@ -339,10 +339,19 @@ done:
 /* h_c = 2h (reading R-7); bottom at min dim 2 (reading R-8).                */
 /* ------------------------------------------------------------------------ */
 #define OR_MAXL 24
+void or_chebyshev(const or_grid* g, double a, double b, const double* alpha, const double* bi,
+                  const double* bj, const double* bk, const double* dinv, double* x,
+                  const double* f, int degree, double lo, double hi, double* xprev,
+                  double* xnext);
+double or_lambda_max(const or_grid* g, double a, double b, const double* alpha, const double* bi,
+                     const double* bj, const double* bk, const double* dinv, double* v,
+                     double* w, int iters);
 typedef struct {
     int nl;
     double a, b;
     int pre, post;
+    int cheby_steps;                  /* NEXT-3: Chebyshev steps per "pair" (0 = GSRB) */
+    double lmax[OR_MAXL];
     or_grid g[OR_MAXL];
     double *alpha[OR_MAXL], *bi[OR_MAXL], *bj[OR_MAXL], *bk[OR_MAXL], *dinv[OR_MAXL];
     double *e[OR_MAXL], *r[OR_MAXL], *res[OR_MAXL];
@@ -402,17 +411,54 @@ void or_mg_level_dims(const or_mg* m, int l, int* d) {
 
 #define LV(m, l) &(m)->g[l], (m)->a, (m)->b, (m)->alpha[l], (m)->bi[l], (m)->bj[l], (m)->bk[l]
 
+/* smoother of V(l): GSRB pairs or, after or_mg_set_chebyshev,
+ * Chebyshev with 'pairs * cheby_steps' steps on [hi/8, hi], hi = 1.05 lambda_max
+ * (reading R-16) */
+static void mg_smooth(or_mg* m, int l, int pairs) {
+    if (!m->cheby_steps) {
+        or_smooth(LV(m, l), m->dinv[l], m->e[l], m->r[l], pairs);
+        return;
+    }
+    if (pairs == 0) return;
+    size_t sz = or_size(m->g[l].nx, m->g[l].ny, m->g[l].nz) * sizeof(double);
+    double* w1 = malloc(sz);
+    double* w2 = malloc(sz);
+    double hi = 1.05 * m->lmax[l], lo = hi / 8.0;
+    or_chebyshev(LV(m, l), m->dinv[l], m->e[l], m->r[l], pairs * m->cheby_steps, lo, hi, w1, w2);
+    free(w1);
+    free(w2);
+}
+
+/* NEXT-3: switch the hierarchy to Chebyshev smoothing; lambda_max(D^-1 A) per
+ * level by 30 power-iteration steps from v = 1 + ((7i + 13j + 29k) mod 17)/17 */
+void or_mg_set_chebyshev(or_mg* m, int steps_per_pair) {
+    m->cheby_steps = steps_per_pair;
+    for (int l = 0; l + 1 < m->nl; l++) {
+        or_grid* g = &m->g[l];
+        size_t sz = or_size(g->nx, g->ny, g->nz);
+        double* v = calloc(sz, sizeof(double));
+        double* w = calloc(sz, sizeof(double));
+        for (int k = 0; k < g->nz; k++)
+            for (int j = 0; j < g->ny; j++)
+                for (int i = 0; i < g->nx; i++)
+                    v[OIDX(g, i, j, k)] = 1.0 + (double)((7L * i + 13L * j + 29L * k) % 17) / 17.0;
+        m->lmax[l] = or_lambda_max(LV(m, l), m->dinv[l], v, w, 30);
+        free(v);
+        free(w);
+    }
+}
+
 /* V(l) on (e[l], r[l]); see SURVEY/DESIGN A9 */
 static int vcycle(or_mg* m, int l) {
     if (l == m->nl - 1) return or_bottom_solve(LV(m, l), m->e[l], m->r[l]);
-    or_smooth(LV(m, l), m->dinv[l], m->e[l], m->r[l], m->pre);
+    mg_smooth(m, l, m->pre);
     or_residual(LV(m, l), m->e[l], m->r[l], m->res[l]);
     or_restrict_cell(&m->g[l + 1], m->r[l + 1], &m->g[l], m->res[l]);
     memset(m->e[l + 1], 0,
            or_size(m->g[l + 1].nx, m->g[l + 1].ny, m->g[l + 1].nz) * sizeof(double));
     int rc = vcycle(m, l + 1);
     or_interp_p0(&m->g[l], m->e[l], 1.0, &m->g[l + 1], m->e[l + 1]);
-    or_smooth(LV(m, l), m->dinv[l], m->e[l], m->r[l], m->post);
+    mg_smooth(m, l, m->post);
     return rc;
 }
 
@@ -565,4 +611,76 @@ void or_jacobi_cc(const or_grid* g, double omega, double* x, const double* f, do
                 size_t c = OIDX(g, i, j, k);
                 out[c] = x[c] + omega * (f[c] - lap_at(g, x, i, j, k)) / d;
             }
+}
+
+/* ------------------------------------------------------------------------ */
+/* NEXT-3: Chebyshev polynomial smoother (PAPER.md:306-308 names "Chebyshev  */
+/* smoothing" as an in-place technique; the paper gives no formula -- reading */
+/* R-16).  Chebyshev acceleration of the Jacobi-preconditioned iteration     */
+/* (Saad, Iterative Methods, Alg. 12.1) for eigenvalues of D^-1 A in         */
+/* [lo, hi]: theta = (hi+lo)/2, delta = (hi-lo)/2, sigma = theta/delta,      */
+/*   x1 = x0 + (1/theta) D^-1 (f - A x0),                                    */
+/*   x_{k+1} = x_k + rho_k rho_{k-1} (x_k - x_{k-1})                         */
+/*                 + (2 rho_k / delta) D^-1 (f - A x_k),                    */
+/*   rho_0 = 1/sigma, rho_k = 1/(2 sigma - rho_{k-1}).                       */
+/* x is overwritten with x_degree; work holds two scratch arrays.            */
+/* ------------------------------------------------------------------------ */
+void or_chebyshev(const or_grid* g, double a, double b, const double* alpha, const double* bi,
+                  const double* bj, const double* bk, const double* dinv, double* x,
+                  const double* f, int degree, double lo, double hi, double* xprev,
+                  double* xnext) {
+    size_t sz = or_size(g->nx, g->ny, g->nz);
+    double theta = 0.5 * (hi + lo), delta = 0.5 * (hi - lo), sigma = theta / delta;
+    double rho_prev = 1.0 / sigma, rho = rho_prev;
+    memcpy(xprev, x, sz * sizeof(double));
+    for (int it = 0; it < degree; it++) {
+        double c1, c2;
+        if (it == 0) {
+            c1 = 0.0;
+            c2 = 1.0 / theta;
+        } else {
+            rho = 1.0 / (2.0 * sigma - rho_prev);
+            c1 = rho * rho_prev;
+            c2 = 2.0 * rho / delta;
+        }
+        or_apply_bc(g, x);
+        for (int k = 0; k < g->nz; k++)
+            for (int j = 0; j < g->ny; j++)
+                for (int i = 0; i < g->nx; i++) {
+                    size_t c = OIDX(g, i, j, k);
+                    double r = f[c] - op_at(g, a, b, alpha, bi, bj, bk, x, i, j, k);
+                    xnext[c] = x[c] + c1 * (x[c] - xprev[c]) + c2 * dinv[c] * r;
+                }
+        memcpy(xprev, x, sz * sizeof(double));
+        memcpy(x, xnext, sz * sizeof(double));
+        if (it > 0) rho_prev = rho;
+    }
+}
+
+/* Largest eigenvalue of D^-1 A by power iteration (setup of the Chebyshev   */
+/* interval, reading R-16): v <- D^-1 A v / ||D^-1 A v||_2, iters times from */
+/* the given start; returns the last ||D^-1 A v||_2 / ||v||_2.              */
+double or_lambda_max(const or_grid* g, double a, double b, const double* alpha, const double* bi,
+                     const double* bj, const double* bk, const double* dinv, double* v,
+                     double* w, int iters) {
+    double lam = 0.0;
+    for (int it = 0; it < iters; it++) {
+        double nv = or_norm_l2(g, v);
+        or_apply_op(g, a, b, alpha, bi, bj, bk, v, w);
+        for (int k = 0; k < g->nz; k++)
+            for (int j = 0; j < g->ny; j++)
+                for (int i = 0; i < g->nx; i++) {
+                    size_t c = OIDX(g, i, j, k);
+                    w[c] = dinv[c] * w[c];
+                }
+        double nw = or_norm_l2(g, w);
+        lam = nw / nv;
+        for (int k = 0; k < g->nz; k++)
+            for (int j = 0; j < g->ny; j++)
+                for (int i = 0; i < g->nx; i++) {
+                    size_t c = OIDX(g, i, j, k);
+                    v[c] = w[c] / nw;
+                }
+    }
+    return lam;
 }

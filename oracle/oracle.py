@@ -69,11 +69,14 @@ def lib():
             "or_mg_levels": (C.c_int, [C.c_void_p]),
             "or_mg_level_dims": (None, [C.c_void_p, C.c_int, C.POINTER(C.c_int)]),
             "or_mg_vcycle": (C.c_int, [C.c_void_p, _P, _P]),
+            "or_mg_set_chebyshev": (None, [C.c_void_p, C.c_int]),
             "or_mg_fcycle": (C.c_int, [C.c_void_p, _P, _P]),
             "or_mg_relres": (d, [C.c_void_p, _P, _P]),
             "or_mg_solve": (C.c_int, [C.c_void_p, _P, _P, C.c_int, d, C.c_int, _P]),
             "or_laplacian_cc": (None, [G, _P, _P]),
             "or_jacobi_cc": (None, [G, d, _P, _P, _P]),
+            "or_chebyshev": (None, [G, d, d, _P, _P, _P, _P, _P, _P, _P, C.c_int, d, d, _P, _P]),
+            "or_lambda_max": (d, [G, d, d, _P, _P, _P, _P, _P, _P, _P, C.c_int]),
             "or_residual_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP, _IP,
                                           _P]),
             "or_gsrb_pair_points": (None, [G, d, d, _P, _P, _P, _P, _P, _P, _P, C.c_int, _IP, _IP,
@@ -189,6 +192,20 @@ class Problem:
                                   _iptr(jj), _iptr(kk), _ptr(out))
         return out
 
+    def chebyshev(self, x, rhs, degree, lo, hi, dinv=None):
+        """NEXT-3: degree Chebyshev steps for D^-1 A eigenvalues in [lo, hi]."""
+        dinv = self.dinv() if dinv is None else dinv
+        xp, rp, dp = pad(x), pad(rhs), pad(dinv)
+        w1, w2 = np.zeros_like(xp), np.zeros_like(xp)
+        lib().or_chebyshev(*self._c(), _ptr(dp), _ptr(xp), _ptr(rp), int(degree), float(lo),
+                           float(hi), _ptr(w1), _ptr(w2))
+        return interior(xp)
+
+    def lambda_max(self, v0, iters, dinv=None):
+        dinv = self.dinv() if dinv is None else dinv
+        vp, dp, w = pad(v0), pad(dinv), np.zeros_like(self.alpha)
+        return lib().or_lambda_max(*self._c(), _ptr(dp), _ptr(vp), _ptr(w), int(iters))
+
     def bottom_solve(self, rhs):
         xp, rp = np.zeros_like(self.alpha), pad(rhs)
         rc = lib().or_bottom_solve(*self._c(), _ptr(xp), _ptr(rp))
@@ -272,6 +289,10 @@ class MG:
         if getattr(self, "h", None):
             lib().or_mg_free(self.h)
             self.h = None
+
+    def set_chebyshev(self, steps_per_pair=2):
+        """NEXT-3: Chebyshev smoothing in every V-cycle (reading R-16)."""
+        lib().or_mg_set_chebyshev(self.h, int(steps_per_pair))
 
     @property
     def levels(self):

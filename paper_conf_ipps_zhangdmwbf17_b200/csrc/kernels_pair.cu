@@ -230,6 +230,92 @@ __global__ void __launch_bounds__(PX* PY) cc_pair_kernel(PV v, double* __restric
     }
 }
 
+// NEXT-3 Chebyshev step (reading R-16): out = x + c1 (x - xp) + c2 Dinv (rhs - A x),
+// A in op_at's term order.  72 B/cell (x, xp, rhs, alpha, beta x3, Dinv, out).
+__global__ void __launch_bounds__(PX* PY) cheby_pair_kernel(PV v, double* __restrict__ out,
+                                                             const double* __restrict__ x,
+                                                             const double* __restrict__ xp,
+                                                             const double* __restrict__ rhs,
+                                                             double c1, double c2, double a,
+                                                             double bh2, int depth) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    if (i >= v.nx || j >= v.ny) return;
+    for (int k = k0; k < k1; k++) {
+        const long c = sf_ix(v, i, j, k);
+        double axa, axb;
+        op_pair(v, x, i, j, v.z0 + k, c, a, bh2, axa, axb);
+        const double2 f = ld2(rhs + c), xc = ld2(x + c), xq = ld2(xp + c),
+                      dv = ld2(v.f[SF_DINV] + c);
+        double2 o;
+        o.x = xc.x + c1 * (xc.x - xq.x) + c2 * dv.x * (f.x - axa);
+        o.y = xc.y + c1 * (xc.y - xq.y) + c2 * dv.y * (f.y - axb);
+        *(double2*)(out + c) = o;
+    }
+}
+
+// power-iteration helpers for lambda_max(D^-1 A): w *= Dinv with sum w^2 (atomic),
+// and v = w * scale[0]
+__global__ void __launch_bounds__(PX* PY) dinv_scale_pair_kernel(PV v, double* __restrict__ w,
+                                                                  int depth, double* sumsq) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    double acc = 0.0;
+    if (i < v.nx && j < v.ny)
+        for (int k = k0; k < k1; k++) {
+            const long c = sf_ix(v, i, j, k);
+            double2 u = ld2(w + c);
+            const double2 dv = ld2(v.f[SF_DINV] + c);
+            u.x = dv.x * u.x;
+            u.y = dv.y * u.y;
+            *(double2*)(w + c) = u;
+            acc += u.x * u.x;
+            acc += u.y * u.y;
+        }
+    __shared__ double rs[PX * PY / 32];
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    const int t = threadIdx.y * PX + threadIdx.x;
+    if ((t & 31) == 0) rs[t >> 5] = acc;
+    __syncthreads();
+    if (t == 0) {
+        for (int wq = 1; wq < PX * PY / 32; wq++) acc += rs[wq];
+        atomicAdd(sumsq, acc);
+    }
+}
+
+// deterministic positive start vector for the power iteration (the oracle
+// test builds the same formula independently):
+// v(i,j,k) = 1 + ((7 gi + 13 gj + 29 gk) mod 17) / 17
+__global__ void __launch_bounds__(PX* PY) start_vector_kernel(PV v, double* __restrict__ y,
+                                                               int depth) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    if (i >= v.nx || j >= v.ny) return;
+    for (int k = k0; k < k1; k++) {
+        const long gk = v.z0 + k;
+        double2 o;
+        o.x = 1.0 + (double)((7L * i + 13L * j + 29L * gk) % 17) / 17.0;
+        o.y = 1.0 + (double)((7L * (i + 1) + 13L * j + 29L * gk) % 17) / 17.0;
+        *(double2*)(y + sf_ix(v, i, j, k)) = o;
+    }
+}
+
+__global__ void __launch_bounds__(PX* PY) scale_pair_kernel(PV v, double* __restrict__ y,
+                                                             const double* __restrict__ src,
+                                                             const double* sumsq, int depth) {
+    const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
+    const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
+    if (i >= v.nx || j >= v.ny) return;
+    const double sc = 1.0 / sqrt(*sumsq);
+    for (int k = k0; k < k1; k++) {
+        const long c = sf_ix(v, i, j, k);
+        double2 u = ld2(src + c);
+        u.x = u.x * sc;
+        u.y = u.y * sc;
+        *(double2*)(y + c) = u;
+    }
+}
+
 __global__ void zero_scalar(double* p) { *p = 0.0; }
 
 // grid over pairs: (ceil(nx/64), ceil(ny/4), z-chunks) with ~16 blocks per SM
@@ -319,6 +405,58 @@ sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi) {
         SF_LAUNCHED();
     }
     return sf_check_launch("cc_pair");
+}
+
+sf_status k_cheby_step(sf_level* L, int out, int x, int xp, int rhs, double c1, double c2, double a,
+                       double b) {
+    if (!pair_ok(L)) return sf_fail(SF_ERR_SHAPE, "Chebyshev smoother needs an even nx");
+    SF_TRY(sf_halo(L, x, 1));
+    const double bh2 = b / (L->h * L->h);
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        cheby_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], v.f[xp], v.f[rhs],
+                                                             c1, c2, a, bh2, depth);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("cheby_pair");
+}
+
+sf_status k_start_vector(sf_level* L, int field) {
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        start_vector_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[field], depth);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("start_vector");
+}
+
+// one power-iteration step: w = Dinv (A v) (into `w`), ||w||^2 -> *sumsq, v = w / ||w||
+sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, double* sumsq) {
+    if (!pair_ok(L)) return sf_fail(SF_ERR_SHAPE, "power iteration needs an even nx");
+    SF_TRY(k_apply_op(L, w_id, v_id, a, b));
+    zero_scalar<<<1, 1, 0, L->stream>>>(sumsq);
+    SF_LAUNCHED();
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        dinv_scale_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[w_id], depth, sumsq);
+        SF_LAUNCHED();
+    }
+    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+        SF_TRY(sf_allreduce_scalar(L->comm, sumsq, 1, L->stream));
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        int depth;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        scale_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[v_id], v.f[w_id], sumsq, depth);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("power_step");
 }
 
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst) {

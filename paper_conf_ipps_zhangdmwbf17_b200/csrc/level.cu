@@ -277,6 +277,67 @@ extern "C" sf_status sf_jacobi(sf_level* L, int out, int x, int f, double omega)
     return k_cc(L, out, x, f, omega, true);
 }
 
+// NEXT-3: Chebyshev smoother (reading R-16; Saad Alg. 12.1, Jacobi-preconditioned).
+// Ids rotate over {x, TMP, R}; the final iterate ends under the id x.
+sf_status sf_chebyshev_impl(sf_level* L, int x, int rhs, double a, double b, int degree, double lo,
+                            double hi) {
+    const double theta = 0.5 * (hi + lo), delta = 0.5 * (hi - lo), sigma = theta / delta;
+    double rho_prev = 1.0 / sigma, rho = rho_prev;
+    int cur = x, prv = SF_TMP, nxt = SF_R;
+    for (int it = 0; it < degree; it++) {
+        double c1, c2;
+        if (it == 0) {
+            c1 = 0.0;
+            c2 = 1.0 / theta;
+        } else {
+            rho = 1.0 / (2.0 * sigma - rho_prev);
+            c1 = rho * rho_prev;
+            c2 = 2.0 * rho / delta;
+        }
+        SF_TRY(k_cheby_step(L, nxt, cur, it == 0 ? cur : prv, rhs, c1, c2, a, b));
+        const int t = prv;
+        prv = cur;
+        cur = nxt;
+        nxt = t;
+        if (it > 0) rho_prev = rho;
+    }
+    // the result lives in the buffer named `cur`: make `x` name it
+    if (cur != x) sf_swap_fields(L, x, cur);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_smooth_chebyshev(sf_level* L, int x, int rhs, double a, double b,
+                                         int degree, double lo, double hi) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(rhs));
+    if (x == SF_TMP || x == SF_R || rhs == SF_TMP || rhs == SF_R || x == rhs)
+        return sf_fail(SF_ERR_INVALID, "x and rhs must be distinct and not TMP/R (scratch)");
+    if (degree < 0 || !(hi > lo) || !(lo > 0)) return sf_fail(SF_ERR_INVALID, "bad degree/interval");
+    return sf_chebyshev_impl(L, x, rhs, a, b, degree, lo, hi);
+}
+
+sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, bool start,
+                             double* out) {
+    if (start) SF_TRY(k_start_vector(L, v));
+    double* sumsq = L->dscratch + 1;
+    for (int it = 0; it < iters; it++) SF_TRY(k_power_step(L, v, SF_R, a, b, sumsq));
+    // last ratio ||D^-1 A v|| / ||v|| with ||v|| = 1 after normalisation
+    SF_CUDA(cudaMemcpyAsync(L->hscratch + 1, sumsq, sizeof(double), cudaMemcpyDeviceToHost,
+                            L->stream));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    *out = sqrt(L->hscratch[1]);
+    return SF_OK;
+}
+
+extern "C" sf_status sf_lambda_max(sf_level* L, int v, double a, double b, int iters, int start,
+                                   double* out) {
+    if (!L || !out) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    SF_TRY(check_field(v));
+    if (v == SF_R || iters < 1) return sf_fail(SF_ERR_INVALID, "v must not be R; iters >= 1");
+    return sf_lambda_max_impl(L, v, a, b, iters, start != 0, out);
+}
+
 extern "C" sf_status sf_residual(sf_level* L, int res, int x, int rhs, double a, double b) {
     if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
     SF_TRY(check_field(res));

@@ -22,7 +22,16 @@ struct sf_mg {
     cudaGraphExec_t gexec[5] = {};  // V+check, F+check, F, first pair+check, rest of V
     long long gnodes[5] = {};
     bool graph_failed = false;
+    std::vector<double> lmax;   // SF_SMOOTH_CHEBY: lambda_max(D^-1 A) per level
 };
+
+// NEXT-3 reading R-16: Chebyshev interval [hi/8, hi], hi = 1.05 lambda_max(D^-1 A)
+// (power iteration, 30 steps from the fixed start vector, at setup)
+static const int CHEBY_POWER_ITERS = 30;
+static void cheby_interval(double lmax, double* lo, double* hi) {
+    *hi = 1.05 * lmax;
+    *lo = *hi / 8.0;
+}
 
 extern "C" void sf_mg_opts_default(sf_mg_opts* o) {
     if (!o) return;
@@ -35,6 +44,7 @@ extern "C" void sf_mg_opts_default(sf_mg_opts* o) {
     o->use_graph = 1;
     o->smoother = SF_SMOOTH_AUTO;
     o->rtol = 1e-10;
+    o->cheby_degree = 2;
 }
 
 static sf_status destroy_levels(sf_mg* m) {
@@ -108,7 +118,8 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
     m->a = a; m->b = b;
     if (opts) m->o = *opts; else sf_mg_opts_default(&m->o);
     if (m->o.pre_pairs < 0 || m->o.post_pairs < 0 || m->o.max_cycles < 1 ||
-        m->o.agglom_min_planes < 2) {
+        m->o.agglom_min_planes < 2 ||
+        (m->o.smoother == SF_SMOOTH_CHEBY && (m->o.cheby_degree < 1 || (fine->gnx & 1)))) {
         delete m;
         return sf_fail(SF_ERR_INVALID, "bad mg options");
     }
@@ -155,6 +166,14 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
         if (e != cudaSuccess) s = sf_fail(SF_ERR_OOM, "bottom inverse: %s", cudaGetErrorString(e));
     }
     if (s == SF_OK) s = k_bottom_setup(B, a, b, m->ainv);
+    if (s == SF_OK && m->o.smoother == SF_SMOOTH_CHEBY) {
+        for (size_t l = 0; l + 1 < m->lv.size() && s == SF_OK; l++) {
+            double lm = 0.0;
+            s = sf_lambda_max_impl(m->lv[l], SF_TMP, a, b, CHEBY_POWER_ITERS, true, &lm);
+            m->lmax.push_back(lm);
+        }
+        if (s == SF_OK) s = k_zero(fine, SF_TMP);
+    }
     if (s == SF_OK) {
         cudaError_t e = cudaStreamSynchronize(fine->stream);
         if (e != cudaSuccess) s = sf_fail(SF_ERR_CUDA, "mg setup: %s", cudaGetErrorString(e));
@@ -181,6 +200,14 @@ extern "C" sf_status sf_mg_level(sf_mg* m, int l, sf_level** out) {
 }
 
 static sf_status smooth(sf_mg* m, sf_level* L, int pairs) {
+    if (m->o.smoother == SF_SMOOTH_CHEBY) {
+        if (pairs == 0) return SF_OK;
+        size_t l = 0;
+        while (m->lv[l] != L) l++;
+        double lo, hi;
+        cheby_interval(m->lmax[l], &lo, &hi);
+        return sf_chebyshev_impl(L, SF_U, SF_F, m->a, m->b, pairs * m->o.cheby_degree, lo, hi);
+    }
     return sf_smooth_gsrb(L, SF_U, SF_F, m->a, m->b, pairs, m->o.smoother);
 }
 
@@ -200,7 +227,8 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     SF_TRY(k_zero(C, SF_U));
     SF_TRY(vcyc(m, l + 1));
     if (m->o.vcycle_interp == SF_INTERP_P0 && m->o.post_pairs >= 1 &&
-        m->o.smoother != SF_SMOOTH_COLOUR && gsrb_fused_supported(L)) {
+        (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
+        gsrb_fused_supported(L)) {
         // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
         SF_TRY(sf_halo(C, SF_U, 1));
         SF_TRY(sf_halo(L, SF_F, 1));
@@ -252,7 +280,8 @@ static sf_status check(sf_mg* m) {
 // max|F - A U_in| of its INPUT while it writes the smoothed iterate to TMP.
 // If that says "converged", U (the previous cycle's result) is untouched.
 static bool fused_check_ok(const sf_mg* m) {
-    return m->lv.size() > 1 && m->o.pre_pairs >= 1 && m->o.smoother != SF_SMOOTH_COLOUR &&
+    return m->lv.size() > 1 && m->o.pre_pairs >= 1 &&
+           (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
            gsrb_fused_supported(m->lv[0]) && (m->o.pre_pairs + m->o.post_pairs) % 2 == 0;
 }
 
@@ -272,6 +301,9 @@ static bool graphs_allowed(const sf_mg* m) {
     if (m->lv[0]->stream == nullptr) return false;  // legacy stream cannot be captured
     // the fused smoother swaps U/TMP per pair; only an even count per captured
     // sequence leaves the host-side mapping unchanged for replays
+    if (m->o.smoother == SF_SMOOTH_CHEBY)   // an n-step application ends with swap(U, [U,R,TMP][n%3]):
+        return (m->o.pre_pairs * m->o.cheby_degree) % 3 ==   // equal pre/post transpositions cancel
+               (m->o.post_pairs * m->o.cheby_degree) % 3;
     return (m->o.pre_pairs % 2 == 0 && m->o.post_pairs % 2 == 0) ||
            m->o.smoother == SF_SMOOTH_COLOUR;
 }

@@ -111,6 +111,15 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
 sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf);
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
 sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi);  // NEXT-2
+// NEXT-3 Chebyshev smoother pieces
+sf_status k_cheby_step(sf_level* L, int out, int x, int xp, int rhs, double c1, double c2, double a,
+                       double b);
+sf_status k_start_vector(sf_level* L, int field);
+sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, double* sumsq);
+sf_status sf_chebyshev_impl(sf_level* L, int x, int rhs, double a, double b, int degree, double lo,
+                            double hi);
+sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, bool start,
+                             double* out);
 
 // fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
 bool gsrb_fused_supported_t32(const sf_level* L);

@@ -28,7 +28,7 @@ SF_NFIELDS = 9
 SF_RESTRICT_CELL, SF_RESTRICT_FACE_I, SF_RESTRICT_FACE_J, SF_RESTRICT_FACE_K = range(4)
 SF_INTERP_P0, SF_INTERP_PL = 0, 1
 SF_NORM_MAX, SF_NORM_L2 = 0, 1
-SF_SMOOTH_AUTO, SF_SMOOTH_COLOUR, SF_SMOOTH_FUSED = 0, 1, 2
+SF_SMOOTH_AUTO, SF_SMOOTH_COLOUR, SF_SMOOTH_FUSED, SF_SMOOTH_CHEBY = 0, 1, 2, 3
 
 FIELD_IDS = {"u": SF_U, "f": SF_F, "r": SF_R, "tmp": SF_TMP, "alpha": SF_ALPHA,
              "beta_i": SF_BETA_I, "beta_j": SF_BETA_J, "beta_k": SF_BETA_K, "dinv": SF_DINV}
@@ -41,7 +41,7 @@ EXPORTS = [
     "sf_apply_bc", "sf_apply_op", "sf_smooth_gsrb", "sf_residual", "sf_restrict",
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
-    "sf_apply_laplacian", "sf_jacobi",
+    "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
 ]
 
 
@@ -55,7 +55,7 @@ class MgOpts(C.Structure):
     _fields_ = [("pre_pairs", C.c_int), ("post_pairs", C.c_int), ("vcycle_interp", C.c_int),
                 ("fcycle_interp", C.c_int), ("agglom_min_planes", C.c_int),
                 ("max_cycles", C.c_int), ("use_graph", C.c_int), ("smoother", C.c_int),
-                ("rtol", C.c_double)]
+                ("rtol", C.c_double), ("cheby_degree", C.c_int)]
 
 
 _lib = None
@@ -95,6 +95,8 @@ def lib():
         "sf_residual": (_i, [_vp, _i, _i, _i, _d, _d]),
         "sf_apply_laplacian": (_i, [_vp, _i, _i]),
         "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
+        "sf_smooth_chebyshev": (_i, [_vp, _i, _i, _d, _d, _i, _d, _d]),
+        "sf_lambda_max": (_i, [_vp, _i, _d, _d, _i, _i, _P]),
         "sf_restrict": (_i, [_vp, _i, _vp, _i, _i]),
         "sf_interpolate": (_i, [_vp, _i, _d, _vp, _i, _i]),
         "sf_norm": (_i, [_vp, _i, _i, _P]),
@@ -213,6 +215,17 @@ def sf_apply_laplacian(level, out, x):
 
 def sf_jacobi(level, out, x, f, omega=2.0 / 3.0):
     _check(lib().sf_jacobi(level, out, x, f, float(omega)))
+
+
+def sf_smooth_chebyshev(level, x, rhs, a, b, degree, lo, hi):
+    _check(lib().sf_smooth_chebyshev(level, x, rhs, float(a), float(b), int(degree), float(lo),
+                                     float(hi)))
+
+
+def sf_lambda_max(level, v, a, b, iters=30, start=True):
+    out = C.c_double()
+    _check(lib().sf_lambda_max(level, v, float(a), float(b), int(iters), int(start), C.byref(out)))
+    return out.value
 
 
 def sf_residual(level, res, x, rhs, a, b):

@@ -394,3 +394,50 @@ def test_cc_decomposition_invariance(sf):
         sf.sf_jacobi(L.handle, sf.SF_TMP, sf.SF_U, sf.SF_F, 2.0 / 3.0)
         outs.append(L.download(sf.SF_TMP))
     assert np.array_equal(outs[0], outs[1])
+
+
+# ------------------------------------------------------- NEXT-3 (Chebyshev smoother)
+def start_vector(shape):
+    nz, ny, nx = shape
+    k, j, i = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    return 1.0 + ((7 * i + 13 * j + 29 * k) % 17) / 17.0
+
+
+@pytest.mark.parametrize("shape", [(16, 16, 16), (8, 6, 10), (20, 64, 64)])
+def test_chebyshev_and_lambda_max(sf, oracle, shape):
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.random_coeffs(nx, ny, nz, 8)
+    L = make_level(sf, shape, coeffs)
+    sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.0, 1.0, *coeffs)
+    lam = sf.sf_lambda_max(L.handle, sf.SF_U, 1.0, 1.0, 20, True)
+    lam_o = P.lambda_max(start_vector(shape), 20)
+    assert abs(lam / lam_o - 1) < 1e-12
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    for degree in (1, 4, 5):
+        L.upload(sf.SF_U, x)
+        sf.sf_smooth_chebyshev(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, degree, 0.1 * lam, 1.05 * lam)
+        exp = P.chebyshev(x, f, degree, 0.1 * lam, 1.05 * lam)
+        assert rel(L.download(sf.SF_U), exp) < TOL
+
+
+@pytest.mark.parametrize("graph", [0, 1])
+def test_chebyshev_multigrid(sf, oracle, graph):
+    n = 32
+    L, M, O = mg_pair(sf, oracle, n, smoother=sf.SF_SMOOTH_CHEBY, cheby_degree=2,
+                      use_graph=graph)
+    O.set_chebyshev(2)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    u = np.zeros((n, n, n))
+    for _ in range(2):
+        M.vcycle(0)
+        u = O.vcycle(u, f)
+        assert rel(L.download(sf.SF_U), u) < 1e-11
+    L.upload(sf.SF_U, np.zeros((n, n, n)))
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10)
+    u_o, hist_o = O.solve(f, fcycle=True, rtol=1e-10)
+    assert cyc == len(hist_o) and rel(L.download(sf.SF_U), u_o) < 1e-10

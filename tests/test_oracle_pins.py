@@ -446,3 +446,61 @@ def test_cc_jacobi_brute_force(oracle):
     # the damped Jacobi iteration converges (spectral radius < 1 for SPD L, omega 2/3)
     Jm = np.eye(K.shape[0]) - (2.0 / 3.0) * K / np.diag(K)[:, None]
     assert np.abs(np.linalg.eigvals(Jm)).max() < 1.0
+
+
+# ------------------------------------------------------- NEXT-3 (Chebyshev smoother)
+def test_chebyshev_is_scaled_chebyshev_polynomial(oracle):
+    """After m steps the error is P_m(D^-1 A) e_0 with
+    P_m(l) = T_m((theta - l)/delta) / T_m(theta/delta) (Saad Alg. 12.1): checked
+    through the eigen-decomposition of the dense D^-1 A."""
+    n, h = 4, 0.25
+    shape = (n, n, n)
+    P = oracle.Problem(oracle.Grid(n, n, n, h), 1.0, 1.0, *I.random_coeffs(n, n, n, 3))
+    A = dense_op(P, shape)
+    D = np.diag(A)
+    M = A / D[:, None]                       # D^-1 A, similar to the SPD D^-1/2 A D^-1/2
+    lam, V = np.linalg.eig(M)
+    lam, V = lam.real, V.real
+    hi, lo = 1.1 * lam.max(), 0.1 * lam.max()
+    theta, delta = (hi + lo) / 2, (hi - lo) / 2
+    f = I.random_field(shape, 1)
+    xs = np.linalg.solve(A, f.ravel())
+    x0 = I.random_field(shape, 0)
+    for m in (1, 2, 4):
+        Tm = np.polynomial.chebyshev.Chebyshev.basis(m)
+        pm = Tm((theta - lam) / delta) / Tm(theta / delta)
+        e0 = np.linalg.solve(V, x0.ravel() - xs)
+        exp = xs + V @ (pm * e0)
+        got = P.chebyshev(x0, f, m, lo, hi)
+        assert np.abs(got.ravel() - exp).max() < 1e-10 * np.abs(exp).max()
+
+
+def test_chebyshev_smooths_and_lambda_max(oracle):
+    n, h = 8, 1.0 / 8
+    shape = (n, n, n)
+    P = oracle.Problem(oracle.Grid(n, n, n, h), 1.0, 1.0, *I.hpgmg_coeffs(n, n, n))
+    A = dense_op(P, shape)
+    lam_true = np.abs(np.linalg.eigvals(A / np.diag(A)[:, None])).max()
+    lam10 = P.lambda_max(I.random_field(shape, 5), 10)
+    lam = P.lambda_max(I.random_field(shape, 5), 200)
+    assert abs(lam / lam_true - 1) < 5e-3 and abs(lam / lam_true - 1) < abs(lam10 / lam_true - 1)
+    # the high-frequency end of the spectrum is damped by at least 1/T_m(sigma)
+    f = np.zeros(shape)
+    x = I.random_field(shape, 6)
+    lo, hi = 0.1 * 1.1 * lam, 1.1 * lam
+    y = P.chebyshev(x, f, 4, lo, hi)
+    J = lambda v: v.ravel() @ A @ v.ravel()
+    assert J(y) < J(x)
+
+
+def test_chebyshev_vcycle_converges(oracle):
+    """V-cycles with Chebyshev smoothing (4 steps pre/post, interval from the
+    power-iteration lambda_max) converge with rho <= 0.25 (reading R-16)."""
+    n = 16
+    mg = _mg(oracle, n)
+    mg.set_chebyshev(2)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    u, hist = mg.solve(f)
+    assert hist[-1] < 1e-10 and len(hist) <= 12
+    rho = [hist[i + 1] / hist[i] for i in range(1, len(hist) - 1)]
+    assert max(rho) <= 0.25
