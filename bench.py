@@ -425,6 +425,14 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
                           "frac_of_peak": bpc * cells / (m_ / 1e3) / 1e9 / pk, "bytes_per_cell": bpc}
         fig7["vc_gsrb_pair"] = {"ms": ms, "gstencil_s": cells / (ms / 1e3) / 1e9, "alg_gbs": gbs,
                                 "frac_of_peak": gbs / pk, "bytes_per_cell": 64}
+        # NEXT-3 Chebyshev step (72 B/cell: x, x_prev, rhs, alpha, beta x3, Dinv, out)
+        lam = sf.sf_lambda_max(G.handle, sf.SF_TMP, 1.0, 1.0, 10, True)
+        mc = per_call(lambda: sf.sf_smooth_chebyshev(G.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1,
+                                                     0.13 * lam, 1.05 * lam), 30)
+        fig7["vc_chebyshev_step"] = {"ms": mc, "gstencil_s": cells / (mc / 1e3) / 1e9,
+                                     "alg_gbs": 72 * cells / (mc / 1e3) / 1e9,
+                                     "frac_of_peak": 72 * cells / (mc / 1e3) / 1e9 / pk,
+                                     "bytes_per_cell": 72}
         out["fig7_256"] = fig7
         out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms,
                           "frac_of_kernel_compulsory": GSRB_KERNEL_BYTES_PER_CELL * cells / (ms / 1e3)
