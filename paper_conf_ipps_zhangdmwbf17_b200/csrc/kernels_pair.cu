@@ -191,42 +191,49 @@ __global__ void __launch_bounds__(PX* PY) cc_pair_kernel(PV v, double* __restric
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     if (i >= v.nx || j >= v.ny) return;
-    for (int k = k0; k < k1; k++) {
-        const long c = sf_ix(v, i, j, k);
+    const double h2w6 = h2w / 6.0;
+    // register streaming along z: the column's planes k-1, k, k+1 ride in registers
+    long c = sf_ix(v, i, j, k0);
+    double2 xb = ld2(x + c - v.ks), xc = ld2(x + c);
+    for (int k = k0; k < k1; k++, c += v.ks) {
         const int gk = v.z0 + k;
-        const double2 xc = ld2(x + c);
+        const double2 xtr = ld2(x + c + v.ks);
         double xw = (i == 0) ? -xc.x : x[c - 1];
         double xe = (i + 1 == v.nx - 1) ? -xc.y : x[c + 2];
         double2 xs = ld2(x + c - v.js), xn = ld2(x + c + v.js);
-        double2 xb = ld2(x + c - v.ks), xt = ld2(x + c + v.ks);
+        double2 xbb = xb, xt = xtr;
         if (j == 0) xs = make_double2(-xc.x, -xc.y);
         if (j == v.ny - 1) xn = make_double2(-xc.x, -xc.y);
-        if (gk == 0) xb = make_double2(-xc.x, -xc.y);
+        if (gk == 0) xbb = make_double2(-xc.x, -xc.y);
         if (gk == v.gnz - 1) xt = make_double2(-xc.x, -xc.y);
         double sa = xc.x - xc.y;
         sa += xc.x - xw;
         sa += xc.x - xn.x;
         sa += xc.x - xs.x;
         sa += xc.x - xt.x;
-        sa += xc.x - xb.x;
+        sa += xc.x - xbb.x;
         double sb = xc.y - xe;
         sb += xc.y - xc.x;
         sb += xc.y - xn.y;
         sb += xc.y - xs.y;
         sb += xc.y - xt.y;
-        sb += xc.y - xb.y;
+        sb += xc.y - xbb.y;
         double2 o;
         if (JACOBI) {
+            // D^-1 = h^2 / (6 + boundary faces): one shared factor for interior cells
             const int nyz = (j == 0) + (j == v.ny - 1) + (gk == 0) + (gk == v.gnz - 1);
+            const int na = nyz + (i == 0), nb = nyz + (i + 1 == v.nx - 1);
             const double2 fv = ld2(f + c);
-            const double da = 6.0 + nyz + (i == 0), db = 6.0 + nyz + (i + 1 == v.nx - 1);
-            o.x = xc.x + h2w * (fv.x - hm2 * sa) / da;
-            o.y = xc.y + h2w * (fv.y - hm2 * sb) / db;
+            const double wa = na ? h2w / (6.0 + na) : h2w6, wb = nb ? h2w / (6.0 + nb) : h2w6;
+            o.x = xc.x + wa * (fv.x - hm2 * sa);
+            o.y = xc.y + wb * (fv.y - hm2 * sb);
         } else {
             o.x = hm2 * sa;
             o.y = hm2 * sb;
         }
-        *(double2*)(out + c) = o;
+        __stcs((double2*)(out + c), o);
+        xb = xc;
+        xc = xtr;
     }
 }
 
