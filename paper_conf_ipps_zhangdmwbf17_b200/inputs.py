@@ -130,6 +130,16 @@ def manufactured(nx, ny, nz, a, b, h=None):
         np.broadcast_to(f, (nz, ny, nx)))
 
 
+def manufactured_at(nx, ny, nz, h, idx):
+    """Exact solution u at the cell-centre sub-grid idx = (i_array, j_array,
+    k_array); returns shape (len(k), len(j), len(i))."""
+    L = (nx * h, ny * h, nz * h)
+    x = ((np.asarray(idx[0]) + 0.5) * h / L[0])[None, None, :]
+    y = ((np.asarray(idx[1]) + 0.5) * h / L[1])[None, :, None]
+    z = ((np.asarray(idx[2]) + 0.5) * h / L[2])[:, None, None]
+    return _X(x) * _X(y) * _X(z)
+
+
 def split_slabs(arr, kind, parts):
     """Split a global array into z-slabs for `parts` parts (layout only).
 
