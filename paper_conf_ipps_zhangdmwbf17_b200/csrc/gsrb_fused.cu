@@ -398,14 +398,19 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         // step before its first read; the two parents a thread needs for plane
         // p are loaded (L2) one step earlier still.
         const int ep0 = tid, ep1 = tid + NT;   // x-box pairs of this thread
-        auto e_addr = [&](int pr, int p) -> long {
+        // in-plane offsets of their coarse parents (fixed per item): only the
+        // coarse plane (p >> 1) changes from step to step
+        auto e_inplane = [&](int pr) -> long {
             const int r = pr / (W / 2), c2 = pr - r * (W / 2);
-            const int I = x0 / 2 - 1 + c2, J = y0 / 2 - 1 + (r >> 1), K = (p >> 1) + cv.zoff;
-            return (long)(K + SF_GZ) * cv.ks + (long)(J + SF_GY) * cv.js + SF_OX + I;
+            const int I = x0 / 2 - 1 + c2, J = y0 / 2 - 1 + (r >> 1);
+            return (long)(J + SF_GY) * cv.js + SF_OX + I;
         };
+        const long eo0 = INTERP ? e_inplane(ep0) : 0;
+        const long eo1 = (INTERP && ep1 < XPAIRS) ? e_inplane(ep1) : eo0;
         auto load_e = [&](int p, double& e0, double& e1) {
-            e0 = __ldg(cv.e + e_addr(ep0, p));
-            e1 = (ep1 < XPAIRS) ? __ldg(cv.e + e_addr(ep1, p)) : 0.0;
+            const double* ep = cv.e + (long)((p >> 1) + cv.zoff + SF_GZ) * cv.ks;
+            e0 = __ldg(ep + eo0);
+            e1 = __ldg(ep + eo1);
         };
         auto correct = [&](int p, double e0, double e1) {
             double* X = Xs + md(p, NXS) * XSLOT;
