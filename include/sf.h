@@ -124,6 +124,17 @@ const char* sf_version(void);
 sf_status sf_comm_create_local(sf_comm** out, int nparts);
 sf_status sf_get_unique_id(unsigned char id[128]);
 sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[128], int nranks, int rank);
+/* Test transport: one part per PROCESS with all
+ * processes on the same GPU (NCCL refuses two ranks per device), halos and
+ * agglomeration by copies from peer buffers opened through CUDA IPC, host
+ * synchronisation and scalar reductions through the caller's all-gather
+ * callback (e.g. torch.distributed/gloo).  allgather(send, n, recv, user)
+ * must gather n bytes from every rank into recv (rank order) and return 0.
+ * Levels created with such a comm (and their agglomerated coarse levels) are
+ * collective; CUDA graphs are not used with it. */
+typedef int (*sf_host_allgather_fn)(const void* send, size_t nbytes, void* recv, void* user);
+sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank, sf_host_allgather_fn allgather,
+                                 void* user);
 sf_status sf_comm_destroy(sf_comm* comm);
 /* number of parts in the job, parts local to this process, first local part */
 sf_status sf_comm_info(const sf_comm* comm, int* nparts, int* nlocal, int* first);

@@ -9,6 +9,8 @@
 #include <dlfcn.h>
 #include <nccl.h>
 
+#include <cuda.h>
+
 #include <mutex>
 
 #include "sf_internal.h"
@@ -107,6 +109,79 @@ extern "C" sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[1
     return SF_OK;
 }
 
+extern "C" sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank,
+                                            sf_host_allgather_fn fn, void* user) {
+    if (!out || !fn || nranks < 1 || rank < 0 || rank >= nranks)
+        return sf_fail(SF_ERR_INVALID, "bad arguments");
+    sf_comm* c = new sf_comm();
+    c->kind = 2;
+    c->nparts = nranks; c->nlocal = 1; c->first = rank;
+    c->rank = rank; c->nranks = nranks;
+    c->nccl = nullptr;
+    c->hostfn = fn;
+    c->hostuser = user;
+    *out = c;
+    return SF_OK;
+}
+
+namespace {
+sf_status host_allgather(const sf_comm* c, const void* send, size_t n, void* recv) {
+    if (c->hostfn(send, n, recv, c->hostuser) != 0)
+        return sf_fail(SF_ERR_NCCL, "host all-gather callback failed");
+    return SF_OK;
+}
+sf_status host_barrier(const sf_comm* c) {
+    char b = 0;
+    std::vector<char> r(c->nranks);
+    return host_allgather(c, &b, 1, r.data());
+}
+double* peer_field(const sf_level* L, int rank, const double* mine) {
+    return (double*)(L->peer[rank] + ((const char*)mine - (const char*)L->buf));
+}
+}  // namespace
+
+sf_status sf_ipc_register(sf_level* L, const sf_comm* c) {
+    if (!c || c->kind != 2) return SF_OK;
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    // base of the allocation holding the level buffer (a torch block may sit inside one)
+    static decltype(&cuMemGetAddressRange) range = nullptr;
+    if (!range) {
+        cudaDriverEntryPointQueryResult q;
+        void* fn = nullptr;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess || !fn)
+            return sf_fail(SF_ERR_CUDA, "cuMemGetAddressRange unavailable");
+        range = (decltype(range))fn;
+    }
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (CUdeviceptr)L->buf) != CUDA_SUCCESS)
+        return sf_fail(SF_ERR_CUDA, "cuMemGetAddressRange failed");
+    struct Rec {
+        cudaIpcMemHandle_t h;
+        unsigned long long off;
+    } mine, all[64];
+    if (c->nranks > 64) return sf_fail(SF_ERR_INVALID, "hostipc supports <= 64 ranks");
+    SF_CUDA(cudaIpcGetMemHandle(&mine.h, (void*)base));
+    mine.off = (unsigned long long)((char*)L->buf - (char*)base);
+    SF_TRY(host_allgather(c, &mine, sizeof(Rec), all));
+    L->peer.assign(c->nranks, nullptr);
+    for (int r = 0; r < c->nranks; r++) {
+        if (r == c->rank) continue;
+        void* p = nullptr;
+        SF_CUDA(cudaIpcOpenMemHandle(&p, all[r].h, cudaIpcMemLazyEnablePeerAccess));
+        L->ipc_opened.push_back(p);
+        L->peer[r] = (char*)p + all[r].off;
+    }
+    return host_barrier(c);
+}
+
+void sf_ipc_close(sf_level* L) {
+    for (void* p : L->ipc_opened) cudaIpcCloseMemHandle(p);
+    L->ipc_opened.clear();
+    L->peer.clear();
+}
+
 extern "C" sf_status sf_comm_destroy(sf_comm* c) {
     if (!c) return SF_OK;
     if (c->kind == 1 && c->nccl) g_nccl.commDestroy((ncclComm_t)c->nccl);
@@ -141,6 +216,21 @@ sf_status sf_halo(sf_level* L, int field, int depth) {
         }
         return SF_OK;
     }
+    if (L->comm->kind == 2) {  // pull the neighbours' boundary planes through IPC
+        const sf_comm* c = L->comm;
+        int r = c->rank, n = c->nranks;
+        double* x = L->parts[0].f[field];
+        SF_CUDA(cudaStreamSynchronize(L->stream));
+        SF_TRY(host_barrier(c));
+        if (r > 0)
+            SF_CUDA(cudaMemcpyAsync(x + lo_dst, peer_field(L, r - 1, x) + hi_src, cnt * sizeof(double),
+                                    cudaMemcpyDeviceToDevice, L->stream));
+        if (r < n - 1)
+            SF_CUDA(cudaMemcpyAsync(x + hi_dst, peer_field(L, r + 1, x) + lo_src, cnt * sizeof(double),
+                                    cudaMemcpyDeviceToDevice, L->stream));
+        SF_CUDA(cudaStreamSynchronize(L->stream));
+        return host_barrier(c);
+    }
     ncclComm_t comm = (ncclComm_t)L->comm->nccl;
     int r = L->comm->rank, n = L->comm->nranks;
     double* x = L->parts[0].f[field];
@@ -162,6 +252,24 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
     const sf_comm* cm = C->rep_comm;
     if (!cm || cm->kind == 0) return SF_OK;
     if (cm->nranks != parts) return sf_fail(SF_ERR_SHAPE, "agglomeration across %d parts", parts);
+    if (cm->kind == 2) {  // every rank copies the other ranks' planes from their buffers
+        double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
+        size_t cnt = (size_t)lnz_per_part * C->ks;
+        SF_CUDA(cudaStreamSynchronize(C->stream));
+        SF_TRY(host_barrier(cm));
+        for (int q = 0; q < parts; q++) {
+            if (q == cm->rank) continue;
+            SF_CUDA(cudaMemcpyAsync(base + q * cnt, peer_field(C, q, base) + q * cnt,
+                                    cnt * sizeof(double), cudaMemcpyDeviceToDevice, C->stream));
+        }
+        if (field == SF_BETA_K && cm->rank != parts - 1) {
+            double* top = base + (size_t)C->gnz * C->ks;
+            SF_CUDA(cudaMemcpyAsync(top, peer_field(C, parts - 1, top), C->ks * sizeof(double),
+                                    cudaMemcpyDeviceToDevice, C->stream));
+        }
+        SF_CUDA(cudaStreamSynchronize(C->stream));
+        return host_barrier(cm);
+    }
     ncclComm_t comm = (ncclComm_t)cm->nccl;
     double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
     size_t cnt = (size_t)lnz_per_part * C->ks;
@@ -174,7 +282,20 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
 }
 
 sf_status sf_allreduce_scalar(const sf_comm* cm, double* dev, int op, cudaStream_t s) {
-    if (!cm || cm->kind != 1 || cm->nranks == 1) return SF_OK;
+    if (!cm || cm->kind == 0 || cm->nranks == 1) return SF_OK;
+    if (cm->kind == 2) {
+        double v;
+        SF_CUDA(cudaMemcpyAsync(&v, dev, sizeof(double), cudaMemcpyDeviceToHost, s));
+        SF_CUDA(cudaStreamSynchronize(s));
+        std::vector<double> all(cm->nranks);
+        SF_TRY(host_allgather(cm, &v, sizeof(double), all.data()));
+        double r = all[0];
+        for (int q = 1; q < cm->nranks; q++)
+            r = op == 0 ? ((all[q] > r || all[q] != all[q]) ? all[q] : r) : r + all[q];
+        SF_CUDA(cudaMemcpyAsync(dev, &r, sizeof(double), cudaMemcpyHostToDevice, s));
+        SF_CUDA(cudaStreamSynchronize(s));
+        return SF_OK;
+    }
     SF_NCCL(g_nccl.allReduce(dev, dev, 1, ncclDouble, op == 0 ? ncclMax : ncclSum,
                              (ncclComm_t)cm->nccl, s));
     return SF_OK;

@@ -454,7 +454,7 @@ sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, doub
         dinv_scale_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[w_id], depth, sumsq);
         SF_LAUNCHED();
     }
-    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+    if (L->comm && L->comm->kind != 0 && L->nparts > 1)
         SF_TRY(sf_allreduce_scalar(L->comm, sumsq, 1, L->stream));
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);

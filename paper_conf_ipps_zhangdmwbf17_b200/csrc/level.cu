@@ -142,6 +142,13 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
     }
     e = cudaMemsetAsync(L->buf, 0, need, L->stream);
     if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+    if (comm && comm->kind == 2) {
+        sf_status s = sf_ipc_register(L, comm);
+        if (s != SF_OK) {
+            sf_level_destroy(L);
+            return s;
+        }
+    }
     *out = L;
     return SF_OK;
 }
@@ -149,6 +156,7 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
 extern "C" sf_status sf_level_destroy(sf_level* L) {
     if (!L) return SF_OK;
     cudaStreamSynchronize(L->stream);
+    sf_ipc_close(L);
     if (L->owns) cudaFree(L->buf);
     cudaFreeHost(L->hscratch);
     delete L;
@@ -421,7 +429,7 @@ extern "C" sf_status sf_interpolate(sf_level* F, int ff, double prescale, sf_lev
 
 sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst) {
     SF_TRY(k_norm(L, field, kind, dst));
-    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+    if (L->comm && L->comm->kind != 0 && L->nparts > 1)
         SF_TRY(sf_allreduce_scalar(L->comm, dst, kind == SF_NORM_MAX ? 0 : 1, L->stream));
     return SF_OK;
 }

@@ -144,7 +144,16 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
             sf_mg_destroy(m);
             return s;
         }
-        if (!P.distributed) C->rep_comm = F->comm ? F->comm : F->rep_comm;
+        if (!P.distributed) {
+            C->rep_comm = F->comm ? F->comm : F->rep_comm;
+            s = sf_ipc_register(C, C->rep_comm);   // kind-2 comm: collective
+            if (s != SF_OK) {
+                m->lv.push_back(C);
+                m->own.push_back(true);
+                sf_mg_destroy(m);
+                return s;
+            }
+        }
         m->lv.push_back(C);
         m->own.push_back(true);
     }
@@ -266,7 +275,7 @@ static sf_status check(sf_mg* m) {
     sf_level* L = m->lv[0];
     if (pair_ok(L)) {  // max|f - Au| reduced in the residual pass, nothing stored
         SF_TRY(k_residual_pair(L, -1, SF_U, SF_F, m->a, m->b, L->dscratch));
-        if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+        if (L->comm && L->comm->kind != 0 && L->nparts > 1)
             SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
     } else {
         SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
@@ -291,7 +300,7 @@ static sf_status first_pair_check(sf_mg* m) {
     SF_TRY(sf_halo(L, SF_U, 2));
     SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
     sf_swap_fields(L, SF_U, SF_TMP);
-    if (L->comm && L->comm->kind == 1 && L->nparts > 1)
+    if (L->comm && L->comm->kind != 0 && L->nparts > 1)
         SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
     return to_host(L);
 }
@@ -299,6 +308,7 @@ static sf_status first_pair_check(sf_mg* m) {
 static bool graphs_allowed(const sf_mg* m) {
     if (!m->o.use_graph || m->graph_failed) return false;
     if (m->lv[0]->stream == nullptr) return false;  // legacy stream cannot be captured
+    if (m->lv[0]->comm && m->lv[0]->comm->kind == 2) return false;  // host-synchronised halos
     // the fused smoother swaps U/TMP per pair; only an even count per captured
     // sequence leaves the host-side mapping unchanged for replays
     if (m->o.smoother == SF_SMOOTH_CHEBY)   // an n-step application ends with swap(U, [U,R,TMP][n%3]):

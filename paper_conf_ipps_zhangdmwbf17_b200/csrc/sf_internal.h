@@ -21,12 +21,14 @@
 #define SF_GZ 2
 
 struct sf_comm {
-    int kind;          // 0 = local (all parts in this process), 1 = NCCL
+    int kind;          // 0 = local (all parts in this process), 1 = NCCL, 2 = host+IPC (tests)
     int nparts;        // parts in the whole job
     int nlocal;        // parts held by this process
     int first;         // global index of the first local part
     int rank, nranks;
     void* nccl;        // ncclComm_t
+    sf_host_allgather_fn hostfn;  // kind 2
+    void* hostuser;
 };
 
 struct SfPart {
@@ -50,6 +52,8 @@ struct sf_level {
     bool owns;
     double* dscratch;          // device scalars (norms)
     double* hscratch;          // pinned host scalars
+    std::vector<char*> peer;   // kind-2 comm: peer ranks' level buffers (CUDA IPC), by rank
+    std::vector<void*> ipc_opened;
 };
 
 // Part view passed to kernels by value.  Kernels must only index f[] with
@@ -140,5 +144,8 @@ sf_status sf_halo(sf_level* L, int field, int depth);
 // Replicated coarse level C receives, on every process, the planes each part
 // of the distributed fine level F wrote into it (in-place all-gather).
 sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part);
+// kind-2 comm: open the peers' buffers of level L (collective)
+sf_status sf_ipc_register(sf_level* L, const sf_comm* c);
+void sf_ipc_close(sf_level* L);
 // Reduce a device scalar over ranks (op 0 = max, 1 = sum); in place.
 sf_status sf_allreduce_scalar(const sf_comm* comm, double* dev, int op, cudaStream_t s);

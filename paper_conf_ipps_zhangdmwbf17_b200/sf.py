@@ -42,6 +42,7 @@ EXPORTS = [
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
+    "sf_comm_create_hostipc",
 ]
 
 
@@ -61,6 +62,8 @@ class MgOpts(C.Structure):
 _lib = None
 _vp, _d, _i = C.c_void_p, C.c_double, C.c_int
 _P = C.POINTER(C.c_double)
+# int (*)(const void* send, size_t nbytes, void* recv, void* user)
+HOST_ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 
 
 def lib():
@@ -79,6 +82,7 @@ def lib():
         "sf_comm_create_local": (_i, [C.POINTER(_vp), _i]),
         "sf_get_unique_id": (_i, [C.c_char_p]),
         "sf_comm_create_nccl": (_i, [C.POINTER(_vp), C.c_char_p, _i, _i]),
+        "sf_comm_create_hostipc": (_i, [C.POINTER(_vp), _i, _i, HOST_ALLGATHER, _vp]),
         "sf_comm_destroy": (_i, [_vp]),
         "sf_comm_info": (_i, [_vp, C.POINTER(_i), C.POINTER(_i), C.POINTER(_i)]),
         "sf_level_bytes_needed": (_i, [_i, _i, _i, _vp, C.POINTER(C.c_size_t)]),
@@ -150,6 +154,13 @@ def sf_get_unique_id():
 def sf_comm_create_nccl(uid, nranks, rank):
     h = _vp()
     _check(lib().sf_comm_create_nccl(C.byref(h), uid, int(nranks), int(rank)))
+    return h
+
+
+def sf_comm_create_hostipc(nranks, rank, allgather_cb):
+    """allgather_cb must be a HOST_ALLGATHER the caller keeps alive."""
+    h = _vp()
+    _check(lib().sf_comm_create_hostipc(C.byref(h), int(nranks), int(rank), allgather_cb, None))
     return h
 
 
@@ -330,6 +341,32 @@ class Comm:
         from . import parallel
         uid, rank, world = parallel.broadcast_unique_id(group)
         return cls(sf_comm_create_nccl(uid, world, rank), world, 1, rank)
+
+    @classmethod
+    def hostipc(cls, group=None):
+        """Test transport: one part per rank of a (gloo) torch.distributed group,
+        all ranks on the SAME GPU; peer buffers through CUDA IPC, host
+        synchronisation through ``group`` (include/sf.h, sf_comm_create_hostipc)."""
+        import torch
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+
+        def allgather(send, n, recv, _user):
+            try:
+                src = torch.frombuffer(bytearray(C.string_at(send, n)), dtype=torch.uint8) if n else \
+                    torch.empty(0, dtype=torch.uint8)
+                outs = [torch.empty(n, dtype=torch.uint8) for _ in range(world)]
+                dist.all_gather(outs, src.clone(), group=group)
+                C.memmove(recv, torch.cat(outs).numpy().tobytes(), n * world)
+                return 0
+            except Exception as e:  # noqa: BLE001 -- reported through the C status
+                print(f"hostipc all-gather failed: {e!r}")
+                return 1
+
+        cb = HOST_ALLGATHER(allgather)
+        c = cls(sf_comm_create_hostipc(world, rank, cb), world, 1, rank)
+        c._cb = cb          # keep the trampoline alive as long as the comm
+        return c
 
     def close(self):
         if self.h:
