@@ -304,8 +304,9 @@ def main():
             "gpu_launches": launches,
             "roofline": roof,
         }
-        line.update({k: v for k, v in side.items() if k in ("e2e", "gsrb_c3", "vcycle",
-                                                             "cpu_baseline", "fig7_256")})
+        line.update({k: v for k, v in side.items() if k in (
+            "e2e", "gsrb_c3", "vcycle", "fcycle", "read_bw", "cpu_baseline", "fig7_256",
+            "gsrb_size_sweep")})
         print(json.dumps(line), flush=True)
     M.close()
     L.close()
@@ -340,6 +341,16 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
     # V-cycle alone (finest level; the solve = 1 F + cyc-1 V)
     vms = timed(lambda: sf.sf_vcycle(M.handle, 0), 5, warm=2)
     out["vcycle"] = {"ms": vms, "dof_s": dof_local * world / (vms / 1e3)}
+    # C4's figure of merit: one F-cycle (HPGMG FOM), same level and operator
+    fms = timed(lambda: sf.sf_fcycle(M.handle), 3, warm=1)
+    out["fcycle"] = {"ms": fms, "dof_s": dof_local * world / (fms / 1e3),
+                     "note": "C4 / HPGMG FOM: one F-cycle (PL up, one V per level) on the workload"}
+    # read-dominated bandwidth (PAPER.md:684-696's dot-product bound): L2 norm of u
+    # (8 B/cell, read-only); each call ends with an 8-byte D2H and a host sync
+    rms = timed(lambda: sf.sf_norm(L.handle, sf.SF_U, sf.SF_NORM_L2), 10, warm=2)
+    out["read_bw"] = {"ms": rms, "gbs": 8 * dof_local / (rms / 1e3) / 1e9,
+                      "kernel": "norm_pair_kernel (sum of squares, 8 B/cell read)",
+                      "note": "includes per-call host sync; context for the copy peak"}
     # pairs on the finest level per solve: F: (pre+post) ; each V: 4 pairs
     pairs_per_solve = 4 * cyc
     out["fine_pair_share"] = None
@@ -434,6 +445,19 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
                                      "frac_of_peak": 72 * cells / (mc / 1e3) / 1e9 / pk,
                                      "bytes_per_cell": 72}
         out["fig7_256"] = fig7
+        # Fig 8 analogue: fused RB pair throughput vs level size
+        sweep = {}
+        for n_ in (32, 64, 128):
+            Gs = sf.Level(n_, n_, n_, 1.0 / n_, stream=s)
+            sf.sf_init_problem(Gs.handle, 1, 1.0, 1.0, 1)
+            sf.sf_rebuild_operator(Gs.handle, 1.0, 1.0)
+            m_ = per_call(lambda: sf.sf_smooth_gsrb(Gs.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1,
+                                                    sf.SF_SMOOTH_FUSED), 200)
+            sweep[str(n_)] = {"ms": m_, "gstencil_s": n_**3 / (m_ / 1e3) / 1e9,
+                              "alg_gbs": 64 * n_**3 / (m_ / 1e3) / 1e9}
+            Gs.close()
+        sweep[str(n3)] = {"ms": ms, "gstencil_s": cells / (ms / 1e3) / 1e9, "alg_gbs": gbs}
+        out["gsrb_size_sweep"] = sweep
         out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms,
                           "frac_of_kernel_compulsory": GSRB_KERNEL_BYTES_PER_CELL * cells / (ms / 1e3)
                           / 1e9 / pk,

@@ -253,6 +253,89 @@ sf_status sf_launch_count(long long* count, int reset);
 /* Per-launch device time of the most recent sf_smooth_gsrb kernels is not
  * tracked here; bench.py times sf_smooth_gsrb with CUDA events. */
 
+/* ------------------------------------------- generic stencils (NEXT-4)
+ * The paper's language core (Table I, Fig 4): a Stencil
+ * associates an expression over meshes (Components = weight arrays applied to
+ * a mesh; weights may themselves be mesh expressions -- variable coefficients),
+ * an output mesh (possibly one of the inputs: in place) and a domain that is a
+ * union of strided RectDomains whose negative bounds are relative to the grid
+ * size; a StencilGroup runs stencils consecutively.  Compiling a group renders
+ * ONE CUDA kernel for it and compiles it at run time for sm_100a (NVRTC), the
+ * B200 counterpart of the paper's JIT micro-compilers.
+ *
+ * Coordinates (reading R-17): ghost-inclusive, one ghost layer as in Fig 4 --
+ * interior cell i of axis d has coordinate i+1, so interior = [1, n_d] and the
+ * Dirichlet ghost layer is 0 and n_d+1.  Rect bounds b < 0 mean N_d + b with
+ * N_d = n_d + 2 (so hi = -1 is the exclusive end n_d+1); lo inclusive, hi
+ * exclusive, stride >= 1; stride 0 makes the axis the single coordinate lo
+ * (Fig 4 l.17's boundary domain).  A READ node reads mesh `mesh` of the output level
+ * (src 0) or of the source level (src 1) at, per axis,
+ *     q = floor((mul*p + pre) / div) + off            (p = output point)
+ * -- plain offsets have mul = div = 1, pre = 0; restriction reads a fine level
+ * at 2p + o (mul 2), P0 interpolation a coarse level at floor((p+1)/2) (div 2,
+ * pre 1).  Reads may reach the storage ghost zone (x: OX = 4, y/z: 2 layers).
+ *
+ * Semantics: every point of a stencil's domain is computed from the values
+ * before the stencil (points of one stencil are independent); stencils of a
+ * group apply in order.  sf_stencil_apply verifies this with the paper's
+ * Diophantine analysis (exact per-axis lattice intersection
+ * by the extended Euclidean algorithm): an in-place stencil whose reads of its
+ * output mesh hit points it writes, other than each point's own, is rejected
+ * (SF_ERR_INVALID); consecutive independent stencils (no RAW/WAR/WAW overlap)
+ * share one launch, a dependence starts a new launch (the paper's greedy
+ * barrier placement). */
+typedef struct sf_stencil sf_stencil;
+enum sf_sx_op {
+    SF_SX_CONST = 0, /* value                                   */
+    SF_SX_READ = 1,  /* mesh[src](affine(p))                     */
+    SF_SX_ADD = 2,   /* node a + node b                          */
+    SF_SX_SUB = 3,   /* node a - node b                          */
+    SF_SX_MUL = 4,   /* node a * node b                          */
+    SF_SX_DIV = 5,   /* node a / node b                          */
+    SF_SX_NEG = 6    /* -node a                                  */
+};
+typedef struct {
+    int op;          /* sf_sx_op                                              */
+    int a, b;        /* operand node indices (must be < this node's index)     */
+    int mesh, src;   /* READ: sf_field, 0 = output level, 1 = source level     */
+    int off[3], mul[3], div[3], pre[3];   /* READ: affine map per axis (x,y,z) */
+    double value;    /* CONST                                                 */
+} sf_sx_node;
+typedef struct {
+    int lo[3], hi[3], stride[3];   /* x, y, z; see coordinates above          */
+} sf_rect;
+typedef struct {
+    int n_nodes;
+    const sf_sx_node* nodes;       /* expression DAG in topological order      */
+    int root;                      /* node whose value is stored               */
+    int out_mesh;                  /* sf_field written on the output level     */
+    int n_rects;                   /* DomainUnion: 1..SF_STENCIL_MAX_RECTS      */
+    const sf_rect* rects;
+} sf_stencil_desc;
+#define SF_STENCIL_MAX_RECTS 64
+/* Validate and render the group (host only; no GPU needed).  The descriptions
+ * are copied.  SF_ERR_INVALID on malformed input. */
+sf_status sf_stencil_compile(sf_stencil** out, const sf_stencil_desc* stencils, int n_stencils);
+/* The rendered CUDA source (NUL-terminated; *len = its length without NUL;
+ * copies min(cap-1, len) bytes when buf != NULL). */
+sf_status sf_stencil_source(const sf_stencil* s, char* buf, size_t cap, size_t* len);
+/* Run the group on `level` (output level, src 0) reading `src` (src 1; NULL =
+ * `level`).  JIT-compiles on first use (NVRTC, sm_100a; SF_ERR_CUDA if NVRTC or
+ * the device is unavailable).  Multi-part levels: same-level reads only, z
+ * halos of read meshes exchanged before each launch (depth <= 2); cross-level
+ * groups need single-part levels.  Enqueued on level's stream.  Errors:
+ * SF_ERR_SHAPE when a domain point or read falls outside the storage,
+ * SF_ERR_INVALID for a racy in-place stencil. */
+sf_status sf_stencil_apply(sf_stencil* s, sf_level* level, sf_level* src);
+/* Host-only dependence analysis of the group on a gnx x gny x gnz grid
+ * (src_is_output: source-level reads hit the output level): *phases = the
+ * launches apply would use; SF_ERR_INVALID for a racy in-place stencil. */
+sf_status sf_stencil_plan(const sf_stencil* s, int gnx, int gny, int gnz, int src_is_output,
+                          int* phases);
+/* Number of launches (dependence phases) the last apply used. */
+sf_status sf_stencil_phases(const sf_stencil* s, int* phases);
+sf_status sf_stencil_destroy(sf_stencil* s);
+
 #ifdef __cplusplus
 }
 #endif

@@ -25,7 +25,8 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
             ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=5", "-DSF_GSRB_SUFFIX=_t32"]),
            ("gsrb_fused.cu", "gsrb_fused_t64.o",
             ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t64"]),
-           ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", [])]
+           ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []),
+           ("stencil.cu", "stencil.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xptxas", "-v",

@@ -42,7 +42,8 @@ EXPORTS = [
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
-    "sf_comm_create_hostipc",
+    "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
+    "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy",
 ]
 
 
@@ -62,6 +63,25 @@ class MgOpts(C.Structure):
 _lib = None
 _vp, _d, _i = C.c_void_p, C.c_double, C.c_int
 _P = C.POINTER(C.c_double)
+# generic stencil IR (include/sf.h, NEXT-4)
+SF_SX_CONST, SF_SX_READ, SF_SX_ADD, SF_SX_SUB, SF_SX_MUL, SF_SX_DIV, SF_SX_NEG = range(7)
+
+
+class SxNode(C.Structure):
+    _fields_ = [("op", C.c_int), ("a", C.c_int), ("b", C.c_int), ("mesh", C.c_int),
+                ("src", C.c_int), ("off", C.c_int * 3), ("mul", C.c_int * 3),
+                ("div", C.c_int * 3), ("pre", C.c_int * 3), ("value", C.c_double)]
+
+
+class SfRect(C.Structure):
+    _fields_ = [("lo", C.c_int * 3), ("hi", C.c_int * 3), ("stride", C.c_int * 3)]
+
+
+class StencilDesc(C.Structure):
+    _fields_ = [("n_nodes", C.c_int), ("nodes", C.POINTER(SxNode)), ("root", C.c_int),
+                ("out_mesh", C.c_int), ("n_rects", C.c_int), ("rects", C.POINTER(SfRect))]
+
+
 # int (*)(const void* send, size_t nbytes, void* recv, void* user)
 HOST_ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 
@@ -84,6 +104,12 @@ def lib():
         "sf_comm_create_nccl": (_i, [C.POINTER(_vp), C.c_char_p, _i, _i]),
         "sf_comm_create_hostipc": (_i, [C.POINTER(_vp), _i, _i, HOST_ALLGATHER, _vp]),
         "sf_comm_destroy": (_i, [_vp]),
+        "sf_stencil_compile": (_i, [C.POINTER(_vp), C.POINTER(StencilDesc), _i]),
+        "sf_stencil_source": (_i, [_vp, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
+        "sf_stencil_apply": (_i, [_vp, _vp, _vp]),
+        "sf_stencil_plan": (_i, [_vp, _i, _i, _i, _i, C.POINTER(_i)]),
+        "sf_stencil_phases": (_i, [_vp, C.POINTER(_i)]),
+        "sf_stencil_destroy": (_i, [_vp]),
         "sf_comm_info": (_i, [_vp, C.POINTER(_i), C.POINTER(_i), C.POINTER(_i)]),
         "sf_level_bytes_needed": (_i, [_i, _i, _i, _vp, C.POINTER(C.c_size_t)]),
         "sf_level_create": (_i, [C.POINTER(_vp), _i, _i, _i, _d, _vp, _vp, _vp, C.c_size_t]),
@@ -162,6 +188,60 @@ def sf_comm_create_hostipc(nranks, rank, allgather_cb):
     h = _vp()
     _check(lib().sf_comm_create_hostipc(C.byref(h), int(nranks), int(rank), allgather_cb, None))
     return h
+
+
+def sf_stencil_compile(stencils):
+    """stencils: list of (nodes, root, out_mesh, rects); nodes = list of dicts with
+    SxNode fields, rects = list of (lo, hi, stride) 3-tuples (x, y, z)."""
+    descs = (StencilDesc * len(stencils))()
+    keep = []
+    for d, (nodes, root, out, rects) in zip(descs, stencils):
+        na = (SxNode * len(nodes))()
+        for x, n in zip(na, nodes):
+            x.op = n["op"]
+            x.a, x.b = n.get("a", 0), n.get("b", 0)
+            x.mesh, x.src = n.get("mesh", 0), n.get("src", 0)
+            for k, dflt in (("off", 0), ("mul", 1), ("div", 1), ("pre", 0)):
+                getattr(x, k)[:] = list(n.get(k, (dflt,) * 3))
+            x.value = float(n.get("value", 0.0))
+        ra = (SfRect * len(rects))()
+        for x, (lo, hi, st) in zip(ra, rects):
+            x.lo[:], x.hi[:], x.stride[:] = list(lo), list(hi), list(st)
+        keep += [na, ra]
+        d.n_nodes, d.nodes, d.root, d.out_mesh = len(nodes), na, int(root), int(out)
+        d.n_rects, d.rects = len(rects), ra
+    h = _vp()
+    _check(lib().sf_stencil_compile(C.byref(h), descs, len(stencils)))
+    return h
+
+
+def sf_stencil_source(h):
+    n = C.c_size_t()
+    _check(lib().sf_stencil_source(h, None, 0, C.byref(n)))
+    buf = C.create_string_buffer(n.value + 1)
+    _check(lib().sf_stencil_source(h, buf, n.value + 1, None))
+    return buf.value.decode()
+
+
+def sf_stencil_apply(h, level, src=None):
+    _check(lib().sf_stencil_apply(h, level, src))
+
+
+def sf_stencil_plan(h, gnx, gny, gnz, src_is_output=True):
+    n = _i()
+    _check(lib().sf_stencil_plan(h, int(gnx), int(gny), int(gnz), int(bool(src_is_output)),
+                                 C.byref(n)))
+    return n.value
+
+
+def sf_stencil_phases(h):
+    n = _i()
+    _check(lib().sf_stencil_phases(h, C.byref(n)))
+    return n.value
+
+
+def sf_stencil_destroy(h):
+    _check(lib().sf_stencil_destroy(h))
 
 
 def sf_comm_destroy(h):
