@@ -306,7 +306,7 @@ def main():
         }
         line.update({k: v for k, v in side.items() if k in (
             "e2e", "gsrb_c3", "vcycle", "fcycle", "read_bw", "cpu_baseline", "fig7_256",
-            "gsrb_size_sweep")})
+            "gsrb_size_sweep", "dsl_256")})
         print(json.dumps(line), flush=True)
     M.close()
     L.close()
@@ -458,6 +458,25 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
             Gs.close()
         sweep[str(n3)] = {"ms": ms, "gstencil_s": cells / (ms / 1e3) / 1e9, "alg_gbs": gbs}
         out["gsrb_size_sweep"] = sweep
+        # NEXT-4: the generic engine's JIT kernels for the same operators (the
+        # paper's DSL path): Fig 4's RB pair and A3, rendered + NVRTC-compiled
+        from paper_conf_ipps_zhangdmwbf17_b200 import stencil as SD
+        hh = 1.0 / n3
+        dpair = SD.hpgmg_gsrb_pair(1.0, 1.0, hh).compile()
+        dop = SD.hpgmg_apply_op(1.0, 1.0, hh).compile()
+        md = per_call(lambda: dpair(G), 20)
+        mo = per_call(lambda: dop(G), 20)
+        out["dsl_256"] = {
+            "gsrb_pair_ms": md, "gsrb_pair_launches": dpair.phases,
+            "gsrb_pair_alg_gbs": 2 * 64 * cells / (md / 1e3) / 1e9,
+            "gsrb_pair_frac_of_peak": 2 * 64 * cells / (md / 1e3) / 1e9 / pk,
+            "vs_handwritten_colour_sweeps": msc / md, "vs_fused_pair": ms / md,
+            "apply_op_ms": mo, "apply_op_alg_gbs": 48 * cells / (mo / 1e3) / 1e9,
+            "apply_op_frac_of_peak": 48 * cells / (mo / 1e3) / 1e9 / pk,
+            "note": "JIT (NVRTC sm_100a) kernels of the generic stencil engine; basis 64 B/cell "
+                    "per colour sweep (2 per pair) and 48 B/cell for A3"}
+        dpair.close()
+        dop.close()
         out["gsrb_c3"] = {"n": n3, "ms_per_rb_pair": ms,
                           "frac_of_kernel_compulsory": GSRB_KERNEL_BYTES_PER_CELL * cells / (ms / 1e3)
                           / 1e9 / pk,

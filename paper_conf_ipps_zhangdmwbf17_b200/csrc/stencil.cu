@@ -80,6 +80,7 @@ struct Drv {
     CUresult (*launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                        unsigned, CUstream, void**, void**);
     CUresult (*unload)(CUmodule);
+    CUresult (*occ)(int*, CUfunction, int, size_t);
 };
 Drv g_drv;
 
@@ -95,6 +96,7 @@ sf_status load_driver() {
     SF_DRV_SYM(get, "cuModuleGetFunction");
     SF_DRV_SYM(launch, "cuLaunchKernel");
     SF_DRV_SYM(unload, "cuModuleUnload");
+    SF_DRV_SYM(occ, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
 #undef SF_DRV_SYM
     g_drv.ok = true;
     return SF_OK;
@@ -257,12 +259,13 @@ bool depends(const St& s, const std::vector<RR>& Ds, const St& t, const std::vec
 // ------------------------------------------------------------------ codegen
 const char* kPrelude = R"(// rendered by libsf sf_stencil_compile (NEXT-4 generic stencil engine)
 #define SF_MAXR 64
-struct SfRect { int lo[3]; int st[3]; int cnt[3]; int sid; long long start; };
+struct SfRect { int lo[3]; int st[3]; int cnt[3]; int ax[3]; int sid; long long start; };
 struct SfArgs {
     double* f[2][9];
     long long js[2], ks[2];
     int xb, yb, zb[2];
     int nrect;
+    int ilv;            // > 0: the rects share one line lattice; line t -> rect t % ilv
     long long total;
     SfRect r[SF_MAXR];
 };
@@ -293,23 +296,14 @@ std::string index_expr(int src, const std::string& x, const std::string& y, cons
 std::string render(const std::vector<St>& group) {
     std::ostringstream o;
     o << kPrelude;
-    o << "extern \"C\" __global__ void __launch_bounds__(256) sf_stencil_group(const __grid_constant__ SfArgs a) {\n"
-         "    const long long nthr = (long long)gridDim.x * blockDim.x;\n"
-         "    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < a.total; t += nthr) {\n"
-         "        int lo = 0, hi = a.nrect - 1;   // rect of t: last start <= t\n"
-         "        while (lo < hi) { int m = (lo + hi + 1) >> 1; if (a.r[m].start <= t) lo = m; else hi = m - 1; }\n"
-         "        const SfRect& R = a.r[lo];\n"
-         "        const int l = (int)(t - R.start);\n"
-         "        const int i = l % R.cnt[0], q = l / R.cnt[0];\n"
-         "        const int j = q % R.cnt[1], k = q / R.cnt[1];\n"
-         "        const int X = R.lo[0] + R.st[0] * i, Y = R.lo[1] + R.st[1] * j, Z = R.lo[2] + R.st[2] * k;\n"
-         "        switch (R.sid) {\n";
+    // one evaluation function per stencil: the DAG in stored order
     for (size_t s = 0; s < group.size(); s++) {
         const St& st = group[s];
-        o << "        case " << s << ": {\n";
+        o << "__device__ __forceinline__ double sf_ev" << s
+          << "(const SfArgs& a, const int X, const int Y, const int Z) {\n";
         for (size_t i = 0; i < st.nodes.size(); i++) {
             const sf_sx_node& n = st.nodes[i];
-            o << "            const double v" << i << " = ";
+            o << "    const double v" << i << " = ";
             switch (n.op) {
                 case SF_SX_CONST: {
                     char buf[64];
@@ -318,8 +312,10 @@ std::string render(const std::vector<St>& group) {
                     break;
                 }
                 case SF_SX_READ:
-                    o << "a.f[" << n.src << "][" << n.mesh << "]["
-                      << index_expr(n.src, axis_expr(n, 0), axis_expr(n, 1), axis_expr(n, 2)) << "]";
+                    // read-only path: the phase analysis guarantees no point read
+                    // in a launch is written by another point of it
+                    o << "__ldg(&a.f[" << n.src << "][" << n.mesh << "]["
+                      << index_expr(n.src, axis_expr(n, 0), axis_expr(n, 1), axis_expr(n, 2)) << "])";
                     break;
                 case SF_SX_ADD: o << "v" << n.a << " + v" << n.b; break;
                 case SF_SX_SUB: o << "v" << n.a << " - v" << n.b; break;
@@ -329,17 +325,54 @@ std::string render(const std::vector<St>& group) {
             }
             o << ";\n";
         }
-        o << "            a.f[0][" << st.out << "][" << index_expr(0, "X", "Y", "Z") << "] = v" << st.root
-          << ";\n";
-        o << "        } break;\n";
+        o << "    return v" << st.root << ";\n}\n";
     }
-    o << "        }\n    }\n}\n";
+    // one block row per (rect, j, k) line of the domain: blockIdx.y walks the
+    // lines of all rects of the launch (start = first line of a rect), the x
+    // threads the points of the line -- one division per line, coalesced x;
+    // each thread evaluates two points before storing either (their loads overlap)
+    o << "extern \"C\" __global__ void __launch_bounds__(256) sf_stencil_group(const __grid_constant__ SfArgs a) {\n"
+         "    const int step = gridDim.x * blockDim.x;\n"
+         "    for (long long row = blockIdx.y; row < a.total; row += gridDim.y) {\n"
+         "        int lo, l;\n"
+         "        if (a.ilv) {   // interleaved: consecutive lines of all rects plane by plane\n"
+         "            lo = (int)(row % a.ilv);\n"
+         "            l = (int)(row / a.ilv);\n"
+         "        } else {       // rect by rect: last start <= row\n"
+         "            lo = 0;\n"
+         "            int hi = a.nrect - 1;\n"
+         "            while (lo < hi) { int m = (lo + hi + 1) >> 1; if (a.r[m].start <= row) lo = m; else hi = m - 1; }\n"
+         "            l = (int)(row - a.r[lo].start);\n"
+         "        }\n"
+         "        const SfRect& R = a.r[lo];\n"
+         "        const int n0 = R.cnt[R.ax[0]], n1 = R.cnt[R.ax[1]];\n"
+         "        const int j = l % n1, k = l / n1;\n"
+         "        for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n0; i += 2 * step) {\n"
+         "        const int i2 = i + step < n0 ? i + step : i;\n"
+         "        const int X = R.lo[0] + R.st[0] * (R.ax[0] == 0 ? i : R.ax[1] == 0 ? j : k);\n"
+         "        const int Y = R.lo[1] + R.st[1] * (R.ax[0] == 1 ? i : R.ax[1] == 1 ? j : k);\n"
+         "        const int Z = R.lo[2] + R.st[2] * (R.ax[0] == 2 ? i : R.ax[1] == 2 ? j : k);\n"
+         "        const int X2 = R.lo[0] + R.st[0] * (R.ax[0] == 0 ? i2 : R.ax[1] == 0 ? j : k);\n"
+         "        const int Y2 = R.lo[1] + R.st[1] * (R.ax[0] == 1 ? i2 : R.ax[1] == 1 ? j : k);\n"
+         "        const int Z2 = R.lo[2] + R.st[2] * (R.ax[0] == 2 ? i2 : R.ax[1] == 2 ? j : k);\n"
+         "        switch (R.sid) {\n";
+    for (size_t s = 0; s < group.size(); s++) {
+        const St& st = group[s];
+        o << "        case " << s << ": {\n"
+          << "            const double r1 = sf_ev" << s << "(a, X, Y, Z);\n"
+          << "            const double r2 = sf_ev" << s << "(a, X2, Y2, Z2);\n"
+          << "            a.f[0][" << st.out << "][" << index_expr(0, "X", "Y", "Z") << "] = r1;\n"
+          << "            if (i2 != i) a.f[0][" << st.out << "][" << index_expr(0, "X2", "Y2", "Z2")
+          << "] = r2;\n"
+          << "        } break;\n";
+    }
+    o << "        }\n        }\n    }\n}\n";
     return o.str();
 }
 
 // host mirror of the generated argument block
 struct SfRectH {
-    int lo[3], st[3], cnt[3], sid;
+    int lo[3], st[3], cnt[3], ax[3], sid;
     long long start;
 };
 struct SfArgsH {
@@ -347,6 +380,7 @@ struct SfArgsH {
     long long js[2], ks[2];
     int xb, yb, zb[2];
     int nrect;
+    int ilv;
     long long total;
     SfRectH r[SF_STENCIL_MAX_RECTS];
 };
@@ -359,6 +393,8 @@ struct sf_stencil {
     std::string src;
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
+    int sms = 0;
+    int occ[9] = {0};   // resident blocks per SM for 32 << b threads
     int phases = 0;
 };
 
@@ -476,6 +512,9 @@ static sf_status jit(sf_stencil* s) {
         return sf_fail(SF_ERR_CUDA, "cuModuleLoadData failed");
     if (g_drv.get(&s->fn, s->mod, "sf_stencil_group") != CUDA_SUCCESS)
         return sf_fail(SF_ERR_CUDA, "cuModuleGetFunction failed");
+    s->sms = p.multiProcessorCount;
+    for (int b = 0; b < 4; b++)   // 32, 64, 128, 256 threads
+        if (g_drv.occ(&s->occ[b], s->fn, 32 << b, 0) != CUDA_SUCCESS || s->occ[b] < 1) s->occ[b] = 1;
     return SF_OK;
 }
 
@@ -607,33 +646,67 @@ extern "C" sf_status sf_stencil_apply(sf_stencil* s, sf_level* L, sf_level* Src)
             A.yb = SF_GY - 1;
             A.zb[0] = SF_GZ - 1 - z0;
             A.zb[1] = same ? A.zb[0] : SF_GZ - 1;
-            long long total = 0;
-            int nr = 0;
+            long long total = 0;   // lines (j, k) of all rects of the phase
+            int nr = 0, maxc0 = 0;
             for (int i : ph)
                 for (const Rect& r : s->st[i].rects) {
                     RR R = resolve(r, gdim, zlo, zhi);
                     if (R.empty()) continue;
                     if (nr == SF_STENCIL_MAX_RECTS)
                         return sf_fail(SF_ERR_INVALID, "more than %d rects in one phase", SF_STENCIL_MAX_RECTS);
-                    if ((long long)R.cnt[0] * R.cnt[1] * R.cnt[2] > INT_MAX)
-                        return sf_fail(SF_ERR_SHAPE, "rect of more than 2^31 points");
+                    // line axis: x unless the rect is one point wide in x (e.g.
+                    // an x-face ghost layer), then the longer of y / z
+                    int a0 = 0;
+                    if (R.cnt[0] == 1) a0 = R.cnt[1] >= R.cnt[2] ? 1 : 2;
+                    const int a1 = a0 == 0 ? 1 : 0, a2 = 3 - a0 - a1;
+                    const long long lines = (long long)R.cnt[a1] * R.cnt[a2];
+                    if (lines > INT_MAX) return sf_fail(SF_ERR_SHAPE, "rect of more than 2^31 lines");
                     SfRectH& h = A.r[nr++];
                     for (int d = 0; d < 3; d++) {
                         h.lo[d] = (int)R.lo[d];
                         h.st[d] = (int)R.st[d];
                         h.cnt[d] = (int)R.cnt[d];
                     }
+                    h.ax[0] = a0; h.ax[1] = a1; h.ax[2] = a2;
                     h.sid = i;
                     h.start = total;
-                    total += (long long)R.cnt[0] * R.cnt[1] * R.cnt[2];
+                    total += lines;
+                    maxc0 = std::max(maxc0, (int)R.cnt[a0]);
                 }
             if (total == 0) continue;
             A.nrect = nr;
             A.total = total;
-            const long long blocks = (total + 255) / 256;
-            const unsigned grid = (unsigned)std::min<long long>(blocks, 148LL * 16);
+            // rects sharing one line lattice (e.g. the 4 rects of a colour) are
+            // walked interleaved, ordered by (outer, middle) start, so the
+            // lines in flight sit in a few neighbouring planes (L2 reuse of
+            // the neighbour planes / rows instead of 4 sweeps of the volume)
+            A.ilv = 0;
+            if (nr > 1) {
+                bool same = true;
+                for (int q = 1; q < nr && same; q++)
+                    for (int d = 0; d < 3; d++)
+                        if (A.r[q].st[d] != A.r[0].st[d] || A.r[q].cnt[d] != A.r[0].cnt[d] ||
+                            A.r[q].ax[d] != A.r[0].ax[d])
+                            same = false;
+                if (same) {
+                    const int a1 = A.r[0].ax[1], a2 = A.r[0].ax[2];
+                    std::sort(A.r, A.r + nr, [&](const SfRectH& x, const SfRectH& y) {
+                        if (x.lo[a2] != y.lo[a2]) return x.lo[a2] < y.lo[a2];
+                        return x.lo[a1] < y.lo[a1];
+                    });
+                    A.ilv = nr;
+                }
+            }
+            const int half = (maxc0 + 1) / 2;   // two points per thread
+            const int bx = half >= 256 ? 256 : half > 64 ? 128 : half > 32 ? 64 : 32;
+            const unsigned gx = (unsigned)std::min(4, (half + bx - 1) / bx);
+            // persistent: exactly the resident blocks (one wave) walk the lines
+            const int bi = bx == 32 ? 0 : bx == 64 ? 1 : bx <= 128 ? 2 : 3;
+            const int bxr = 32 << bi;
+            const unsigned gy = (unsigned)std::min<long long>(
+                total, std::max(1, s->sms * s->occ[bi] / (int)gx));
             void* params[] = {&A};
-            if (g_drv.launch(s->fn, grid, 1, 1, 256, 1, 1, 0, L->stream, params, nullptr) != CUDA_SUCCESS)
+            if (g_drv.launch(s->fn, gx, gy, 1, bxr, 1, 1, 0, L->stream, params, nullptr) != CUDA_SUCCESS)
                 return sf_fail(SF_ERR_CUDA, "cuLaunchKernel failed");
             SF_LAUNCHED();
         }

@@ -348,3 +348,22 @@ def helmholtz_ax(a, b, h, x="u"):
     return Component(x, SparseArray({(0, 0, 0): centre, (-1, 0, 0): c * bw, (1, 0, 0): c * be,
                                      (0, -1, 0): c * bs, (0, 1, 0): c * bn,
                                      (0, 0, -1): c * bb, (0, 0, 1): c * bt}))
+
+
+def gsrb_update(a, b, h, x="u", rhs="f"):
+    """x + lambda (rhs - A x) (Fig 4 l.6-10; lambda = Dinv, reading R-4)."""
+    return (Component(x, {(0, 0, 0): 1.0}) + Component("dinv", {(0, 0, 0): 1.0})
+            * (Component(rhs, {(0, 0, 0): 1.0}) - helmholtz_ax(a, b, h, x)))
+
+
+def hpgmg_gsrb_pair(a, b, h, x="u", rhs="f"):
+    """One RB pair as the paper writes it: [BC, red, BC, black]."""
+    red, black = red_black_domains()
+    return StencilGroup(dirichlet_faces(x) + [Stencil(gsrb_update(a, b, h, x, rhs), x, red)]
+                        + dirichlet_faces(x) + [Stencil(gsrb_update(a, b, h, x, rhs), x, black)])
+
+
+def hpgmg_apply_op(a, b, h, out="r", x="u"):
+    """[BC, out = A x] over the interior (A2 + A3)."""
+    return StencilGroup(dirichlet_faces(x) + [
+        Stencil(helmholtz_ax(a, b, h, x), out, RectDomain((1, 1, 1), (-1, -1, -1)))])

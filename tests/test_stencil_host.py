@@ -37,8 +37,8 @@ def test_render_and_source():
     assert 'extern "C" __global__' in src and "sf_stencil_group" in src
     assert src.count("case ") == 14          # 12 boundary stencils + red + black
     # the weight-array lowering reads each (mesh, offset) once per stencil
-    red_case = src.split("case 6:")[1].split("case 7:")[0]
-    assert red_case.count("a.f[0][0][") == 7 + 1   # u at 7 offsets + the store
+    red_ev = src.split("sf_ev6(")[1].split("sf_ev7(")[0]
+    assert red_ev.count("a.f[0][0][") == 7          # u at its 7 offsets, each once
     c.close()
 
 
