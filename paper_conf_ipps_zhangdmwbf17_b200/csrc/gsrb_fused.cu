@@ -119,6 +119,18 @@ __device__ __forceinline__ void tma3(void* dst, const CUtensorMap* m, int c0, in
         "l"((unsigned long long)m), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
         : "memory");
 }
+__device__ __forceinline__ void mbar_expect_u(unsigned b, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void tma3u(unsigned dst, const CUtensorMap* m, int c0, int c1, int c2,
+                                      unsigned bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(dst),
+        "l"((unsigned long long)m), "r"(c0), "r"(c1), "r"(c2), "r"(bar)
+        : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -325,18 +337,29 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         const int cyx = y0, cyc = y0 + 1;     // TMA y coordinates (x box, coef box)
         const unsigned seq0 = seq;            // pre-bundle; bundle q -> seq0 + 2 + q - z0
 
-        // bundle q: x(q+1), alpha/Dinv/rhs/beta_i/beta_j (q), beta_k(q+1); needed by R(q)
+        // bundle q: x(q+1), Dinv/rhs/beta_i/beta_j (q), beta_k(q+1); needed by R(q).
+        // Part k of the bundle (0: arrive.expect_tx + x, 1..4: coefficient
+        // arrays, 5: beta_k) -- in the steady state lane 0 of warp k issues part
+        // k, so no single warp carries the whole issue latency into the next
+        // step (arrivals and complete_tx may come in any order within a phase).
+        const unsigned xs_u = smem_u32(Xs), cs_u = smem_u32(Cs), ks_u = smem_u32(Ks);
+        const unsigned mb_u = smem_u32(mbar);
+        auto issue_part = [&](int q, int part) {
+            const unsigned sq = seq0 + 2 + (q - z0);
+            const unsigned b = mb_u + 8u * (sq % NMB);
+            if (part == 0) {
+                mbar_expect_u(b, BUNDLE_BYTES);
+                tma3u(xs_u + 8u * (md(q + 1, NXS) * XSLOT), &mp.x, cx, cyx, q + 1 + SF_GZ, b);
+            } else if (part == 5) {
+                tma3u(ks_u + 8u * (md(q + 1, NKS) * CARR), &mp.bk, cx, cyc, q + 1 + SF_GZ, b);
+            } else {
+                const unsigned c = cs_u + 8u * (md(q, NCS) * CSLOT + (part - 1) * CARR);
+                const CUtensorMap* m = part == 1 ? &mp.dv : part == 2 ? &mp.rh : part == 3 ? &mp.bi : &mp.bj;
+                tma3u(c, m, cx, cyc, q + SF_GZ, b);
+            }
+        };
         auto issue = [&](int q) {
-            unsigned sq = seq0 + 2 + (q - z0);
-            unsigned long long* b = &mbar[sq % NMB];
-            mbar_expect(b, BUNDLE_BYTES);
-            tma3(Xs + md(q + 1, NXS) * XSLOT, &mp.x, cx, cyx, q + 1 + SF_GZ, b);
-            double* c = Cs + md(q, NCS) * CSLOT;
-            tma3(c + CA_DV * CARR, &mp.dv, cx, cyc, q + SF_GZ, b);
-            tma3(c + CA_RH * CARR, &mp.rh, cx, cyc, q + SF_GZ, b);
-            tma3(c + CA_BI * CARR, &mp.bi, cx, cyc, q + SF_GZ, b);
-            tma3(c + CA_BJ * CARR, &mp.bj, cx, cyc, q + SF_GZ, b);
-            tma3(Ks + md(q + 1, NKS) * CARR, &mp.bk, cx, cyc, q + 1 + SF_GZ, b);
+            for (int k = 0; k < 6; k++) issue_part(q, k);
         };
         if (tid == 0) {
             fence_proxy_async();  // generic smem writes of the previous item before TMA reuse
