@@ -245,6 +245,19 @@ sf_status sf_vcycle(sf_mg* mg, int l);
 sf_status sf_fcycle(sf_mg* mg);
 sf_status sf_solve(sf_mg* mg, int fcycle, double rtol, int max_cycles, int* cycles, double* hist);
 sf_status sf_mg_destroy(sf_mg* mg);
+/* Pipelined multi-RHS solve (the serving path): for k = 0..n-1 solve
+ * A u_k = f_k exactly as sf_solve does (F-cycle first when fcycle, else from
+ * u = 0), reading f_k from host_f[k] and writing u_k to host_u[k] (packed
+ * interior host layout of the finest level's local parts, as
+ * sf_level_upload/download; pinned memory makes the copies asynchronous).
+ * The host->device copy of f_{k+1} and the device->host copy of u_{k-1} run
+ * on their own streams while solve k runs, through two packed device staging
+ * buffers allocated for the call (2 x one field).  cycles[k] (may be NULL)
+ * receives each solve's cycle count.  Synchronises; returns the first failing
+ * solve's status (later right-hand sides are not solved).  Leaves F = f_{last}
+ * and U = u_{last} on the level. */
+sf_status sf_solve_stream(sf_mg* mg, int fcycle, double rtol, int max_cycles, int n,
+                          const double* const* host_f, double* const* host_u, int* cycles);
 
 /* -------------------------------------------------------------- measurement
  * Number of kernels libsf launched since the counter was last reset (host-side

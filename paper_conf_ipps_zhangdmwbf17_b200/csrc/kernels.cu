@@ -11,6 +11,8 @@
 #include <cfloat>
 #include <cmath>
 
+#include <algorithm>
+
 #include "sf_internal.h"
 
 namespace {
@@ -489,6 +491,41 @@ sf_status k_norm(sf_level* L, int field, int kind, double* dst) {
         SF_LAUNCHED();
     }
     return sf_check_launch("norm");
+}
+
+// packed host-layout buffer (nzh, nyh, nxh) <-> strided field interior of one part
+__global__ void __launch_bounds__(256) pack_kernel(double* __restrict__ field, long js, long ks,
+                                                   double* __restrict__ buf, int nxh, int nyh,
+                                                   int nzh, int up) {
+    const long rows = (long)nyh * nzh;
+    for (long r = blockIdx.x; r < rows; r += gridDim.x) {
+        const int j = (int)(r % nyh), k = (int)(r / nyh);
+        double* f = field + (long)(k + SF_GZ) * ks + (long)(j + SF_GY) * js + SF_OX;
+        double* b = buf + r * nxh;
+        for (int i = threadIdx.x; i < nxh; i += blockDim.x) {
+            if (up)
+                f[i] = __ldcs(b + i);
+            else
+                __stcs(b + i, f[i]);
+        }
+    }
+}
+
+// SM copy between a field and a packed device buffer (the staging buffers of
+// sf_solve_stream): a strided 3-D cudaMemcpy D2D runs on a copy engine at a
+// fraction of HBM speed and would contend with the PCIe copies
+sf_status k_pack(sf_level* L, int field, double* buf, bool up) {
+    const int nxh = L->nx + (field == SF_BETA_I), nyh = L->ny + (field == SF_BETA_J);
+    const int nzh = L->lnz + (field == SF_BETA_K);
+    for (int q = 0; q < L->nlocal; q++) {
+        double* b = buf + (size_t)q * L->lnz * nyh * nxh;
+        const long rows = (long)nyh * nzh;
+        const int grid = (int)std::min<long>(rows, 148L * 16);
+        pack_kernel<<<grid, 256, 0, L->stream>>>(L->parts[q].f[field], L->js, L->ks, b, nxh, nyh,
+                                                 nzh, up ? 1 : 0);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("pack");
 }
 
 sf_status k_zero(sf_level* L, int field) {

@@ -134,7 +134,8 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
         }
     }
     L->dscratch = (double*)p;  // 256 bytes = 32 device scalars
-    cudaError_t e = cudaMallocHost(&L->hscratch, 256);
+    cudaError_t e = cudaHostAlloc(&L->hscratch, 256, cudaHostAllocMapped);
+    if (e == cudaSuccess) e = cudaHostGetDevicePointer(&L->hscratch_dev, L->hscratch, 0);
     if (e != cudaSuccess) {
         if (L->owns) cudaFree(L->buf);
         delete L;
@@ -184,7 +185,9 @@ static void host_extent(const sf_level* L, int field, int* nxh, int* nyh, int* n
     *nzh = L->lnz + (field == SF_BETA_K);
 }
 
-static sf_status copy3d(sf_level* L, int field, double* host, bool up) {
+// copy a field's interior between the level and a packed host-layout buffer
+// (host memory or device memory: cudaMemcpyDefault) on `stream`
+sf_status sf_copy_field(sf_level* L, int field, double* host, bool up, cudaStream_t stream) {
     int nxh, nyh, nzh;
     host_extent(L, field, &nxh, &nyh, &nzh);
     for (int q = 0; q < L->nlocal; q++) {
@@ -196,13 +199,18 @@ static sf_status copy3d(sf_level* L, int field, double* host, bool up) {
         cudaPitchedPtr hpp = make_cudaPitchedPtr(hp, nxh * sizeof(double), nxh * sizeof(double), nyh);
         m.extent = make_cudaExtent(nxh * sizeof(double), nyh, nzh);
         if (up) {
-            m.srcPtr = hpp; m.dstPtr = dp; m.kind = cudaMemcpyHostToDevice;
+            m.srcPtr = hpp; m.dstPtr = dp;
         } else {
-            m.srcPtr = dp; m.dstPtr = hpp; m.kind = cudaMemcpyDeviceToHost;
+            m.srcPtr = dp; m.dstPtr = hpp;
         }
-        SF_CUDA(cudaMemcpy3DAsync(&m, L->stream));
+        m.kind = cudaMemcpyDefault;
+        SF_CUDA(cudaMemcpy3DAsync(&m, stream));
     }
     return SF_OK;
+}
+
+static sf_status copy3d(sf_level* L, int field, double* host, bool up) {
+    return sf_copy_field(L, field, host, up, L->stream);
 }
 
 extern "C" sf_status sf_level_upload(sf_level* L, int field, const double* host) {
@@ -331,8 +339,7 @@ sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, 
     double* sumsq = L->dscratch + 1;
     for (int it = 0; it < iters; it++) SF_TRY(k_power_step(L, v, SF_R, a, b, sumsq));
     // last ratio ||D^-1 A v|| / ||v|| with ||v|| = 1 after normalisation
-    SF_CUDA(cudaMemcpyAsync(L->hscratch + 1, sumsq, sizeof(double), cudaMemcpyDeviceToHost,
-                            L->stream));
+    SF_TRY(sf_scalar_to_host(L, sumsq, 1));
     SF_CUDA(cudaStreamSynchronize(L->stream));
     *out = sqrt(L->hscratch[1]);
     return SF_OK;
@@ -434,13 +441,23 @@ sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst) {
     return SF_OK;
 }
 
+// A device scalar -> hscratch[slot] through mapped pinned memory, written by a
+// one-thread kernel: no copy-engine transfer, so the per-cycle convergence
+// scalar never queues behind bulk PCIe copies (sf_solve_stream).
+static __global__ void scalar_to_host_kernel(const double* src, double* dst) { *dst = *src; }
+
+sf_status sf_scalar_to_host(sf_level* L, const double* src, int slot) {
+    scalar_to_host_kernel<<<1, 1, 0, L->stream>>>(src, L->hscratch_dev + slot);
+    SF_LAUNCHED();
+    return sf_check_launch("scalar_to_host");
+}
+
 extern "C" sf_status sf_norm(sf_level* L, int field, int kind, double* out) {
     if (!L || !out) return sf_fail(SF_ERR_INVALID, "NULL argument");
     SF_TRY(check_field(field));
     if (kind != SF_NORM_MAX && kind != SF_NORM_L2) return sf_fail(SF_ERR_INVALID, "bad norm kind");
     SF_TRY(sf_norm_async(L, field, kind, L->dscratch));
-    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
-                            L->stream));
+    SF_TRY(sf_scalar_to_host(L, L->dscratch, 0));
     SF_CUDA(cudaStreamSynchronize(L->stream));
     double v = L->hscratch[0];
     *out = (kind == SF_NORM_L2) ? sqrt(v) : v;

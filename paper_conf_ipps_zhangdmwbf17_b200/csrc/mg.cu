@@ -264,11 +264,7 @@ static sf_status fcyc(sf_mg* m) {
     return SF_OK;
 }
 
-static sf_status to_host(sf_level* L) {
-    SF_CUDA(cudaMemcpyAsync(L->hscratch, L->dscratch, sizeof(double), cudaMemcpyDeviceToHost,
-                            L->stream));
-    return SF_OK;
-}
+static sf_status to_host(sf_level* L) { return sf_scalar_to_host(L, L->dscratch, 0); }
 
 // separate convergence check: max|F - A U| of the finest level (A6 + A10)
 static sf_status check(sf_mg* m) {
@@ -468,4 +464,65 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
         SF_TRY(run(m, G_REST));
         done++;
     }
+}
+
+// Pipelined multi-RHS solve (include/sf.h): copies of f_{k+1} (H2D) and
+// u_{k-1} (D2H) run on their own streams under solve k; two packed staging
+// buffers decouple them from the level's F and U.
+extern "C" sf_status sf_solve_stream(sf_mg* m, int fcycle, double rtol, int max_cycles, int n,
+                                     const double* const* host_f, double* const* host_u,
+                                     int* cycles) {
+    if (!m || n < 0 || (n > 0 && (!host_f || !host_u))) return sf_fail(SF_ERR_INVALID, "bad arguments");
+    if (n == 0) return SF_OK;
+    sf_level* L = m->lv[0];
+    const size_t bytes = (size_t)L->nlocal * L->lnz * L->ny * L->nx * sizeof(double);
+    double *stf = nullptr, *stu = nullptr;
+    cudaStream_t sin = nullptr, sout = nullptr;
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};   // f_ready, f_free, u_ready, u_free
+    sf_status st = SF_OK;
+    auto cu = [&](cudaError_t e, const char* what) {
+        if (e != cudaSuccess && st == SF_OK) st = sf_fail(SF_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+        return st == SF_OK;
+    };
+    if (cu(cudaMalloc(&stf, bytes), "staging f") && cu(cudaMalloc(&stu, bytes), "staging u") &&
+        cu(cudaStreamCreateWithFlags(&sin, cudaStreamNonBlocking), "stream") &&
+        cu(cudaStreamCreateWithFlags(&sout, cudaStreamNonBlocking), "stream")) {
+        for (int i = 0; i < 4 && st == SF_OK; i++)
+            cu(cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming), "event");
+    }
+    if (st == SF_OK && cu(cudaMemcpyAsync(stf, host_f[0], bytes, cudaMemcpyDefault, sin), "H2D f") &&
+        cu(cudaEventRecord(ev[0], sin), "record")) {
+        for (int k = 0; k < n && st == SF_OK; k++) {
+            if (!cu(cudaStreamWaitEvent(L->stream, ev[0], 0), "wait")) break;
+            if ((st = k_pack(L, SF_F, stf, true)) != SF_OK) break;
+            if (!cu(cudaEventRecord(ev[1], L->stream), "record")) break;
+            if (k + 1 < n && !(cu(cudaStreamWaitEvent(sin, ev[1], 0), "wait") &&
+                               cu(cudaMemcpyAsync(stf, host_f[k + 1], bytes, cudaMemcpyDefault, sin), "H2D f") &&
+                               cu(cudaEventRecord(ev[0], sin), "record")))
+                break;
+            if (!fcycle && (st = k_zero(L, SF_U)) != SF_OK) break;
+            int c = 0;
+            st = sf_solve(m, fcycle, rtol, max_cycles, &c, nullptr);
+            if (cycles) cycles[k] = c;
+            if (st != SF_OK) break;
+            if (!cu(cudaStreamWaitEvent(L->stream, ev[3], 0), "wait")) break;
+            if ((st = k_pack(L, SF_U, stu, false)) != SF_OK) break;
+            if (!(cu(cudaEventRecord(ev[2], L->stream), "record") &&
+                  cu(cudaStreamWaitEvent(sout, ev[2], 0), "wait") &&
+                  cu(cudaMemcpyAsync(host_u[k], stu, bytes, cudaMemcpyDefault, sout), "D2H u") &&
+                  cu(cudaEventRecord(ev[3], sout), "record")))
+                break;
+        }
+    }
+    sf_status keep = st;
+    if (sin) cudaStreamSynchronize(sin);
+    if (sout) cudaStreamSynchronize(sout);
+    cudaStreamSynchronize(L->stream);
+    for (cudaEvent_t e : ev)
+        if (e) cudaEventDestroy(e);
+    if (sin) cudaStreamDestroy(sin);
+    if (sout) cudaStreamDestroy(sout);
+    cudaFree(stf);
+    cudaFree(stu);
+    return keep;
 }

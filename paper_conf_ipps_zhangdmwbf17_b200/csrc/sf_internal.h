@@ -51,7 +51,8 @@ struct sf_level {
     void* buf;
     bool owns;
     double* dscratch;          // device scalars (norms)
-    double* hscratch;          // pinned host scalars
+    double* hscratch;          // pinned, mapped host scalars
+    double* hscratch_dev;      // their device alias
     std::vector<char*> peer;   // kind-2 comm: peer ranks' level buffers (CUDA IPC), by rank
     std::vector<void*> ipc_opened;
 };
@@ -74,6 +75,8 @@ PV sf_view(const sf_level* L, int p);
 void sf_swap_fields(sf_level* L, int f1, int f2);   // host-side id <-> buffer mapping
 
 sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst);
+sf_status sf_scalar_to_host(sf_level* L, const double* src, int slot);
+sf_status sf_copy_field(sf_level* L, int field, double* host, bool up, cudaStream_t stream);
 
 // ------------------------------------------------------------------ errors
 sf_status sf_fail(sf_status s, const char* fmt, ...);
@@ -103,6 +106,7 @@ sf_status k_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind);
 sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind);
 sf_status k_norm(sf_level* L, int field, int kind, double* dst_dev);
 sf_status k_zero(sf_level* L, int field);
+sf_status k_pack(sf_level* L, int field, double* buf, bool up);
 sf_status k_init_problem(sf_level* L, int problem, double a, double b, int want_rhs);
 sf_status k_bottom_setup(sf_level* L, double a, double b, double* ainv);
 sf_status k_bottom_solve(sf_level* L, int x, int rhs, const double* ainv);

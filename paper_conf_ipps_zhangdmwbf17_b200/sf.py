@@ -43,7 +43,7 @@ EXPORTS = [
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
     "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
-    "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy",
+    "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
 ]
 
 
@@ -138,6 +138,8 @@ def lib():
         "sf_fcycle": (_i, [_vp]),
         "sf_solve": (_i, [_vp, _i, _d, _i, C.POINTER(_i), _P]),
         "sf_mg_destroy": (_i, [_vp]),
+        "sf_solve_stream": (_i, [_vp, _i, _d, _i, _i, C.POINTER(_vp), C.POINTER(_vp),
+                                 C.POINTER(_i)]),
         "sf_launch_count": (_i, [C.POINTER(C.c_longlong), _i]),
         "sf_mg_plan": (_i, [_i, _i, _i, _i, _i, _i, C.POINTER(_i), C.POINTER(_i), C.POINTER(_i)]),
     }
@@ -378,6 +380,19 @@ def sf_solve(mg, fcycle=True, rtol=1e-10, max_cycles=50, raise_on_error=True):
     return st, cyc.value, list(hist[:cyc.value])
 
 
+def sf_solve_stream(mg, host_f_ptrs, host_u_ptrs, fcycle=True, rtol=1e-10, max_cycles=50):
+    """Pipelined multi-RHS solve; pointers are ints (pinned host or device
+    addresses).  Returns the cycle count of each solve."""
+    n = len(host_f_ptrs)
+    if len(host_u_ptrs) != n:
+        raise ValueError("one output per right-hand side")
+    fa = (_vp * max(n, 1))(*host_f_ptrs)
+    ua = (_vp * max(n, 1))(*host_u_ptrs)
+    cyc = (_i * max(n, 1))()
+    _check(lib().sf_solve_stream(mg, int(fcycle), float(rtol), int(max_cycles), n, fa, ua, cyc))
+    return list(cyc[:n])
+
+
 def sf_mg_destroy(mg):
     _check(lib().sf_mg_destroy(mg))
 
@@ -543,6 +558,19 @@ class MG:
 
     def solve(self, fcycle=True, rtol=1e-10, max_cycles=50, raise_on_error=True):
         return sf_solve(self.handle, fcycle, rtol, max_cycles, raise_on_error)
+
+    def solve_stream(self, fs, us, fcycle=True, rtol=1e-10, max_cycles=50):
+        """Solve for each host rhs in `fs` (arrays of the level's host shape,
+        pinned torch tensors for overlap) into the matching `us`; the copies of
+        neighbouring right-hand sides overlap each solve (sf_solve_stream)."""
+        def ptr(a):
+            if hasattr(a, "data_ptr"):
+                return a.data_ptr()
+            if not a.flags.c_contiguous or a.dtype != np.float64:
+                raise ValueError("C-contiguous float64 arrays expected")
+            return a.ctypes.data
+        return sf_solve_stream(self.handle, [ptr(f) for f in fs], [ptr(u) for u in us], fcycle,
+                               rtol, max_cycles)
 
     def vcycle(self, l=0):
         sf_vcycle(self.handle, l)
