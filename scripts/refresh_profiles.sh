@@ -1,0 +1,24 @@
+#!/bin/bash
+# One gpurun call that refreshes every round-1 evidence file under gpurun_out/
+# (copied into profiles/r01/ by hand afterwards).
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.json 2> gpurun_out/bench.err
+echo "bench exit $?"
+SF_PROFILE_TIMED=1 timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none --csv \
+   --log-file gpurun_out/bench_launches.csv python bench.py --steps 1 --warmup 3 --quick > gpurun_out/bench_launches_run.log 2>&1
+echo "timed-region launch list exit $?"
+timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
+   --log-file gpurun_out/solve_launches.csv python scripts/solve_profile.py 512 0 > gpurun_out/solve_launches.log 2>&1
+echo "solve launch list exit $?"
+for n in 512 256; do
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:gsrb_pair -s 2 -c 1 \
+     -o gpurun_out/prof_gsrb_v10_$n -f python scripts/prof_gsrb.py $n 3 fused > gpurun_out/ncu_v10_$n.log 2>&1
+  echo "ncu pair $n exit $?"
+done
+bash scripts/prof_variants.sh v10 > /dev/null 2>&1; echo "variants exit $?"
+timeout 600 ncu --set full --clock-control none -k regex:sf_stencil_group -c 6 -o gpurun_out/prof_dsl_256 -f \
+   python scripts/dsl_once.py 256 > gpurun_out/ncu_dsl.log 2>&1; echo "dsl exit $?"
+python scripts/dsl_time.py 256 > gpurun_out/dsl_time.txt 2>&1
+python scripts/e2e_probe.py 512 > gpurun_out/e2e_probe.txt 2>&1
+ls gpurun_out
