@@ -43,10 +43,12 @@ def parse():
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="sf", choices=["sf", "reference"])
-    p.add_argument("--n", type=int, default=512, help="cells per side per GPU (weak scaling)")
+    p.add_argument("--side", type=int, default=512, help="cells per side per GPU (weak scaling)")
     p.add_argument("--gsrb-n", type=int, default=256)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--quick", action="store_true", help="skip the side measurements")
+    p.add_argument("--comm", default="p2p", choices=["p2p", "nccl"],
+                   help="N>1 transport: device-initiated peer-memory exchanges (p2p) or NCCL")
     return p.parse_args()
 
 
@@ -157,7 +159,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    nx, ny, nz = dims_for(args.n, 1)
+    nx, ny, nz = dims_for(args.side, 1)
     shp, scale = oracle_shape((nx, ny, nz))
     steps = []
     for s in range(args.warmup + args.steps):
@@ -205,10 +207,19 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # SF_BENCH_SHARED_GPU=1 (tests only): every rank on cuda:0, gloo process group
+    shared = os.environ.get("SF_BENCH_SHARED_GPU") == "1"
+    local = 0 if shared else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    host_group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared:
+            dist.init_process_group("gloo")
+            host_group = dist.group.WORLD
+        else:
+            dist.init_process_group("nccl", device_id=dev)
+            host_group = dist.new_group(backend="gloo")   # IPC-handle exchange (p2p)
     sf.lib()
 
     def barrier():
@@ -219,10 +230,12 @@ def main():
     from paper_conf_ipps_zhangdmwbf17_b200.parallel import max_over_ranks as _mor
 
     def max_over_ranks(x):
-        return _mor(x, device=dev)
+        return _mor(x, device=None if shared else dev)
 
-    nx, ny, nz = dims_for(args.n, world)
-    comm = sf.Comm.nccl() if world > 1 else None
+    nx, ny, nz = dims_for(args.side, world)
+    comm = None
+    if world > 1:
+        comm = sf.Comm.p2p(host_group) if args.comm == "p2p" else sf.Comm.nccl()
     h = 1.0 / max(nx, ny, nz)
     L = sf.Level(nx, ny, nz, h, comm=comm)
     sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)       # HPGMG problem + manufactured f
@@ -297,6 +310,7 @@ def main():
             "data": "synthetic (HPGMG-shaped VC Helmholtz, manufactured rhs, on-device init)",
             "config": {"workload": f"C5 HPGMG-FV VC Helmholtz {nx}x{ny}x{nz // world} per GPU",
                        "global": [nx, ny, nz], "parallelism": f"z-slab x{world}",
+                       "transport": (args.comm if world > 1 else "none"),
                        "cycles_per_solve": cyc, "final_relres": hist[-1] if hist else None,
                        "max_err_vs_manufactured": err,
                        "smoother": "colour-fused GSRB, 2+2 pairs", "l2": "inputs >> L2, no flush"},

@@ -135,6 +135,16 @@ sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[128], int nr
 typedef int (*sf_host_allgather_fn)(const void* send, size_t nbytes, void* recv, void* user);
 sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank, sf_host_allgather_fn allgather,
                                  void* user);
+/* Device-initiated transport: one part per process
+ * (one GPU each, or several processes sharing a GPU in tests); every level's
+ * buffer is opened by every peer through CUDA IPC (peer access over NVLink
+ * when the processes own different GPUs) and halos, agglomeration and scalar
+ * all-reduces are kernels that read the peers' memory directly and
+ * synchronise through flags in device memory (no NCCL, no host round trip;
+ * CUDA-graph capturable).  The host all-gather is used only at level
+ * creation to exchange the IPC handles; same contract as hostipc. */
+sf_status sf_comm_create_p2p(sf_comm** out, int nranks, int rank, sf_host_allgather_fn allgather,
+                             void* user);
 sf_status sf_comm_destroy(sf_comm* comm);
 /* number of parts in the job, parts local to this process, first local part */
 sf_status sf_comm_info(const sf_comm* comm, int* nparts, int* nlocal, int* first);

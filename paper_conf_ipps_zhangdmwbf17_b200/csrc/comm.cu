@@ -13,6 +13,8 @@
 
 #include <mutex>
 
+#include <algorithm>
+
 #include "sf_internal.h"
 
 namespace {
@@ -109,12 +111,14 @@ extern "C" sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[1
     return SF_OK;
 }
 
-extern "C" sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank,
-                                            sf_host_allgather_fn fn, void* user) {
+static sf_status create_ipc_comm(sf_comm** out, int nranks, int rank, sf_host_allgather_fn fn,
+                                 void* user, int kind) {
     if (!out || !fn || nranks < 1 || rank < 0 || rank >= nranks)
         return sf_fail(SF_ERR_INVALID, "bad arguments");
+    if (kind == 3 && nranks > SF_P2P_MAX_RANKS)
+        return sf_fail(SF_ERR_INVALID, "p2p comm supports <= %d ranks", SF_P2P_MAX_RANKS);
     sf_comm* c = new sf_comm();
-    c->kind = 2;
+    c->kind = kind;
     c->nparts = nranks; c->nlocal = 1; c->first = rank;
     c->rank = rank; c->nranks = nranks;
     c->nccl = nullptr;
@@ -122,6 +126,16 @@ extern "C" sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank,
     c->hostuser = user;
     *out = c;
     return SF_OK;
+}
+
+extern "C" sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank,
+                                            sf_host_allgather_fn fn, void* user) {
+    return create_ipc_comm(out, nranks, rank, fn, user, 2);
+}
+
+extern "C" sf_status sf_comm_create_p2p(sf_comm** out, int nranks, int rank, sf_host_allgather_fn fn,
+                                        void* user) {
+    return create_ipc_comm(out, nranks, rank, fn, user, 3);
 }
 
 namespace {
@@ -140,8 +154,132 @@ double* peer_field(const sf_level* L, int rank, const double* mine) {
 }
 }  // namespace
 
+// ------------------------------------------------------------ kind 3: P2P
+// Device-initiated exchanges over peer memory.  Every exchange is one op of a
+// per-level sequence that all ranks run in the same order (SPMD); op s:
+//   1. "ready = s" (release, system scope): my data for op s is final (all
+//      earlier kernels of the stream are done);
+//   2. wait until every peer involved shows ready >= s (acquire), read its
+//      data straight from its memory (NVLink loads), write mine;
+//   3. "consumed = s", then wait until those peers show consumed >= s: nobody
+//      overwrites data a peer is still reading, and a peer can be at most one
+//      op ahead.
+// The sequence number lives in device memory (read at kernel start, advanced
+// by the last CTA), so the kernels replay correctly from CUDA graphs.
+__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void wait_ge(const unsigned long long* p, unsigned long long v) {
+    while (ld_acquire_sys(p) < v) __nanosleep(64);
+}
+
+struct P2PPeers {
+    const unsigned long long* sync[SF_P2P_MAX_RANKS];   // peers' sync blocks (nullptr: not involved)
+};
+
+// op start: every CTA learns s; CTA 0 publishes ready; thread 0 of each CTA
+// waits for the peers' ready
+__device__ __forceinline__ unsigned long long p2p_begin(unsigned long long* my, const P2PPeers& pe,
+                                                        int npeers) {
+    __shared__ unsigned long long s_seq;
+    if (threadIdx.x == 0) {
+        const unsigned long long s = *(volatile unsigned long long*)&my[2] + 1;
+        if (blockIdx.x == 0) st_release_sys(&my[0], s);
+        for (int q = 0; q < npeers; q++)
+            if (pe.sync[q]) wait_ge(&pe.sync[q][0], s);
+        s_seq = s;
+    }
+    __syncthreads();
+    return s_seq;
+}
+
+// op end: the last CTA publishes consumed, waits for the peers', advances s
+__device__ __forceinline__ void p2p_end(unsigned long long* my, const P2PPeers& pe, int npeers,
+                                        unsigned long long s) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned prev = atomicAdd((unsigned*)&my[3], 1u);
+        if (prev == gridDim.x - 1) {
+            __threadfence();
+            my[3] = 0;
+            st_release_sys(&my[1], s);
+            for (int q = 0; q < npeers; q++)
+                if (pe.sync[q]) wait_ge(&pe.sync[q][1], s);
+            *(volatile unsigned long long*)&my[2] = s;
+        }
+    }
+}
+
+// halo: my ghosts <- the neighbours' boundary planes (peers 0 = lower, 1 = upper)
+__global__ void __launch_bounds__(256) p2p_halo_kernel(double* x, const double* lo_x, const double* hi_x,
+                                                       unsigned long long* my, P2PPeers pe, long lo_dst,
+                                                       long hi_src, long hi_dst, long lo_src, long cnt) {
+    const unsigned long long s = p2p_begin(my, pe, 2);
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) {
+        if (lo_x) x[lo_dst + i] = lo_x[hi_src + i];
+        if (hi_x) x[hi_dst + i] = hi_x[lo_src + i];
+    }
+    p2p_end(my, pe, 2, s);
+}
+
+struct P2PPtrs {
+    const double* p[SF_P2P_MAX_RANKS];
+};
+
+// all-reduce of one scalar: my slot <- v; every rank reduces all ranks' slots
+// in rank order (the same result on every rank)
+__global__ void p2p_allreduce_kernel(double* v, unsigned long long* my, P2PPeers pe, P2PPtrs slot,
+                                     int nranks, int op) {
+    // my slot is rewritten only after every peer consumed the previous op
+    if (threadIdx.x == 0) *(double*)(my + 8) = *v;
+    const unsigned long long s = p2p_begin(my, pe, nranks);
+    if (threadIdx.x == 0) {
+        double r = 0.0;
+        for (int q = 0; q < nranks; q++) {
+            const double y = *(const volatile double*)slot.p[q];
+            if (q == 0) r = y;
+            else if (op == 0) r = (y > r || y != y) ? y : r;
+            else r = r + y;
+        }
+        *v = r;
+    }
+    p2p_end(my, pe, nranks, s);
+}
+
+// agglomeration: copy every other rank's planes of a replicated level
+__global__ void __launch_bounds__(256) p2p_gather_kernel(double* base, P2PPtrs peer_base,
+                                                         unsigned long long* my, P2PPeers pe, int nranks,
+                                                         int rank, long cnt, double* top,
+                                                         const double* peer_top, long topcnt) {
+    const unsigned long long s = p2p_begin(my, pe, nranks);
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (int q = 0; q < nranks; q++) {
+        if (q == rank) continue;
+        const double* src = peer_base.p[q] + q * cnt;
+        double* dst = base + q * cnt;
+        for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) dst[i] = src[i];
+    }
+    if (peer_top)
+        for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < topcnt; i += stride) top[i] = peer_top[i];
+    p2p_end(my, pe, nranks, s);
+}
+
+static unsigned long long* peer_sync(const sf_level* L, int r) {
+    return (unsigned long long*)(L->peer[r] + ((const char*)L->dsync - (const char*)L->buf));
+}
+
 sf_status sf_ipc_register(sf_level* L, const sf_comm* c) {
-    if (!c || c->kind != 2) return SF_OK;
+    if (!c || (c->kind != 2 && c->kind != 3)) return SF_OK;
+    if (c->kind == 3) {   // fresh sync block (the buffer may be recycled memory)
+        SF_CUDA(cudaMemsetAsync(L->dsync, 0, SF_SCRATCH_BYTES - 256, L->stream));
+    }
     SF_CUDA(cudaStreamSynchronize(L->stream));
     // base of the allocation holding the level buffer (a torch block may sit inside one)
     static decltype(&cuMemGetAddressRange) range = nullptr;
@@ -169,7 +307,7 @@ sf_status sf_ipc_register(sf_level* L, const sf_comm* c) {
     for (int r = 0; r < c->nranks; r++) {
         if (r == c->rank) continue;
         void* p = nullptr;
-        SF_CUDA(cudaIpcOpenMemHandle(&p, all[r].h, cudaIpcMemLazyEnablePeerAccess));
+        SF_CUDA(cudaIpcOpenMemHandle(&p, all[r].h, cudaIpcMemLazyEnablePeerAccess));   // NVLink P2P
         L->ipc_opened.push_back(p);
         L->peer[r] = (char*)p + all[r].off;
     }
@@ -216,6 +354,21 @@ sf_status sf_halo(sf_level* L, int field, int depth) {
         }
         return SF_OK;
     }
+    if (L->comm->kind == 3) {  // device-initiated: neighbours' planes over peer memory
+        const sf_comm* c = L->comm;
+        const int r = c->rank, n = c->nranks;
+        double* x = L->parts[0].f[field];
+        P2PPeers pe = {};
+        const double* lo_x = nullptr;
+        const double* hi_x = nullptr;
+        if (r > 0) { pe.sync[0] = peer_sync(L, r - 1); lo_x = peer_field(L, r - 1, x); }
+        if (r < n - 1) { pe.sync[1] = peer_sync(L, r + 1); hi_x = peer_field(L, r + 1, x); }
+        const int grid = (int)std::min<long>(148, ((long)cnt + 255) / 256);
+        p2p_halo_kernel<<<grid, 256, 0, L->stream>>>(x, lo_x, hi_x, L->dsync, pe, lo_dst, hi_src, hi_dst,
+                                                     lo_src, (long)cnt);
+        SF_LAUNCHED();
+        return sf_check_launch("p2p_halo");
+    }
     if (L->comm->kind == 2) {  // pull the neighbours' boundary planes through IPC
         const sf_comm* c = L->comm;
         int r = c->rank, n = c->nranks;
@@ -252,6 +405,25 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
     const sf_comm* cm = C->rep_comm;
     if (!cm || cm->kind == 0) return SF_OK;
     if (cm->nranks != parts) return sf_fail(SF_ERR_SHAPE, "agglomeration across %d parts", parts);
+    if (cm->kind == 3) {  // device-initiated gather over peer memory
+        double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
+        const long cnt = (long)lnz_per_part * C->ks;
+        P2PPeers pe = {};
+        P2PPtrs pb = {};
+        for (int q = 0; q < parts; q++)
+            if (q != cm->rank) {
+                pe.sync[q] = peer_sync(C, q);
+                pb.p[q] = peer_field(C, q, base);
+            }
+        double* top = base + (size_t)C->gnz * C->ks;
+        const double* ptop = (field == SF_BETA_K && cm->rank != parts - 1) ? peer_field(C, parts - 1, top)
+                                                                           : nullptr;
+        const int grid = (int)std::min<long>(148, (cnt + 255) / 256);
+        p2p_gather_kernel<<<grid, 256, 0, C->stream>>>(base, pb, C->dsync, pe, parts, cm->rank, cnt, top,
+                                                       ptop, C->ks);
+        SF_LAUNCHED();
+        return sf_check_launch("p2p_gather");
+    }
     if (cm->kind == 2) {  // every rank copies the other ranks' planes from their buffers
         double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
         size_t cnt = (size_t)lnz_per_part * C->ks;
@@ -281,8 +453,20 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
     return SF_OK;
 }
 
-sf_status sf_allreduce_scalar(const sf_comm* cm, double* dev, int op, cudaStream_t s) {
+sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int op) {
     if (!cm || cm->kind == 0 || cm->nranks == 1) return SF_OK;
+    cudaStream_t s = L->stream;
+    if (cm->kind == 3) {
+        P2PPeers pe = {};
+        P2PPtrs sl = {};
+        for (int q = 0; q < cm->nranks; q++) {
+            if (q != cm->rank) pe.sync[q] = peer_sync(L, q);
+            sl.p[q] = (const double*)((q == cm->rank ? L->dsync : peer_sync(L, q)) + 8);
+        }
+        p2p_allreduce_kernel<<<1, 32, 0, s>>>(dev, L->dsync, pe, sl, cm->nranks, op);
+        SF_LAUNCHED();
+        return sf_check_launch("p2p_allreduce");
+    }
     if (cm->kind == 2) {
         double v;
         SF_CUDA(cudaMemcpyAsync(&v, dev, sizeof(double), cudaMemcpyDeviceToHost, s));

@@ -455,7 +455,7 @@ sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, doub
         SF_LAUNCHED();
     }
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
-        SF_TRY(sf_allreduce_scalar(L->comm, sumsq, 1, L->stream));
+        SF_TRY(sf_allreduce_scalar(L, L->comm, sumsq, 1));
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         int depth;

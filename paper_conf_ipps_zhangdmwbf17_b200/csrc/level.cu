@@ -81,7 +81,7 @@ extern "C" sf_status sf_level_bytes_needed(int gnx, int gny, int gnz, const sf_c
     long js, ks;
     size_t fe;
     layout(gnx, gny, gnz / np, &js, &ks, &fe);
-    *bytes = (size_t)nl * SF_NFIELDS * field_bytes_aligned(fe) + 256;
+    *bytes = (size_t)nl * SF_NFIELDS * field_bytes_aligned(fe) + SF_SCRATCH_BYTES;
     return SF_OK;
 }
 
@@ -133,7 +133,8 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
             p += fb;
         }
     }
-    L->dscratch = (double*)p;  // 256 bytes = 32 device scalars
+    L->dscratch = (double*)p;  // 32 device scalars, then the P2P sync words
+    L->dsync = (unsigned long long*)(L->dscratch + 32);
     cudaError_t e = cudaHostAlloc(&L->hscratch, 256, cudaHostAllocMapped);
     if (e == cudaSuccess) e = cudaHostGetDevicePointer(&L->hscratch_dev, L->hscratch, 0);
     if (e != cudaSuccess) {
@@ -143,7 +144,7 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
     }
     e = cudaMemsetAsync(L->buf, 0, need, L->stream);
     if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
-    if (comm && comm->kind == 2) {
+    if (comm && (comm->kind == 2 || comm->kind == 3)) {
         sf_status s = sf_ipc_register(L, comm);
         if (s != SF_OK) {
             sf_level_destroy(L);
@@ -437,7 +438,7 @@ extern "C" sf_status sf_interpolate(sf_level* F, int ff, double prescale, sf_lev
 sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst) {
     SF_TRY(k_norm(L, field, kind, dst));
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
-        SF_TRY(sf_allreduce_scalar(L->comm, dst, kind == SF_NORM_MAX ? 0 : 1, L->stream));
+        SF_TRY(sf_allreduce_scalar(L, L->comm, dst, kind == SF_NORM_MAX ? 0 : 1));
     return SF_OK;
 }
 

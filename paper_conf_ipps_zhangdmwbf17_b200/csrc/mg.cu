@@ -146,7 +146,7 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
         }
         if (!P.distributed) {
             C->rep_comm = F->comm ? F->comm : F->rep_comm;
-            s = sf_ipc_register(C, C->rep_comm);   // kind-2 comm: collective
+            s = sf_ipc_register(C, C->rep_comm);   // kind-2/3 comm: collective
             if (s != SF_OK) {
                 m->lv.push_back(C);
                 m->own.push_back(true);
@@ -272,7 +272,7 @@ static sf_status check(sf_mg* m) {
     if (pair_ok(L)) {  // max|f - Au| reduced in the residual pass, nothing stored
         SF_TRY(k_residual_pair(L, -1, SF_U, SF_F, m->a, m->b, L->dscratch));
         if (L->comm && L->comm->kind != 0 && L->nparts > 1)
-            SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
+            SF_TRY(sf_allreduce_scalar(L, L->comm, L->dscratch, 0));
     } else {
         SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
         SF_TRY(sf_norm_async(L, SF_R, SF_NORM_MAX, L->dscratch));
@@ -297,7 +297,7 @@ static sf_status first_pair_check(sf_mg* m) {
     SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
     sf_swap_fields(L, SF_U, SF_TMP);
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
-        SF_TRY(sf_allreduce_scalar(L->comm, L->dscratch, 0, L->stream));
+        SF_TRY(sf_allreduce_scalar(L, L->comm, L->dscratch, 0));
     return to_host(L);
 }
 
@@ -305,6 +305,8 @@ static bool graphs_allowed(const sf_mg* m) {
     if (!m->o.use_graph || m->graph_failed) return false;
     if (m->lv[0]->stream == nullptr) return false;  // legacy stream cannot be captured
     if (m->lv[0]->comm && m->lv[0]->comm->kind == 2) return false;  // host-synchronised halos
+    for (const sf_level* l : m->lv)   // agglomeration through the host (kind 2) likewise
+        if (l->rep_comm && l->rep_comm->kind == 2) return false;
     // the fused smoother swaps U/TMP per pair; only an even count per captured
     // sequence leaves the host-side mapping unchanged for replays
     if (m->o.smoother == SF_SMOOTH_CHEBY)   // an n-step application ends with swap(U, [U,R,TMP][n%3]):

@@ -19,9 +19,15 @@
 #define SF_OX 4
 #define SF_GY 2
 #define SF_GZ 2
+// per-level device scratch after the fields: 32 doubles + the P2P sync block
+// (comm kind 3): u64 [0] ready, [1] consumed, [2] op sequence, [3] CTA count,
+// [8, 8 + SF_P2P_MAX_RANKS) all-reduce slots (doubles)
+#define SF_P2P_MAX_RANKS 64
+#define SF_SCRATCH_BYTES (256 + 8 * (8 + SF_P2P_MAX_RANKS))
 
 struct sf_comm {
-    int kind;          // 0 = local (all parts in this process), 1 = NCCL, 2 = host+IPC (tests)
+    int kind;          // 0 = local (all parts in this process), 1 = NCCL, 2 = host+IPC (tests),
+                       // 3 = device-initiated P2P (peer memory over NVLink, CUDA IPC)
     int nparts;        // parts in the whole job
     int nlocal;        // parts held by this process
     int first;         // global index of the first local part
@@ -51,6 +57,7 @@ struct sf_level {
     void* buf;
     bool owns;
     double* dscratch;          // device scalars (norms)
+    unsigned long long* dsync; // P2P sync block (inside buf: peers reach it through IPC)
     double* hscratch;          // pinned, mapped host scalars
     double* hscratch_dev;      // their device alias
     std::vector<char*> peer;   // kind-2 comm: peer ranks' level buffers (CUDA IPC), by rank
@@ -152,4 +159,4 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part);
 sf_status sf_ipc_register(sf_level* L, const sf_comm* c);
 void sf_ipc_close(sf_level* L);
 // Reduce a device scalar over ranks (op 0 = max, 1 = sum); in place.
-sf_status sf_allreduce_scalar(const sf_comm* comm, double* dev, int op, cudaStream_t s);
+sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* comm, double* dev, int op);

@@ -44,6 +44,7 @@ EXPORTS = [
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
     "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
+    "sf_comm_create_p2p",
 ]
 
 
@@ -103,6 +104,7 @@ def lib():
         "sf_get_unique_id": (_i, [C.c_char_p]),
         "sf_comm_create_nccl": (_i, [C.POINTER(_vp), C.c_char_p, _i, _i]),
         "sf_comm_create_hostipc": (_i, [C.POINTER(_vp), _i, _i, HOST_ALLGATHER, _vp]),
+        "sf_comm_create_p2p": (_i, [C.POINTER(_vp), _i, _i, HOST_ALLGATHER, _vp]),
         "sf_comm_destroy": (_i, [_vp]),
         "sf_stencil_compile": (_i, [C.POINTER(_vp), C.POINTER(StencilDesc), _i]),
         "sf_stencil_source": (_i, [_vp, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
@@ -244,6 +246,13 @@ def sf_stencil_phases(h):
 
 def sf_stencil_destroy(h):
     _check(lib().sf_stencil_destroy(h))
+
+
+def sf_comm_create_p2p(nranks, rank, allgather_cb):
+    """allgather_cb must be a HOST_ALLGATHER the caller keeps alive."""
+    h = _vp()
+    _check(lib().sf_comm_create_p2p(C.byref(h), int(nranks), int(rank), allgather_cb, None))
+    return h
 
 
 def sf_comm_destroy(h):
@@ -438,10 +447,22 @@ class Comm:
         return cls(sf_comm_create_nccl(uid, world, rank), world, 1, rank)
 
     @classmethod
+    def p2p(cls, group=None):
+        """Device-initiated transport: one part per rank, halos / agglomeration /
+        all-reduces by kernels reading the peers' memory (CUDA IPC, NVLink P2P
+        across GPUs); ``group`` (e.g. gloo) only exchanges the IPC handles when
+        levels are created (include/sf.h, sf_comm_create_p2p)."""
+        return cls._ipc(group, sf_comm_create_p2p)
+
+    @classmethod
     def hostipc(cls, group=None):
         """Test transport: one part per rank of a (gloo) torch.distributed group,
         all ranks on the SAME GPU; peer buffers through CUDA IPC, host
         synchronisation through ``group`` (include/sf.h, sf_comm_create_hostipc)."""
+        return cls._ipc(group, sf_comm_create_hostipc)
+
+    @classmethod
+    def _ipc(cls, group, create):
         import torch
         import torch.distributed as dist
         rank, world = dist.get_rank(group), dist.get_world_size(group)
@@ -459,7 +480,7 @@ class Comm:
                 return 1
 
         cb = HOST_ALLGATHER(allgather)
-        c = cls(sf_comm_create_hostipc(world, rank, cb), world, 1, rank)
+        c = cls(create(world, rank, cb), world, 1, rank)
         c._cb = cb          # keep the trampoline alive as long as the comm
         return c
 

@@ -5,8 +5,10 @@ device, so the NCCL transport cannot run here.  These tests run the same
 per-rank code (one part per process: slab offsets, depth-1/2 halos before
 every operator/pair, all-reduced norms and lambda_max, agglomeration of the
 coarse planes onto every rank, replicated coarse levels) with the hostipc
-transport: world_size processes on cuda:0, peer buffers opened through CUDA
-IPC, host synchronisation over gloo.  The result must equal the in-process
+transport (world_size processes on cuda:0, peer buffers opened through CUDA
+IPC, host synchronisation over gloo) and with the p2p transport (the same
+peer buffers, but halos / agglomeration / all-reduces are kernels that read
+the peers' memory and synchronise through device flags, CUDA graphs on).  The result must equal the in-process
 loopback decomposition (itself pinned to the undecomposed run and to the
 oracle in test_gpu_parity.py)."""
 import socket
@@ -73,7 +75,7 @@ def _run(sf, comm, world, rank, out_key, out):
     out[out_key] = res
 
 
-def _worker(rank, world, port, out):
+def _worker(rank, world, port, out, transport):
     import torch
     import torch.distributed as dist
 
@@ -82,7 +84,7 @@ def _worker(rank, world, port, out):
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
                             world_size=world)
     try:
-        comm = sf.Comm.hostipc()
+        comm = sf.Comm.hostipc() if transport == "hostipc" else sf.Comm.p2p()
         _run(sf, comm, world, rank, rank, out)
         dist.barrier()
         comm.close()
@@ -101,11 +103,12 @@ def sf():
     return S
 
 
+@pytest.mark.parametrize("transport", ["hostipc", "p2p"])
 @pytest.mark.parametrize("world", [2, 4])
-def test_hostipc_matches_loopback(sf, world):
+def test_per_rank_matches_loopback(sf, world, transport):
     with mp.Manager() as m:
         out = m.dict()
-        mp.spawn(_worker, args=(world, _free_port(), out), nprocs=world, join=True)
+        mp.spawn(_worker, args=(world, _free_port(), out, transport), nprocs=world, join=True)
         ranks = {r: out[r] for r in range(world)}
     ref = {}
     comm = sf.Comm.local(world)
