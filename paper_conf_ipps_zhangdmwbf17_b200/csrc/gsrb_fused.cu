@@ -467,12 +467,6 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 const unsigned sq = seq0 + 2 + (q - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
             }
-            if (INTERP && q + 1 <= z1) {   // bundle t+2 (x(t+3)) one step early, corrected now
-                const unsigned sq = seq0 + 2 + (q + 1 - z0);
-                mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
-                correct(t + 3, ce0, ce1);
-                if (t + 4 <= z1 + 1) load_e(t + 4, ce0, ce1);
-            }
             const int gkr = g.z0 + q;                    // plane of R
             const bool rin = q <= z1 && gkr >= 0 && gkr < g.gnz;
             const bool bin = t - 1 >= z0;                // B(t-1) on the tile
@@ -531,6 +525,14 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                                   SF_OX + gxa), o);
 #pragma unroll
             for (int i = 0; i < 8; i++) stash[i] = nb[i];
+            // INTERP: correct x(t+3) (bundle t+2) at the END of the step: no one
+            // reads that plane before step t+1, and the TMA had the whole step
+            if (INTERP && q + 1 <= z1) {
+                const unsigned sq = seq0 + 2 + (q + 1 - z0);
+                mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
+                correct(t + 3, ce0, ce1);
+                if (t + 4 <= z1 + 1) load_e(t + 4, ce0, ce1);
+            }
             fence_proxy_async();
             __syncthreads();
             // refill bundle t+PF+1 (its slots were last read before this barrier)
