@@ -270,9 +270,10 @@ __device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int gx,
 
 // B for the pair; SEL = position (0: even x, 1: odd x) of the black cell in
 // the pair.  Returns the output pair (red-new, black-new in place).
-template <int SEL>
+template <int SEL, bool TOPREG = false>
 __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx, int gy,
-                                              const Geo& g, int gkm, double bh2, const double* rb) {
+                                              const Geo& g, int gkm, double bh2, const double* rb,
+                                              double top = 0.0) {
     const double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
     double xw, xe;
     if (SEL == 0) {
@@ -287,7 +288,9 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
     const double xs = (gy == 0) ? 0.0 : s.Xm[col - W];
     const double xn = (gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
     const double xb = (gkm == 0) ? 0.0 : s.Xmm[col];
-    const double xt = (gkm == g.gnz - 1) ? 0.0 : s.Xk[col];
+    // TOPREG: the red cell above is this thread's own red-new of the previous
+    // step, not yet stored (RESID defers its red writes by one step)
+    const double xt = (gkm == g.gnz - 1) ? 0.0 : (TOPREG ? top : s.Xk[col]);
     const double bnew =
         rb[6] * (rb[7] + bh2 * sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
     return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
@@ -460,6 +463,13 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             __syncthreads();
         }
 
+        // RESID: red-new values (tile + ring) of the plane computed at step t are
+        // stored at the end of step t+1, after the barrier that ends step t:
+        // the black residuals of step t read that plane's red-OLD values, so an
+        // immediate store would need a second barrier per step
+        double prn = 0.0, prr = 0.0;
+        int pxo = 0, pro = 0;
+        bool pw = false, pwr = false;
         auto step = [&](int t, double* stash) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
@@ -494,13 +504,13 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             if (sel == 0) {
                 if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
                                                  rres, rold_new, xpair);
-                if (bin) o = black_pair<1>(sb, xoff, gxa, gy, g, gkm, bh2, stash);
+                if (bin) o = black_pair<1, RESID>(sb, xoff, gxa, gy, g, gkm, bh2, stash, prn);
                 if (RESID && rin)
                     bres = black_resid<1>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
             } else {
                 if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
                                                  rres, rold_new, xpair);
-                if (bin) o = black_pair<0>(sb, xoff, gxa, gy, g, gkm, bh2, stash);
+                if (bin) o = black_pair<0, RESID>(sb, xoff, gxa, gy, g, gkm, bh2, stash, prn);
                 if (RESID && rin)
                     bres = black_resid<0>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
             }
@@ -516,10 +526,17 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const int ro = par ? rxo[1] : rxo[0];
             double rr = 0.0;
             if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], bh2, zlo, zhi);
-            if (RESID) __syncthreads();   // black residuals read red-OLD cells of plane q
-            double* Xw = Xs + ix_p1 * XSLOT;
-            if (rin) Xw[xoff + sel] = rn;
-            if (ring) Xw[ro] = rr;
+            if (RESID) {
+                double* Xp = Xs + ix_0 * XSLOT;   // plane t: computed at step t-1
+                if (pw) Xp[pxo] = prn;
+                if (pwr) Xp[pro] = prr;
+                prn = rn; pxo = xoff + sel; pw = rin;
+                prr = rr; pro = ro; pwr = ring;
+            } else {
+                double* Xw = Xs + ix_p1 * XSLOT;
+                if (rin) Xw[xoff + sel] = rn;
+                if (ring) Xw[ro] = rr;
+            }
             if (bin)   // streaming store: do not evict halo lines other tiles still need
                 __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
