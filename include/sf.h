@@ -193,6 +193,19 @@ sf_status sf_apply_op(sf_level* level, int out, int x, double a, double b);
 sf_status sf_smooth_gsrb(sf_level* level, int x, int rhs, double a, double b, int rb_pairs, int kind);
 /* A6: res = rhs - A x */
 sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double b);
+/* A5 + A6 + A7, the tail of V(l)'s pre-smoothing: one RB
+ * pair on fine.x (exactly sf_smooth_gsrb with rb_pairs = 1), then
+ * coarse.c_field = R_cell(rhs - A x) of the smoothed x.  By default a pair, a
+ * residual into SF_R and a restriction produce it.  With the environment
+ * variable SF_RR=1, on single-part levels with nx % 32 == 0, ny % 16 == 0 and
+ * x = SF_U or SF_TMP, one kernel does all three in a single HBM pass and the
+ * residual is never stored (the U/TMP ids are swapped as by the fused
+ * smoother); it is measured slower on B200, hence opt-in.
+ * x must differ from rhs, SF_R and SF_DINV.  coarse dims must be fine dims / 2
+ * (SF_ERR_SHAPE); c_field must not be SF_DINV.  Enqueued on the fine level's
+ * stream; the coarse level must be idle on its own stream. */
+sf_status sf_smooth_residual_restrict(sf_level* fine, int x, int rhs, double a, double b,
+                                      sf_level* coarse, int c_field);
 /* A7: coarse.c_field = R(fine.f_field); coarse dims must be fine dims / 2
  * (PAPER.md:293-297, 466-468).  kind: enum sf_restrict_kind. */
 sf_status sf_restrict(sf_level* coarse, int c_field, sf_level* fine, int f_field, int kind);

@@ -25,6 +25,7 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
             ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=5", "-DSF_GSRB_SUFFIX=_t32"]),
            ("gsrb_fused.cu", "gsrb_fused_t64.o",
             ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t64"]),
+           ("gsrb_rr.cu", "gsrb_rr.o", []),
            ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []),
            ("stencil.cu", "stencil.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -44,7 +45,8 @@ def _compile(spec, force):
     src, obj, extra = spec
     s = os.path.join(CSRC, src)
     o = os.path.join(BUILD, obj)
-    deps = [s, os.path.join(CSRC, "sf_internal.h"), os.path.join(INCLUDE, "sf.h")]
+    deps = [s, os.path.join(CSRC, "sf_internal.h"), os.path.join(CSRC, "tma_common.cuh"),
+            os.path.join(INCLUDE, "sf.h")]
     if not force and not _needs(o, deps):
         return o, ""
     cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", s, "-o", o]

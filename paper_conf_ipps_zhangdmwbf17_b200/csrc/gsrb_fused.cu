@@ -92,82 +92,7 @@ struct CoarseView {
     int zoff;   // coarse plane of fine plane 0 inside a replicated coarse part
 };
 
-__device__ __forceinline__ unsigned smem_u32(const void* p) {
-    return (unsigned)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(unsigned long long* b, unsigned n) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(n));
-}
-__device__ __forceinline__ void mbar_expect(unsigned long long* b, unsigned bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)),
-                 "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* b, unsigned parity) {
-    asm volatile(
-        "{\n .reg .pred p;\n"
-        "W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-        " @!p bra W;\n}" ::"r"(smem_u32(b)),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void tma3(void* dst, const CUtensorMap* m, int c0, int c1, int c2,
-                                     unsigned long long* bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(smem_u32(dst)),
-        "l"((unsigned long long)m), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
-        : "memory");
-}
-__device__ __forceinline__ void mbar_expect_u(unsigned b, unsigned bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void tma3u(unsigned dst, const CUtensorMap* m, int c0, int c1, int c2,
-                                      unsigned bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(dst),
-        "l"((unsigned long long)m), "r"(c0), "r"(c1), "r"(c2), "r"(bar)
-        : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-
-__device__ __forceinline__ int md(int k, int m) { return ((k % m) + m) % m; }
-
-// Gauss-Seidel update in lambda-form.  With lambda = Dinv the EXACT inverse
-// diagonal of A including the Dirichlet fold (reading R-4),
-//     x + lambda (rhs - A x)  ==  lambda (rhs + b h^-2 S),
-//     S = sum over the cell's interior faces of beta_f * x(nbr_f),
-// because A x = D x(c) - b h^-2 S (a boundary face's ghost term -2 beta x(c)
-// is part of D).  The smoother therefore never reads alpha: 56 instead of the
-// 64 compulsory bytes of PAPER.md:669-672.  Boundary neighbours enter S as 0.
-// S is summed as a tree (depth 3): the per-plane step is latency-bound.
-// 1/d for the check-fused residual: hardware reciprocal estimate + two Newton
-// steps (relative error ~1e-16, far below what the 1e-10 convergence test needs;
-// avoids the long IEEE division sequence in the hot loop)
-__device__ __forceinline__ double inv_fast(double d) {
-    double y;
-    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
-    y = y * (2.0 - d * y);
-    y = y * (2.0 - d * y);
-    return y;
-}
-
-__device__ __forceinline__ double sum6(double xw, double xe, double xs, double xn, double xb,
-                                      double xt, double bw, double be, double bs, double bn,
-                                      double bb, double bt) {
-    const double sx = be * xe + bw * xw;
-    const double sy = bn * xn + bs * xs;
-    const double sz = bt * xt + bb * xb;
-    return (sx + sy) + sz;
-}
-
-__device__ __forceinline__ unsigned long long abits(double v) {
-    return (unsigned long long)__double_as_longlong(fabs(v));
-}
+#include "tma_common.cuh"
 
 struct Geo {
     int nx, ny, nz, z0, gnz;
@@ -223,15 +148,15 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     double r, S;
     if (SEL == 0) {
         S = sum6(xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x);
-        const double q = rh2.x + bh2 * S;
-        r = dv2.x * q;
+        const double q = gs_q(rh2.x, bh2, S);
+        r = __dmul_rn(dv2.x, q);
         if (RESID) rres = q - xp2.x * inv_fast(dv2.x);
         nb[0] = bi2.y; nb[1] = bie; nb[2] = bjl.y; nb[3] = bjh.y; nb[4] = bkl.y; nb[5] = bkh.y;
         nb[6] = dv2.y; nb[7] = rh2.y;
     } else {
         S = sum6(xw, xe, xs, xn, xb, xt, bi2.y, bie, bjl.y, bjh.y, bkl.y, bkh.y);
-        const double q = rh2.y + bh2 * S;
-        r = dv2.y * q;
+        const double q = gs_q(rh2.y, bh2, S);
+        r = __dmul_rn(dv2.y, q);
         if (RESID) rres = q - xp2.y * inv_fast(dv2.y);
         nb[0] = bi2.x; nb[1] = bi2.y; nb[2] = bjl.x; nb[3] = bjh.x; nb[4] = bkl.x; nb[5] = bkh.x;
         nb[6] = dv2.x; nb[7] = rh2.x;
@@ -292,7 +217,7 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
     // step, not yet stored (RESID defers its red writes by one step)
     const double xt = (gkm == g.gnz - 1) ? 0.0 : (TOPREG ? top : s.Xk[col]);
     const double bnew =
-        rb[6] * (rb[7] + bh2 * sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
+        gs_upd(rb[6], rb[7], bh2, sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
     return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
 }
 
@@ -308,7 +233,7 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
     const double S = sum6(xw, xe, xs, xn, xb, xt, s.C[CA_BI * CARR + co_],
                           s.C[CA_BI * CARR + co_ + 1], s.C[CA_BJ * CARR + co_],
                           s.C[CA_BJ * CARR + co_ + W], s.Klo[co_], s.Khi[co_]);
-    return s.C[CA_DV * CARR + co_] * (s.C[CA_RH * CARR + co_] + bh2 * S);
+    return gs_upd(s.C[CA_DV * CARR + co_], s.C[CA_RH * CARR + co_], bh2, S);
 }
 
 template <bool RESID, bool INTERP>

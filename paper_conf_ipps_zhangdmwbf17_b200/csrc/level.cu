@@ -363,6 +363,31 @@ extern "C" sf_status sf_residual(sf_level* L, int res, int x, int rhs, double a,
     return k_residual(L, res, x, rhs, a, b);
 }
 
+static bool coarse_of(const sf_level* C, const sf_level* F);
+
+extern "C" sf_status sf_smooth_residual_restrict(sf_level* F, int x, int rhs, double a, double b,
+                                                 sf_level* C, int cf) {
+    if (!F || !C) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(rhs));
+    SF_TRY(check_field(cf));
+    if (x == rhs || x == SF_DINV || rhs == SF_DINV || x == SF_R || rhs == SF_R || cf == SF_DINV)
+        return sf_fail(SF_ERR_INVALID, "x, rhs, R and DINV must be distinct fields");
+    if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
+    if ((x == SF_U || x == SF_TMP) && rhs != SF_U && rhs != SF_TMP && gsrb_fused_supported(F) &&
+        gsrb_rr_supported(F, C)) {
+        const int other = (x == SF_U) ? SF_TMP : SF_U;
+        SF_TRY(sf_halo(F, rhs, 1));
+        SF_TRY(sf_halo(F, x, 2));
+        SF_TRY(k_gsrb_pair_rr(F, x, other, rhs, a, b, C, cf));
+        sf_swap_fields(F, x, other);
+        return SF_OK;
+    }
+    SF_TRY(sf_smooth_gsrb(F, x, rhs, a, b, 1, SF_SMOOTH_AUTO));
+    SF_TRY(k_residual(F, SF_R, x, rhs, a, b));
+    return k_restrict(C, cf, F, SF_R, SF_RESTRICT_CELL);
+}
+
 bool gsrb_fused_supported(const sf_level* L) {
     return gsrb_fused_supported_t32(L) || gsrb_fused_supported_t64(L);
 }

@@ -226,12 +226,22 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     sf_level* L = m->lv[l];
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     sf_level* C = m->lv[l + 1];
-    SF_TRY(smooth(m, L, m->o.pre_pairs - (skip_first ? 1 : 0)));
-    if (pair_ok(L)) {  // residual never stored: A6 + A7 in one pass
-        SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F));
+    const int pre = m->o.pre_pairs - (skip_first ? 1 : 0);
+    if (pre >= 1 && (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
+        gsrb_fused_supported(L) && gsrb_rr_supported(L, C)) {
+        // the last pre-smoothing pair also forms the residual and restricts it
+        // (A5 + A6 + A7 in one pass; gsrb_rr.cu)
+        SF_TRY(smooth(m, L, pre - 1));
+        SF_TRY(k_gsrb_pair_rr(L, SF_U, SF_TMP, SF_F, m->a, m->b, C, SF_F));
+        sf_swap_fields(L, SF_U, SF_TMP);
     } else {
-        SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
-        SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
+        SF_TRY(smooth(m, L, pre));
+        if (pair_ok(L)) {  // residual never stored: A6 + A7 in one pass
+            SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F));
+        } else {
+            SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
+            SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
+        }
     }
     SF_TRY(k_zero(C, SF_U));
     SF_TRY(vcyc(m, l + 1));

@@ -148,6 +148,11 @@ bool gsrb_fused_supported(const sf_level* L);
 // C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
                             double* rmax = nullptr, sf_level* C = nullptr, int cf = 0);
+// last pre-smoothing pair fused with residual + restriction (gsrb_rr.cu):
+// xout = pair(xin); C.cf = R_cell(rhs - A xout).  Single-part levels, 32x16 tiles.
+bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
+sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
+                         int cf);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.

@@ -44,7 +44,7 @@ EXPORTS = [
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
     "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
-    "sf_comm_create_p2p",
+    "sf_comm_create_p2p", "sf_smooth_residual_restrict",
 ]
 
 
@@ -125,6 +125,7 @@ def lib():
         "sf_apply_op": (_i, [_vp, _i, _i, _d, _d]),
         "sf_smooth_gsrb": (_i, [_vp, _i, _i, _d, _d, _i, _i]),
         "sf_residual": (_i, [_vp, _i, _i, _i, _d, _d]),
+        "sf_smooth_residual_restrict": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
         "sf_apply_laplacian": (_i, [_vp, _i, _i]),
         "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
         "sf_smooth_chebyshev": (_i, [_vp, _i, _i, _d, _d, _i, _d, _d]),
@@ -309,6 +310,10 @@ def sf_apply_op(level, out, x, a, b):
 
 def sf_smooth_gsrb(level, x, rhs, a, b, rb_pairs, kind=SF_SMOOTH_AUTO):
     _check(lib().sf_smooth_gsrb(level, x, rhs, float(a), float(b), int(rb_pairs), int(kind)))
+
+
+def sf_smooth_residual_restrict(fine, x, rhs, a, b, coarse, c_field):
+    _check(lib().sf_smooth_residual_restrict(fine, x, rhs, float(a), float(b), coarse, c_field))
 
 
 def sf_apply_laplacian(level, out, x):

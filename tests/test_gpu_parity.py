@@ -223,6 +223,85 @@ def mg_pair(sf, oracle, n, shape=None, parts=1, cc=False, **opts):
     return L, M, O
 
 
+RR_SHAPES = [(4, 16, 32), (10, 32, 64), (16, 48, 96), (34, 16, 32), (64, 64, 64), (6, 32, 160)]
+
+
+@pytest.mark.parametrize("shape", RR_SHAPES)
+@pytest.mark.parametrize("depth", [None, "2", "6"])
+@pytest.mark.parametrize("ab", [(1.0, 1.0), (2.5, 0.75)])
+def test_smooth_residual_restrict(sf, oracle, shape, depth, ab, monkeypatch):
+    """A5+A6+A7 fused (sf_smooth_residual_restrict): the smoothed x equals the
+    oracle's RB pair (1e-12) and bit-for-bit the plain fused pair; the coarse
+    rhs equals R_cell(rhs - A x) of the oracle (1e-12).  Chunk depths 2 and 6
+    put item boundaries (extended z ranges, recomputed planes) inside the grid."""
+    nz, ny, nx = shape
+    a, b = ab
+    monkeypatch.setenv("SF_RR", "1")
+    if depth:
+        monkeypatch.setenv("SF_RR_DEPTH", depth)
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.hpgmg_coeffs(nx, ny, nz) if nx >= 64 else I.random_coeffs(nx, ny, nz, 5)
+    L = make_level(sf, shape, coeffs)
+    L2 = make_level(sf, shape, coeffs)
+    C = make_level(sf, (nz // 2, ny // 2, nx // 2), I.random_coeffs(nx // 2, ny // 2, nz // 2, 6))
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), a, b, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    for lv in (L, L2):
+        sf.sf_rebuild_operator(lv.handle, a, b)
+        lv.upload(sf.SF_U, x)
+        lv.upload(sf.SF_F, f)
+    sf.sf_smooth_residual_restrict(L.handle, sf.SF_U, sf.SF_F, a, b, C.handle, sf.SF_F)
+    sf.sf_smooth_gsrb(L2.handle, sf.SF_U, sf.SF_F, a, b, 1, sf.SF_SMOOTH_FUSED)
+    got = L.download(sf.SF_U)
+    assert np.array_equal(got, L2.download(sf.SF_U))
+    xs = P.smooth(x, f, 1, dinv=P.dinv())
+    assert rel(got, xs) < TOL
+    exp = oracle.restrict_cell(P.residual(xs, f))
+    assert rel(C.download(sf.SF_F), exp) < TOL
+
+
+def test_smooth_residual_restrict_general(sf, oracle):
+    """Shapes the fused kernel does not take (nx % 32 != 0, 2 parts) go through
+    pair + residual + restriction with the same result."""
+    for shape, parts in [((8, 8, 16), 1), ((16, 16, 32), 2)]:
+        nz, ny, nx = shape
+        h = I.level_h(nx, ny, nz)
+        coeffs = I.random_coeffs(nx, ny, nz, 7)
+        L = make_level(sf, shape, coeffs, parts=parts)
+        C = make_level(sf, (nz // 2, ny // 2, nx // 2), I.random_coeffs(nx // 2, ny // 2, nz // 2, 6),
+                       parts=parts)
+        P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.0, 1.0, *coeffs)
+        x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+        sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+        L.upload(sf.SF_U, x)
+        L.upload(sf.SF_F, f)
+        sf.sf_smooth_residual_restrict(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, sf.SF_F)
+        xs = P.smooth(x, f, 1, dinv=P.dinv())
+        assert rel(L.download(sf.SF_U), xs) < TOL
+        assert rel(C.download(sf.SF_F), oracle.restrict_cell(P.residual(xs, f))) < TOL
+    with pytest.raises(sf.SfError):
+        sf.sf_smooth_residual_restrict(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, L.handle, sf.SF_F)
+
+
+@pytest.mark.parametrize("n", [32, 64])
+def test_vcycle_rr_matches_separate_residual(sf, monkeypatch, n):
+    """The V-cycle with the fused last pre-smoothing pair (gsrb_rr) and with the
+    separate residual_restrict pass agree to rounding (1e-13)."""
+    out = []
+    for on in ("1", "0"):
+        monkeypatch.setenv("SF_RR", on)
+        h = 1.0 / n
+        coeffs = I.hpgmg_coeffs(n, n, n)
+        L = make_level(sf, (n, n, n), coeffs, h=h)
+        M = sf.MG(L, 1.0, 1.0)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        for _ in range(3):
+            M.vcycle(0)
+        out.append(L.download(sf.SF_U))
+    assert rel(out[0], out[1]) < 1e-13
+
+
 @pytest.mark.parametrize("n", [4, 16, 32, 64])
 def test_vcycle_parity(sf, oracle, n):
     L, M, O = mg_pair(sf, oracle, n)
