@@ -58,7 +58,15 @@ namespace {
 #define SF_CAT(a, b) SF_CAT2(a, b)
 constexpr int TX = SF_GSRB_TX;         // tile width (cells)
 constexpr int PPR = TX / 2;            // pairs per row = lanes per row segment
-constexpr int NWARP = 8;
+#ifndef SF_GSRB_NWARP
+#define SF_GSRB_NWARP 8
+#endif
+#ifndef SF_GSRB_MINB   // resident CTAs per SM the variant is built for
+#define SF_GSRB_MINB 1
+#endif
+constexpr int NWARP = SF_GSRB_NWARP;
+constexpr int MINB = SF_GSRB_MINB;
+static_assert(NWARP % 2 == 0, "rows w and w + NWARP must have the same parity");
 constexpr int TY = NWARP * 32 / PPR;   // tile height (rows): 16 for TX = 32
 constexpr int NT = 32 * NWARP;         // 256 threads
 constexpr int W = TX + 4;              // smem row: gx in [x0-2, x0+TX+2)
@@ -73,6 +81,7 @@ constexpr int CSLOT = NCA * CARR;
 constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8;
 constexpr int BUNDLE_BYTES = XBYTES + (NCA + 1) * CBYTES;
 constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR) + 64;
+static_assert(MINB * (SMEM + 1024) <= 228 * 1024, "MINB CTAs per SM must fit in shared memory");
 // fused P0 interpolation (INTERP): each x-box pair (2 cells, one parent) is
 // corrected in smem; a thread owns pairs tid and tid+NT of the box
 constexpr int XPAIRS = XH * (W / 2);
@@ -237,7 +246,7 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
 }
 
 template <bool RESID, bool INTERP>
-__global__ void __launch_bounds__(NT, 1)
+__global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
                      CoarseView cv) {
@@ -529,9 +538,17 @@ sf_status encode(CUtensorMap* m, const sf_level* L, const double* base, int rows
     cuuint64_t strides[2] = {(cuuint64_t)L->js * 8, (cuuint64_t)L->ks * 8};
     cuuint32_t box[3] = {(cuuint32_t)W, (cuuint32_t)rows, 1};
     cuuint32_t es[3] = {1, 1, 1};
+    // L2 fill granularity of the box loads (SF_TMA_PROMO = 0/64/128/256 for A/B runs)
+    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    if (const char* e = getenv("SF_TMA_PROMO")) {
+        const int v = atoi(e);
+        promo = v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+                : v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                : v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }
     CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, (void*)base, dims, strides, box, es,
-                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, promo,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return sf_fail(SF_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
     return SF_OK;
 }
@@ -561,6 +578,14 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
         SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, true>,
                                      cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
+        if (MINB > 1) {   // room for MINB CTAs per SM
+            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, false>,
+                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<true, false>,
+                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, true>,
+                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+        }
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
         SF_CUDA(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
@@ -568,7 +593,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     }
     const int ntx = L->nx / TX, nty = L->ny / TY, tiles = ntx * nty;
     // chunk depth: minimise rounds * (depth + prologue) over persistent CTAs
-    const int G = g_num_sms;
+    const int G = g_num_sms * MINB;   // resident CTAs
     int best_d = L->lnz;
     double best = 1e30;
     for (int nch = 1; nch <= L->lnz; nch++) {

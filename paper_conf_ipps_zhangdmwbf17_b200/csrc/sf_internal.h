@@ -143,6 +143,10 @@ sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double 
                                 double* rmax, sf_level* C, int cf);
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf);
+// 32x8 tiles, 4 warps, 2 CTAs per SM (two independent z-step chains per SM)
+bool gsrb_fused_supported_t32w4(const sf_level* L);
+sf_status k_gsrb_pair_fused_t32w4(sf_level* L, int xin, int xout, int rhs, double a, double b,
+                                  double* rmax, sf_level* C, int cf);
 bool gsrb_fused_supported(const sf_level* L);
 // rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax;
 // C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)

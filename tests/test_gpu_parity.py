@@ -223,6 +223,51 @@ def mg_pair(sf, oracle, n, shape=None, parts=1, cc=False, **opts):
     return L, M, O
 
 
+@pytest.mark.parametrize("depth", ["1", "2", "3", "5", "8"])
+def test_fused_pair_chunk_depths(sf, oracle, depth, monkeypatch):
+    """Small z-chunks: many items per CTA, so every item's prologue is issued in
+    the previous item's last steps (pipelined item transition); the result
+    matches the oracle per pair and is bit-identical to the default chunking."""
+    shape = (24, 32, 64)
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.random_coeffs(nx, ny, nz, 8)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.0, 1.0, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    outs = []
+    for dep in (None, depth):
+        if dep:
+            monkeypatch.setenv("SF_GSRB_DEPTH", dep)
+        L = make_level(sf, shape, coeffs)
+        sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+        L.upload(sf.SF_U, x)
+        L.upload(sf.SF_F, f)
+        for _ in range(3):
+            sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED)
+        outs.append(L.download(sf.SF_U))
+    assert np.array_equal(outs[0], outs[1])
+    assert rel(outs[1], P.smooth(x, f, 3, dinv=P.dinv())) < TOL
+
+
+@pytest.mark.parametrize("depth", ["2", "3"])
+def test_vcycle_chunk_depth_invariant(sf, depth, monkeypatch):
+    """The V-cycle's fused variants (check-fused, P0-fused, plain) give the same
+    bits whatever the z-chunking (items pipelined into each other)."""
+    n = 64
+    out = []
+    for dep in (None, depth):
+        if dep:
+            monkeypatch.setenv("SF_GSRB_DEPTH", dep)
+        L = make_level(sf, (n, n, n), I.hpgmg_coeffs(n, n, n), h=1.0 / n)
+        M = sf.MG(L, 1.0, 1.0)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        st, cyc, hist = M.solve(fcycle=True, rtol=1e-10)
+        out.append((cyc, list(hist), L.download(sf.SF_U)))
+    assert out[0][0] == out[1][0] and out[0][1] == out[1][1]
+    assert np.array_equal(out[0][2], out[1][2])
+
+
 RR_SHAPES = [(4, 16, 32), (10, 32, 64), (16, 48, 96), (34, 16, 32), (64, 64, 64), (6, 32, 160)]
 
 
