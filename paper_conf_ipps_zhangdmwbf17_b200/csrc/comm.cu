@@ -15,6 +15,8 @@
 
 #include <algorithm>
 
+#include <cstdlib>
+
 #include "sf_internal.h"
 
 namespace {
@@ -335,8 +337,13 @@ extern "C" sf_status sf_comm_info(const sf_comm* c, int* nparts, int* nlocal, in
     return SF_OK;
 }
 
-sf_status sf_halo(sf_level* L, int field, int depth) {
+sf_status sf_halo(sf_level* L, int field, int depth) { return sf_halo_on(L, field, depth, L->stream); }
+
+sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t stream) {
     if (L->nparts <= 1 || !L->comm) return SF_OK;
+    // beside a running sweep (stream != the level's) the device-initiated copy
+    // keeps to a few CTAs: the sweep leaves only a couple of SMs free
+    const int max_ctas = stream == L->stream ? 148 : 16;
     if (depth > SF_GZ || depth > L->lnz) return sf_fail(SF_ERR_SHAPE, "halo depth %d too deep", depth);
     size_t cnt = (size_t)depth * L->ks;
     const long lo_src = (long)SF_GZ * L->ks;                  // planes [0, d)
@@ -348,9 +355,9 @@ sf_status sf_halo(sf_level* L, int field, int depth) {
             double* lo = L->parts[q].f[field];
             double* hi = L->parts[q + 1].f[field];
             SF_CUDA(cudaMemcpyAsync(hi + lo_dst, lo + hi_src, cnt * sizeof(double),
-                                    cudaMemcpyDeviceToDevice, L->stream));
+                                    cudaMemcpyDeviceToDevice, stream));
             SF_CUDA(cudaMemcpyAsync(lo + hi_dst, hi + lo_src, cnt * sizeof(double),
-                                    cudaMemcpyDeviceToDevice, L->stream));
+                                    cudaMemcpyDeviceToDevice, stream));
         }
         return SF_OK;
     }
@@ -363,8 +370,8 @@ sf_status sf_halo(sf_level* L, int field, int depth) {
         const double* hi_x = nullptr;
         if (r > 0) { pe.sync[0] = peer_sync(L, r - 1); lo_x = peer_field(L, r - 1, x); }
         if (r < n - 1) { pe.sync[1] = peer_sync(L, r + 1); hi_x = peer_field(L, r + 1, x); }
-        const int grid = (int)std::min<long>(148, ((long)cnt + 255) / 256);
-        p2p_halo_kernel<<<grid, 256, 0, L->stream>>>(x, lo_x, hi_x, L->dsync, pe, lo_dst, hi_src, hi_dst,
+        const int grid = (int)std::min<long>(max_ctas, ((long)cnt + 255) / 256);
+        p2p_halo_kernel<<<grid, 256, 0, stream>>>(x, lo_x, hi_x, L->dsync, pe, lo_dst, hi_src, hi_dst,
                                                      lo_src, (long)cnt);
         SF_LAUNCHED();
         return sf_check_launch("p2p_halo");
@@ -389,12 +396,12 @@ sf_status sf_halo(sf_level* L, int field, int depth) {
     double* x = L->parts[0].f[field];
     SF_NCCL(g_nccl.groupStart());
     if (r > 0) {
-        SF_NCCL(g_nccl.send(x + lo_src, cnt, ncclDouble, r - 1, comm, L->stream));
-        SF_NCCL(g_nccl.recv(x + lo_dst, cnt, ncclDouble, r - 1, comm, L->stream));
+        SF_NCCL(g_nccl.send(x + lo_src, cnt, ncclDouble, r - 1, comm, stream));
+        SF_NCCL(g_nccl.recv(x + lo_dst, cnt, ncclDouble, r - 1, comm, stream));
     }
     if (r < n - 1) {
-        SF_NCCL(g_nccl.send(x + hi_src, cnt, ncclDouble, r + 1, comm, L->stream));
-        SF_NCCL(g_nccl.recv(x + hi_dst, cnt, ncclDouble, r + 1, comm, L->stream));
+        SF_NCCL(g_nccl.send(x + hi_src, cnt, ncclDouble, r + 1, comm, stream));
+        SF_NCCL(g_nccl.recv(x + hi_dst, cnt, ncclDouble, r + 1, comm, stream));
     }
     SF_NCCL(g_nccl.groupEnd());
     return SF_OK;
@@ -483,4 +490,36 @@ sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int o
     SF_NCCL(g_nccl.allReduce(dev, dev, 1, ncclDouble, op == 0 ? ncclMax : ncclSum,
                              (ncclComm_t)cm->nccl, s));
     return SF_OK;
+}
+
+// Depth-2 x halo + fused RB pair with the exchange hidden under the interior
+// (SURVEY 8e performance variant).  On a multi-part level the halo runs on a
+// side stream (fork/join by events, so CUDA graphs capture it) while the
+// interior z-chunks [1, nch-1) are smoothed -- they read no ghost plane -- and
+// the boundary chunks 0 and nch-1 run after the join.  Same arithmetic per
+// cell as one launch over all chunks (bit-identical).  SF_HALO_OVERLAP=0 turns
+// it off (exchange, then one launch).
+sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, double b, double* rmax,
+                           sf_level* C, int cf) {
+    const char* ev = getenv("SF_HALO_OVERLAP");
+    const int ov = ev ? atoi(ev) : 1;
+    const bool split = ov && L->nparts > 1 && L->comm && L->comm->kind != 2 && L->lnz >= 24;
+    if (!split) {
+        SF_TRY(sf_halo(L, xin, 2));
+        return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf);
+    }
+    if (!L->side) {
+        SF_CUDA(cudaStreamCreateWithFlags(&L->side, cudaStreamNonBlocking));
+        SF_CUDA(cudaEventCreateWithFlags(&L->ev_fork, cudaEventDisableTiming));
+        SF_CUDA(cudaEventCreateWithFlags(&L->ev_join, cudaEventDisableTiming));
+    }
+    SF_CUDA(cudaEventRecord(L->ev_fork, L->stream));
+    SF_CUDA(cudaStreamWaitEvent(L->side, L->ev_fork, 0));
+    SF_TRY(sf_halo_on(L, xin, 2, L->side));
+    SF_CUDA(cudaEventRecord(L->ev_join, L->side));
+    // copy-engine transfers (kind 0) need no SM; kernels / NCCL get two
+    const int reserve = L->comm->kind == 0 ? 0 : 2;
+    SF_TRY(k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 1, reserve));
+    SF_CUDA(cudaStreamWaitEvent(L->stream, L->ev_join, 0));
+    return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 2, 0);
 }

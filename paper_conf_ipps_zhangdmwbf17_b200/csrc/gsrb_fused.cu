@@ -249,7 +249,7 @@ template <bool RESID, bool INTERP>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
-                     CoarseView cv) {
+                     CoarseView cv, int c0, int cstride) {
     constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
@@ -267,7 +267,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
     unsigned long long rbits = 0ull;  // RESID: max |rhs - A x_in| of this thread's cells
     unsigned seq = 0;  // bundles issued by this CTA so far (all threads track it)
     for (int item = blockIdx.x; item < nitems; item += gridDim.x) {
-        const int chunk = item / ntiles, tile = item - chunk * ntiles;
+        const int ci = item / ntiles, tile = item - ci * ntiles;
+        const int chunk = c0 + ci * cstride;  // z-chunks of this launch (all / interior / boundary)
         const int x0 = (tile % ntx) * TX, y0 = (tile / ntx) * TY;
         const int z0 = chunk * depth, z1 = min(z0 + depth, g.nz);
         const int cx = SF_OX + x0 - 2;        // TMA x coordinate of the box
@@ -566,8 +567,13 @@ static __global__ void zero_bits(double* p) { *p = 0.0; }
 // rmax != NULL: also reduce max |rhs - A x_in| of the INPUT iterate into *rmax
 // (device scalar; the caller all-reduces across ranks).
 // C != NULL: fuse fine.xin += P0(C.cf) (A8, V-cycle) into the pair (INTERP).
+// phase 0: every z-chunk; 1: the interior chunks [1, nch-1) with `reserve` SMs
+// left free (the halo exchange runs beside it); 2: the boundary chunks 0 and
+// nch-1, which read the exchanged ghost planes.  Phases 1 and 2 use at least
+// 3 chunks per part.
 sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
-                                                    double b, double* rmax, sf_level* C, int cf) {
+                                                    double b, double* rmax, sf_level* C, int cf,
+                                                    int phase, int reserve) {
     if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
     SF_TRY(get_encoder());
     static bool attr = false;
@@ -596,9 +602,12 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     const int G = g_num_sms * MINB;   // resident CTAs
     int best_d = L->lnz;
     double best = 1e30;
-    for (int nch = 1; nch <= L->lnz; nch++) {
+    const int min_nch = phase ? 3 : 1;
+    if (L->lnz < min_nch) return sf_fail(SF_ERR_SHAPE, "split fused pair needs >= 3 planes per part");
+    for (int nch = min_nch; nch <= L->lnz; nch++) {
         int d = (L->lnz + nch - 1) / nch;
-        if (d < 8 && nch > 1) break;
+        if (d < 8 && nch > min_nch) break;
+        if ((L->lnz + d - 1) / d < min_nch) continue;
         int n = (L->lnz + d - 1) / d;
         long items = (long)tiles * n;
         double rounds = (double)((items + G - 1) / G);
@@ -607,8 +616,12 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     }
     const char* ed = getenv("SF_GSRB_DEPTH");   // tuning override
     if (ed && atoi(ed) > 0) best_d = std::min(L->lnz, atoi(ed));
+    if (phase) best_d = std::min(best_d, L->lnz / 3);
     const int depth = best_d, nch = (L->lnz + depth - 1) / depth;
-    const int items = tiles * nch;
+    const int c0 = phase == 1 ? 1 : 0;
+    const int cstride = phase == 2 ? nch - 1 : 1;
+    const int items = tiles * (phase == 0 ? nch : phase == 1 ? nch - 2 : 2);
+    const int Gl = phase == 1 ? std::max(1, g_num_sms - reserve) * MINB : G;
     const double bh2 = b / (L->h * L->h);
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
@@ -620,7 +633,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY(encode(&mp.bj, L, v.f[SF_BETA_J], CHH));
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
-        int grid = std::min(items, G);
+        int grid = std::min(items, Gl);
         CoarseView cvw{nullptr, 0, 0, 0};
         if (C) {
             const bool rep = C->nparts == 1 && L->nparts > 1;
@@ -628,18 +641,18 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
             cvw = CoarseView{c.f[cf], C->js, C->ks, rep ? v.z0 / 2 : 0};
         }
         if (rmax) {
-            if (p == 0) {
+            if (p == 0 && phase != 2) {
                 zero_bits<<<1, 1, 0, L->stream>>>(rmax);
                 SF_LAUNCHED();
             }
             gsrb_pair_tma_kernel<true, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax, cvw);
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax, cvw, c0, cstride);
         } else if (C) {
             gsrb_pair_tma_kernel<false, true><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw);
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw, c0, cstride);
         } else {
             gsrb_pair_tma_kernel<false, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw);
+                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw, c0, cstride);
         }
         SF_LAUNCHED();
     }

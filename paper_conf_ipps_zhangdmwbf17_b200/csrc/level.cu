@@ -160,6 +160,12 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
 extern "C" sf_status sf_level_destroy(sf_level* L) {
     if (!L) return SF_OK;
     cudaStreamSynchronize(L->stream);
+    if (L->side) {
+        cudaStreamSynchronize(L->side);
+        cudaStreamDestroy(L->side);
+    }
+    if (L->ev_fork) cudaEventDestroy(L->ev_fork);
+    if (L->ev_join) cudaEventDestroy(L->ev_join);
     sf_ipc_close(L);
     if (L->owns) cudaFree(L->buf);
     cudaFreeHost(L->hscratch);
@@ -395,17 +401,17 @@ bool gsrb_fused_supported(const sf_level* L) {
 }
 
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                            double* rmax, sf_level* C, int cf) {
+                            double* rmax, sf_level* C, int cf, int phase, int reserve) {
     // 32x8 tiles with two CTAs per SM measured 1.5-2 % faster up to 256^3 and
     // 1.7 % slower at 512^3 than 32x16 with one (profiles/r01/ncu_variants_ab.txt);
     // SF_GSRB_W4 = 0 / 1 forces the choice
     static const int w4 = getenv("SF_GSRB_W4") ? atoi(getenv("SF_GSRB_W4")) : -1;
     const bool small = (long)L->nx * L->ny * L->lnz <= (1L << 24);
     if ((w4 == 1 || (w4 < 0 && small)) && gsrb_fused_supported_t32w4(L))
-        return k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, rmax, C, cf);
+        return k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve);
     if (gsrb_fused_supported_t32(L))
-        return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax, C, cf);
-    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b, rmax, C, cf);
+        return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve);
+    return k_gsrb_pair_fused_t64(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve);
 }
 
 void sf_swap_fields(sf_level* L, int f1, int f2) {
@@ -430,8 +436,7 @@ extern "C" sf_status sf_smooth_gsrb(sf_level* L, int x, int rhs, double a, doubl
         int other = (x == SF_U) ? SF_TMP : SF_U;
         SF_TRY(sf_halo(L, rhs, 1));
         for (int p = 0; p < rb_pairs; p++) {
-            SF_TRY(sf_halo(L, x, 2));
-            SF_TRY(k_gsrb_pair_fused(L, x, other, rhs, a, b));
+            SF_TRY(k_gsrb_pair_halo(L, x, other, rhs, a, b));
             sf_swap_fields(L, x, other);  // result now lives under the id `x`
         }
         return SF_OK;

@@ -251,8 +251,7 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
         // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
         SF_TRY(sf_halo(C, SF_U, 1));
         SF_TRY(sf_halo(L, SF_F, 1));
-        SF_TRY(sf_halo(L, SF_U, 2));
-        SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, nullptr, C, SF_U));
+        SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, nullptr, C, SF_U));
         sf_swap_fields(L, SF_U, SF_TMP);
         SF_TRY(smooth(m, L, m->o.post_pairs - 1));
         return SF_OK;
@@ -303,8 +302,7 @@ static bool fused_check_ok(const sf_mg* m) {
 static sf_status first_pair_check(sf_mg* m) {
     sf_level* L = m->lv[0];
     SF_TRY(sf_halo(L, SF_F, 1));
-    SF_TRY(sf_halo(L, SF_U, 2));
-    SF_TRY(k_gsrb_pair_fused(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
+    SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
     sf_swap_fields(L, SF_U, SF_TMP);
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
         SF_TRY(sf_allreduce_scalar(L, L->comm, L->dscratch, 0));

@@ -21,7 +21,7 @@ from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
 
 pytestmark = pytest.mark.gpu
 
-SMOOTH_SHAPE = (32, 16, 64)
+SMOOTH_SHAPE = (96, 16, 64)   # >= 24 planes per rank: halo overlapped with the interior chunks
 N_SOLVE = 64
 
 

@@ -423,6 +423,41 @@ def test_decomposition_invariance_smoother(sf, parts):
 
 
 @pytest.mark.parametrize("parts", [2, 4])
+@pytest.mark.parametrize("overlap", ["1", "0"])
+def test_halo_overlap_bit_identical(sf, oracle, parts, overlap, monkeypatch):
+    """>= 24 planes per part: the depth-2 halo runs on a side stream beside the
+    interior z-chunks, the boundary chunks after the join (SF_HALO_OVERLAP=1),
+    or before one launch (0).  Both equal the undecomposed level bit for bit,
+    for the plain, check-fused (solve) and P0-fused (V-cycle) pairs."""
+    monkeypatch.setenv("SF_HALO_OVERLAP", overlap)
+    shape = (96, 32, 64)
+    nz, ny, nx = shape
+    coeffs = I.hpgmg_coeffs(nx, ny, nz)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    out = {}
+    for P in (1, parts):
+        L = make_level(sf, shape, coeffs, parts=P)
+        sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+        L.upload(sf.SF_U, x)
+        L.upload(sf.SF_F, f)
+        sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 3, sf.SF_SMOOTH_FUSED)
+        out[P] = L.download(sf.SF_U)
+    assert np.array_equal(out[1], out[parts])
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, I.level_h(nx, ny, nz)), 1.0, 1.0, *coeffs)
+    assert rel(out[parts], P.smooth(x, f, 3, dinv=P.dinv())) < TOL
+    n = 96
+    sol = {}
+    for Pn in (1, parts):
+        L, M, O = mg_pair(sf, oracle, n, shape=(n, 64, 64), parts=Pn, agglom_min_planes=4)
+        _, fm = I.manufactured(64, 64, n, 1.0, 1.0)
+        L.upload(sf.SF_F, fm)
+        st, cyc, hist = M.solve(fcycle=True)
+        sol[Pn] = (L.download(sf.SF_U), cyc)
+    assert sol[1][1] == sol[parts][1]
+    assert rel(sol[parts][0], sol[1][0]) < 1e-13
+
+
+@pytest.mark.parametrize("parts", [2, 4])
 def test_decomposition_invariance_solve(sf, oracle, parts):
     n = 64
     shape = (n, n, n)
