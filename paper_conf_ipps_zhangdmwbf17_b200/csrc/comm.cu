@@ -500,13 +500,13 @@ sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int o
 // cell as one launch over all chunks (bit-identical).  SF_HALO_OVERLAP=0 turns
 // it off (exchange, then one launch).
 sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, double b, double* rmax,
-                           sf_level* C, int cf) {
+                           sf_level* C, int cf, int rmode) {
     const char* ev = getenv("SF_HALO_OVERLAP");
     const int ov = ev ? atoi(ev) : 1;
     const bool split = ov && L->nparts > 1 && L->comm && L->comm->kind != 2 && L->lnz >= 24;
     if (!split) {
         SF_TRY(sf_halo(L, xin, 2));
-        return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf);
+        return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 0, 0, rmode);
     }
     if (!L->side) {
         SF_CUDA(cudaStreamCreateWithFlags(&L->side, cudaStreamNonBlocking));
@@ -519,7 +519,7 @@ sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, do
     SF_CUDA(cudaEventRecord(L->ev_join, L->side));
     // copy-engine transfers (kind 0) need no SM; kernels / NCCL get two
     const int reserve = L->comm->kind == 0 ? 0 : 2;
-    SF_TRY(k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 1, reserve));
+    SF_TRY(k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 1, reserve, rmode));
     SF_CUDA(cudaStreamWaitEvent(L->stream, L->ev_join, 0));
-    return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 2, 0);
+    return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 2, 0, rmode);
 }

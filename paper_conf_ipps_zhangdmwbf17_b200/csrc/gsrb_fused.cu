@@ -126,11 +126,11 @@ struct StepCtx {
 // the odd cell of the pair is red at this plane (warp-uniform).  Returns the
 // red-new value; leaves the black cell's coefficients of the plane in nb
 // (bw, be, bs, bn, bb, bt, dinv, rhs).  RESID: rres = rhs - A x_in at the red
-// cell (A x = x(c)/dinv - b h^-2 S), rold = its old value, xpair = old pair.
+// cell (A x = x(c)/dinv - b h^-2 S): the red part of the INPUT's residual.
 template <int SEL, bool RESID>
 __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
                                            int gy, const Geo& g, bool zlo, bool zhi, double bh2,
-                                           double* nb, double& rres, double& rold, double2& xpair) {
+                                           double* nb, double& rres) {
     const double2 xp2 = *(const double2*)&s.Xk[xo_];
     const double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
     const double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
@@ -170,44 +170,18 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
         nb[0] = bi2.x; nb[1] = bi2.y; nb[2] = bjl.x; nb[3] = bjh.x; nb[4] = bkl.x; nb[5] = bkh.x;
         nb[6] = dv2.x; nb[7] = rh2.x;
     }
-    rold = SEL ? xp2.y : xp2.x;
-    xpair = xp2;
     return r;
 }
 
-// Residual rhs - A x of the INPUT iterate at the black cell (position BS) of
-// plane q, computed during R(q) before any red write: in-plane red neighbours
-// are still old in smem, the red cell below (same column, plane q-1) is this
-// thread's red-old value of the previous plane, the one above is untouched.
-template <int BS>
-__device__ __forceinline__ double black_resid(const StepCtx& s, int xo_, int gx, int gy,
-                                              const Geo& g, bool zlo, bool zhi, double bh2,
-                                              const double* nb, double rold_below, double2 xp2) {
-    double xw, xe;
-    if (BS == 1) {
-        xw = xp2.x; xe = s.Xk[xo_ + 2];
-    } else {
-        xw = s.Xk[xo_ - 1]; xe = xp2.y;
-    }
-    const double xc = BS ? xp2.y : xp2.x;
-    const int gxb = gx + BS;
-    if (gxb == 0) xw = 0.0;
-    if (gxb == g.nx - 1) xe = 0.0;
-    const int col = xo_ + BS;
-    const double xs = (gy == 0) ? 0.0 : s.Xk[col - W];
-    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
-    const double xb = zlo ? 0.0 : rold_below;
-    const double xt = zhi ? 0.0 : s.Xp[col];
-    const double S = sum6(xw, xe, xs, xn, xb, xt, nb[0], nb[1], nb[2], nb[3], nb[4], nb[5]);
-    return (nb[7] + bh2 * S) - xc * inv_fast(nb[6]);
-}
-
 // B for the pair; SEL = position (0: even x, 1: odd x) of the black cell in
-// the pair.  Returns the output pair (red-new, black-new in place).
-template <int SEL, bool TOPREG = false>
+// the pair.  Returns the output pair (red-new, black-new in place).  BRES: bres
+// = rhs - A x at the black cell AFTER its update, q - x_new/dinv with q the
+// quantity the update just formed (its red neighbours are final: this is the
+// black part of the residual of the pair's output).
+template <int SEL, bool BRES>
 __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx, int gy,
                                               const Geo& g, int gkm, double bh2, const double* rb,
-                                              double top = 0.0) {
+                                              double& bres) {
     const double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
     double xw, xe;
     if (SEL == 0) {
@@ -222,11 +196,10 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
     const double xs = (gy == 0) ? 0.0 : s.Xm[col - W];
     const double xn = (gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
     const double xb = (gkm == 0) ? 0.0 : s.Xmm[col];
-    // TOPREG: the red cell above is this thread's own red-new of the previous
-    // step, not yet stored (RESID defers its red writes by one step)
-    const double xt = (gkm == g.gnz - 1) ? 0.0 : (TOPREG ? top : s.Xk[col]);
-    const double bnew =
-        gs_upd(rb[6], rb[7], bh2, sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
+    const double xt = (gkm == g.gnz - 1) ? 0.0 : s.Xk[col];
+    const double q = gs_q(rb[7], bh2, sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
+    const double bnew = __dmul_rn(rb[6], q);
+    if (BRES) bres = __fma_rn(-bnew, inv_fast(rb[6]), q);
     return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
 }
 
@@ -245,7 +218,10 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
     return gs_upd(s.C[CA_DV * CARR + co_], s.C[CA_RH * CARR + co_], bh2, S);
 }
 
-template <bool RESID, bool INTERP>
+// RESID: max |rhs - A x| over the red cells of the INPUT (the black part of
+// that residual was reduced by the BRES pair that produced the input).
+// BRES: max |rhs - A x| over the black cells of the OUTPUT.  Both into *rmax.
+template <bool RESID, bool INTERP, bool BRES>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
@@ -264,7 +240,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
     }
     __syncthreads();
 
-    unsigned long long rbits = 0ull;  // RESID: max |rhs - A x_in| of this thread's cells
+    unsigned long long rbits = 0ull;  // RESID / BRES: max |rhs - A x| of this thread's cells
     unsigned seq = 0;  // bundles issued by this CTA so far (all threads track it)
     for (int item = blockIdx.x; item < nitems; item += gridDim.x) {
         const int ci = item / ntiles, tile = item - ci * ntiles;
@@ -343,7 +319,6 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                            ((rgy == g.ny - 1) << 3);
             }
         }
-        double rold = 0.0;  // RESID: red-old value of the previous plane (this pair)
         double stA[8], stB[8];
 #pragma unroll
         for (int i = 0; i < 8; i++) stA[i] = stB[i] = 0.0;
@@ -398,13 +373,6 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             __syncthreads();
         }
 
-        // RESID: red-new values (tile + ring) of the plane computed at step t are
-        // stored at the end of step t+1, after the barrier that ends step t:
-        // the black residuals of step t read that plane's red-OLD values, so an
-        // immediate store would need a second barrier per step
-        double prn = 0.0, prr = 0.0;
-        int pxo = 0, pro = 0;
-        bool pw = false, pwr = false;
         auto step = [&](int t, double* stash) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
@@ -434,40 +402,28 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const int gkm = g.z0 + t - 1;
             // planes t+1 and t-1 have the same parity: the black cell of
             // plane t-1 is the pair's other cell (position 1-sel)
-            double rres = 0.0, rold_new = 0.0, bres = 0.0;
-            double2 xpair = make_double2(0.0, 0.0);
+            double rres = 0.0, bres = 0.0;
             if (sel == 0) {
-                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
-                                                 rres, rold_new, xpair);
-                if (bin) o = black_pair<1, RESID>(sb, xoff, gxa, gy, g, gkm, bh2, stash, prn);
-                if (RESID && rin)
-                    bres = black_resid<1>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
+                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
+                if (bin) o = black_pair<1, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres);
             } else {
-                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb,
-                                                 rres, rold_new, xpair);
-                if (bin) o = black_pair<0, RESID>(sb, xoff, gxa, gy, g, gkm, bh2, stash, prn);
-                if (RESID && rin)
-                    bres = black_resid<0>(s, xoff, gxa, gy, g, zlo, zhi, bh2, nb, rold, xpair);
+                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
+                if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres);
             }
-            if (RESID) {
-                if (rin && q >= z0 && q < z1) {   // this item's planes only
-                    unsigned long long m2 = abits(rres) > abits(bres) ? abits(rres) : abits(bres);
-                    rbits = m2 > rbits ? m2 : rbits;
-                }
-                rold = rold_new;
+            if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
+                const unsigned long long m2 = abits(rres);
+                rbits = m2 > rbits ? m2 : rbits;
+            }
+            if (BRES && bin) {
+                const unsigned long long m2 = abits(bres);
+                rbits = m2 > rbits ? m2 : rbits;
             }
             const int par = gkr & 1;
             const bool ring = rin && (par ? rok[1] : rok[0]);
             const int ro = par ? rxo[1] : rxo[0];
             double rr = 0.0;
             if (ring) rr = red_ring(s, ro, par ? rco[1] : rco[0], par ? rfl[1] : rfl[0], bh2, zlo, zhi);
-            if (RESID) {
-                double* Xp = Xs + ix_0 * XSLOT;   // plane t: computed at step t-1
-                if (pw) Xp[pxo] = prn;
-                if (pwr) Xp[pro] = prr;
-                prn = rn; pxo = xoff + sel; pw = rin;
-                prr = rr; pro = ro; pwr = ring;
-            } else {
+            {
                 double* Xw = Xs + ix_p1 * XSLOT;
                 if (rin) Xw[xoff + sel] = rn;
                 if (ring) Xw[ro] = rr;
@@ -503,7 +459,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
     }
-    if (RESID) {   // CTA max -> one atomic (bit order = numeric order for |r|; NaN wins)
+    if (RESID || BRES) {   // CTA max -> one atomic (bit order = numeric order for |r|; NaN wins)
         __shared__ unsigned long long wmax[NWARP];
         for (int o2 = 16; o2 > 0; o2 >>= 1) {
             unsigned long long v = __shfl_xor_sync(0xffffffffu, rbits, o2);
@@ -564,8 +520,20 @@ bool SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(const sf_level* L) {
 
 static __global__ void zero_bits(double* p) { *p = 0.0; }
 
-// rmax != NULL: also reduce max |rhs - A x_in| of the INPUT iterate into *rmax
-// (device scalar; the caller all-reduces across ranks).
+template <bool R, bool I, bool B>
+static sf_status set_attrs() {
+    SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
+    if (MINB > 1)   // room for MINB CTAs per SM
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B>,
+                                     cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+    return SF_OK;
+}
+
+// rmode SF_RM_INPUT_RED: reduce max |rhs - A x| over the red cells of the
+// INPUT into *rmax (no reset: the BRES pair that produced the input holds the
+// black part there).  SF_RM_OUTPUT_BLACK: reset *rmax, reduce the black cells
+// of the OUTPUT.  The caller all-reduces *rmax across ranks.
 // C != NULL: fuse fine.xin += P0(C.cf) (A8, V-cycle) into the pair (INTERP).
 // phase 0: every z-chunk; 1: the interior chunks [1, nch-1) with `reserve` SMs
 // left free (the halo exchange runs beside it); 2: the boundary chunks 0 and
@@ -573,25 +541,18 @@ static __global__ void zero_bits(double* p) { *p = 0.0; }
 // 3 chunks per part.
 sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
                                                     double b, double* rmax, sf_level* C, int cf,
-                                                    int phase, int reserve) {
+                                                    int phase, int reserve, int rmode) {
     if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
+    if (rmode != SF_RM_NONE && !rmax) return sf_fail(SF_ERR_INVALID, "residual mode needs a scalar");
+    if (rmode == SF_RM_INPUT_RED && C) return sf_fail(SF_ERR_INVALID, "input residual with P0 fusion");
     SF_TRY(get_encoder());
     static bool attr = false;
     if (!attr) {
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, false>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<true, false>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, true>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
-        if (MINB > 1) {   // room for MINB CTAs per SM
-            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, false>,
-                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<true, false>,
-                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-            SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<false, true>,
-                                         cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-        }
+        SF_TRY((set_attrs<false, false, false>()));
+        SF_TRY((set_attrs<true, false, false>()));
+        SF_TRY((set_attrs<false, true, false>()));
+        SF_TRY((set_attrs<false, false, true>()));
+        SF_TRY((set_attrs<false, true, true>()));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
         SF_CUDA(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
@@ -640,20 +601,20 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
             PV c = sf_view(C, rep ? 0 : p);
             cvw = CoarseView{c.f[cf], C->js, C->ks, rep ? v.z0 / 2 : 0};
         }
-        if (rmax) {
-            if (p == 0 && phase != 2) {
-                zero_bits<<<1, 1, 0, L->stream>>>(rmax);
-                SF_LAUNCHED();
-            }
-            gsrb_pair_tma_kernel<true, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, rmax, cvw, c0, cstride);
-        } else if (C) {
-            gsrb_pair_tma_kernel<false, true><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw, c0, cstride);
-        } else {
-            gsrb_pair_tma_kernel<false, false><<<grid, NT, SMEM, L->stream>>>(
-                mp, g, v.f[xout], a, bh2, depth, ntx, tiles, items, nullptr, cvw, c0, cstride);
+        if (rmode == SF_RM_OUTPUT_BLACK && p == 0 && phase != 2) {
+            zero_bits<<<1, 1, 0, L->stream>>>(rmax);
+            SF_LAUNCHED();
         }
+        double* xo = v.f[xout];
+#define SF_LAUNCH_PAIR(R, I, B)                                                                     \
+    gsrb_pair_tma_kernel<R, I, B><<<grid, NT, SMEM, L->stream>>>(mp, g, xo, a, bh2, depth, ntx, tiles, \
+                                                                items, rmax, cvw, c0, cstride)
+        if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
+        else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);
+        else if (rmode == SF_RM_OUTPUT_BLACK) SF_LAUNCH_PAIR(false, false, true);
+        else if (C) SF_LAUNCH_PAIR(false, true, false);
+        else SF_LAUNCH_PAIR(false, false, false);
+#undef SF_LAUNCH_PAIR
         SF_LAUNCHED();
     }
     return sf_check_launch("gsrb_pair_tma");

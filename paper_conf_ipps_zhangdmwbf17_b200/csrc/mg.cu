@@ -220,9 +220,23 @@ static sf_status smooth(sf_mg* m, sf_level* L, int pairs) {
     return sf_smooth_gsrb(L, SF_U, SF_F, m->a, m->b, pairs, m->o.smoother);
 }
 
+static bool fused_check_ok(const sf_mg* m);
+
+// The finest level's last post-smoothing pair of a cycle also reduces the black
+// part of max|F - A U| of its output into dscratch (BRES); the next cycle's
+// first pair adds the red part of the same iterate (fused check, below).
+static sf_status bres_pair(sf_mg* m, sf_level* L) {
+    SF_TRY(sf_halo(L, SF_F, 1));
+    SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch, nullptr, 0,
+                            SF_RM_OUTPUT_BLACK));
+    sf_swap_fields(L, SF_U, SF_TMP);
+    return SF_OK;
+}
+
 // V(l): smooth, residual, restrict, zero e_{l+1}, V(l+1), e_l += P0 e_{l+1}, smooth.
 // skip_first: the first pre-smoothing pair was already run (fused check, below).
 static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
+    const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     sf_level* C = m->lv[l + 1];
@@ -251,12 +265,22 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
         // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
         SF_TRY(sf_halo(C, SF_U, 1));
         SF_TRY(sf_halo(L, SF_F, 1));
-        SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, nullptr, C, SF_U));
+        const bool last = bres && m->o.post_pairs == 1;
+        SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, last ? L->dscratch : nullptr, C,
+                                SF_U, last ? SF_RM_OUTPUT_BLACK : SF_RM_NONE));
         sf_swap_fields(L, SF_U, SF_TMP);
+        if (bres && m->o.post_pairs >= 2) {
+            SF_TRY(smooth(m, L, m->o.post_pairs - 2));
+            return bres_pair(m, L);
+        }
         SF_TRY(smooth(m, L, m->o.post_pairs - 1));
         return SF_OK;
     }
     SF_TRY(k_interp(L, SF_U, 1.0, C, SF_U, m->o.vcycle_interp));
+    if (bres) {
+        SF_TRY(smooth(m, L, m->o.post_pairs - 1));
+        return bres_pair(m, L);
+    }
     SF_TRY(smooth(m, L, m->o.post_pairs));
     return SF_OK;
 }
@@ -289,12 +313,15 @@ static sf_status check(sf_mg* m) {
     return to_host(L);
 }
 
-// The convergence check fused into the next cycle's first pre-smoothing pair:
-// the colour-fused pair streams every operand anyway and reduces
-// max|F - A U_in| of its INPUT while it writes the smoothed iterate to TMP.
-// If that says "converged", U (the previous cycle's result) is untouched.
+// The convergence check rides in the colour-fused pairs that stream every
+// operand anyway: max|F - A U| of the iterate after a cycle is the max of its
+// black part, reduced by the cycle's last post-smoothing pair right after each
+// black update (BRES: the red neighbours are final then), and its red part,
+// reduced by the next cycle's first pre-smoothing pair from its INPUT while it
+// writes the smoothed iterate to TMP.  If that says "converged", U (the
+// previous cycle's result) is untouched.
 static bool fused_check_ok(const sf_mg* m) {
-    return m->lv.size() > 1 && m->o.pre_pairs >= 1 &&
+    return m->lv.size() > 1 && m->o.pre_pairs >= 1 && m->o.post_pairs >= 1 &&
            (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
            gsrb_fused_supported(m->lv[0]) && (m->o.pre_pairs + m->o.post_pairs) % 2 == 0;
 }
@@ -302,7 +329,8 @@ static bool fused_check_ok(const sf_mg* m) {
 static sf_status first_pair_check(sf_mg* m) {
     sf_level* L = m->lv[0];
     SF_TRY(sf_halo(L, SF_F, 1));
-    SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch));
+    SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch, nullptr, 0,
+                            SF_RM_INPUT_RED));
     sf_swap_fields(L, SF_U, SF_TMP);
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
         SF_TRY(sf_allreduce_scalar(L, L->comm, L->dscratch, 0));

@@ -105,6 +105,9 @@ sf_status sf_fail(sf_status s, const char* fmt, ...);
 void sf_count_launch(long long n = 1);
 sf_status sf_check_launch(const char* what);
 
+// residual reductions riding in a fused pair (rmax = device scalar)
+enum { SF_RM_NONE = 0, SF_RM_INPUT_RED = 1, SF_RM_OUTPUT_BLACK = 2 };
+
 // ------------------------------------------------------------------ kernels (kernels.cu)
 sf_status k_apply_op(sf_level* L, int out, int x, double a, double b);
 sf_status k_residual(sf_level* L, int res, int x, int rhs, double a, double b);
@@ -142,24 +145,28 @@ sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, 
 bool gsrb_fused_supported_t32(const sf_level* L);
 bool gsrb_fused_supported_t64(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                                double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0);
+                                double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
+                                int rmode = 0);
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                                double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0);
+                                double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
+                                int rmode = 0);
 // 32x8 tiles, 4 warps, 2 CTAs per SM (two independent z-step chains per SM)
 bool gsrb_fused_supported_t32w4(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32w4(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                                  double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0);
+                                  double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
+                                int rmode = 0);
 bool gsrb_fused_supported(const sf_level* L);
 // rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax;
 // C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
                             double* rmax = nullptr, sf_level* C = nullptr, int cf = 0,
-                            int phase = 0, int reserve = 0);
+                            int phase = 0, int reserve = 0, int rmode = SF_RM_NONE);
 // the depth-2 x halo exchange + fused pair, overlapped on multi-part levels:
 // the halo runs on a side stream while the interior z-chunks are smoothed, then
 // the boundary chunks (comm.cu)
 sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, double b,
-                           double* rmax = nullptr, sf_level* C = nullptr, int cf = 0);
+                           double* rmax = nullptr, sf_level* C = nullptr, int cf = 0,
+                           int rmode = SF_RM_NONE);
 // halo exchange enqueued on stream s instead of the level's stream (kinds 0, 1, 3)
 sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t s);
 // last pre-smoothing pair fused with residual + restriction (gsrb_rr.cu):
