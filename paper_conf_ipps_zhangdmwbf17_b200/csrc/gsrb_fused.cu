@@ -380,6 +380,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 const unsigned sq = seq0 + 2 + (q - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
             }
+
             const int gkr = g.z0 + q;                    // plane of R
             const bool rin = q <= z1 && gkr >= 0 && gkr < g.gnz;
             const bool bin = t - 1 >= z0;                // B(t-1) on the tile
@@ -435,6 +436,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             for (int i = 0; i < 8; i++) stash[i] = nb[i];
             // INTERP: correct x(t+3) (bundle t+2) at the END of the step: no one
             // reads that plane before step t+1, and the TMA had the whole step
+            // (correcting at the start of the step instead measured slower:
+            // the wait for bundle t+2 then stalls the step's stencils)
             if (INTERP && q + 1 <= z1) {
                 const unsigned sq = seq0 + 2 + (q + 1 - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);

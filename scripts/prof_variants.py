@@ -10,6 +10,8 @@ sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
 M = sf.MG(L, 1.0, 1.0, use_graph=0)
 if mode == "vcycle":
     sf.sf_vcycle(M.handle, 0)
+elif mode == "fcycle":
+    sf.sf_fcycle(M.handle)
 else:
     M.solve(fcycle=False, max_cycles=2, raise_on_error=False)
 sf.sf_sync(L.handle)

@@ -13,10 +13,10 @@ timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum,dram__
 echo "solve launch list exit $?"
 for n in 512 256; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:gsrb_pair -s 2 -c 1 \
-     -o gpurun_out/prof_gsrb_v10_$n -f python scripts/prof_gsrb.py $n 3 fused > gpurun_out/ncu_v10_$n.log 2>&1
+     -o gpurun_out/prof_gsrb_v11_$n -f python scripts/prof_gsrb.py $n 3 fused > gpurun_out/ncu_v11_$n.log 2>&1
   echo "ncu pair $n exit $?"
 done
-bash scripts/prof_variants.sh v10 > /dev/null 2>&1; echo "variants exit $?"
+bash scripts/prof_variants.sh v11 > /dev/null 2>&1; echo "variants exit $?"
 timeout 600 ncu --set full --clock-control none -k regex:sf_stencil_group -c 6 -o gpurun_out/prof_dsl_256 -f \
    python scripts/dsl_once.py 256 > gpurun_out/ncu_dsl.log 2>&1; echo "dsl exit $?"
 python scripts/dsl_time.py 256 > gpurun_out/dsl_time.txt 2>&1
