@@ -361,7 +361,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 *(double2*)&X[2 * ep1] = u;
             }
         };
-        double ce0 = 0.0, ce1 = 0.0;   // parents for the next plane to correct
+        // parents of the next two planes to correct (loaded two steps ahead: the
+        // coarse field may come from DRAM, slower than one z step)
+        double ce0 = 0.0, ce1 = 0.0, cn0 = 0.0, cn1 = 0.0;
         if (INTERP) {
             mbar_wait(&mbar[(seq0 + 1) % NMB], ((seq0 + 1) / NMB) & 1);   // bundle z0-1: x(z0)
             for (int p = z0 - 2; p <= z0; p++) {
@@ -370,6 +372,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 correct(p, e0, e1);
             }
             if (z0 + 1 <= z1 + 1) load_e(z0 + 1, ce0, ce1);
+            if (z0 + 2 <= z1 + 1) load_e(z0 + 2, cn0, cn1);
             __syncthreads();
         }
 
@@ -442,7 +445,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 const unsigned sq = seq0 + 2 + (q + 1 - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
                 correct(t + 3, ce0, ce1);
-                if (t + 4 <= z1 + 1) load_e(t + 4, ce0, ce1);
+                ce0 = cn0;
+                ce1 = cn1;
+                if (t + 5 <= z1 + 1) load_e(t + 5, cn0, cn1);
             }
             fence_proxy_async();
             __syncthreads();
