@@ -18,7 +18,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsf.so")
+# SF_LIB: A/B timing of another build of the same library (scripts/ab_lib.sh)
+LIB_PATH = os.environ.get("SF_LIB") or os.path.join(_HERE, "libsf.so")
 
 # enums (include/sf.h)
 SF_OK, SF_ERR_INVALID, SF_ERR_SHAPE, SF_ERR_OOM, SF_ERR_CUDA, SF_ERR_NCCL = range(6)

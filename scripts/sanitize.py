@@ -22,3 +22,24 @@ for n, parts in ((32, 1), (64, 1), (64, 2)):
     M.close(); L.close()
     if comm:
         comm.close()
+
+# halo exchange beside the interior chunks (2 parts x 24 planes), the pair +
+# residual + restriction kernel (SF_RR=1) and the 32x16 build (SF_GSRB_W4=0)
+comm = sf.Comm.local(2)
+L = sf.Level(64, 32, 48, 1.0 / 64, comm=comm)
+sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
+sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, sf.SF_SMOOTH_FUSED)
+sf.sf_sync(L.handle)
+print("ok overlap", flush=True)
+L.close()
+comm.close()
+os.environ["SF_RR"] = "1"
+F = sf.Level(64, 32, 12, 1.0 / 64)
+C = sf.Level(32, 16, 6, 2.0 / 64)
+sf.sf_init_problem(F.handle, 1, 1.0, 1.0, 1)
+sf.sf_rebuild_operator(F.handle, 1.0, 1.0)
+sf.sf_smooth_residual_restrict(F.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, sf.SF_F)
+sf.sf_sync(F.handle)
+print("ok rr", flush=True)
+F.close(); C.close()
