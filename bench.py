@@ -280,7 +280,7 @@ def main():
     side = {}
     if not args.quick:
         side = side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_ranks,
-                                 dof_local, cyc)
+                                 dof_local, cyc, comm)
 
     if rank == 0:
         pk, pk_src = peaks()
@@ -319,7 +319,7 @@ def main():
             "roofline": roof,
         }
         line.update({k: v for k, v in side.items() if k in (
-            "e2e", "gsrb_c3", "vcycle", "fcycle", "read_bw", "cpu_baseline", "fig7_256",
+            "e2e", "gsrb_c3", "vcycle", "fcycle", "fcycle_strong", "read_bw", "cpu_baseline", "fig7_256",
             "gsrb_size_sweep", "dsl_256")})
         print(json.dumps(line), flush=True)
     M.close()
@@ -331,7 +331,7 @@ def main():
 
 
 def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_ranks, dof_local,
-                      cyc):
+                      cyc, comm=None):
     out = {}
     stream = L.stream
     nx, ny, nz = L.gnx, L.gny, L.gnz
@@ -359,6 +359,23 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
     fms = timed(lambda: sf.sf_fcycle(M.handle), 3, warm=1)
     out["fcycle"] = {"ms": fms, "dof_s": dof_local * world / (fms / 1e3),
                      "note": "C4 / HPGMG FOM: one F-cycle (PL up, one V per level) on the workload"}
+    # BASELINE C4: the side^3 problem itself split across the ranks -- strong
+    # scaling of one F-cycle (at N = 1 this is the fcycle line above)
+    if world > 1 and args.side % world == 0 and (args.side // world) % 2 == 0:
+        n = args.side
+        Ls = sf.Level(n, n, n, 1.0 / n, comm=comm)
+        sf.sf_init_problem(Ls.handle, 1, 1.0, 1.0, 1)
+        Ms = sf.MG(Ls, 1.0, 1.0)
+        sms = timed(lambda: sf.sf_fcycle(Ms.handle), 3, warm=1)
+        out["fcycle_strong"] = {"global": [n, n, n], "ms": sms, "dof_s": n**3 / (sms / 1e3),
+                                "note": "C4: one F-cycle of the global problem in z-slabs over "
+                                        "the ranks (strong scaling; max over ranks)"}
+        Ms.close()
+        Ls.close()
+        torch.cuda.empty_cache()
+    else:
+        out["fcycle_strong"] = {"global": [nx, ny, nz], "ms": fms, "dof_s": dof_local * world / (fms / 1e3),
+                                "note": "C4 at N = 1: the fcycle line"}
     # read-dominated bandwidth (PAPER.md:684-696's dot-product bound): L2 norm of u
     # (8 B/cell, read-only); each call ends with an 8-byte D2H and a host sync
     rms = timed(lambda: sf.sf_norm(L.handle, sf.SF_U, sf.SF_NORM_L2), 10, warm=2)
