@@ -7,29 +7,40 @@
 // paper's "multicolor reordering" and OpenCL "tall-skinny blocking" (2-D tiles
 // rolled up through the remaining dimension):
 //
-//   (x,y) tile of 64 x 8 cells, streamed along z by one CTA; step p runs
-//   R(p)    red cells of plane p on the tile AND on a one-cell ring around it
-//           (the ring belongs to neighbouring tiles; recomputing it here,
-//           bit-identically, means the black update needs no other CTA), then
-//   B(p-1)  black cells of plane p-1 on the tile, which read red-new values of
-//           planes p-2, p-1 (incl. ring) and p.
+//   (x,y) tile (32 x 16 cells; 32 x 8 in the two-CTA-per-SM build) streamed
+//   along z by one CTA; step t runs
+//   R(t+1)  red cells of plane t+1 on the tile AND on a one-cell ring around
+//           it (the ring belongs to neighbouring tiles; recomputing it here,
+//           bit-identically, means the black update needs no other CTA), and
+//   B(t-1)  black cells of plane t-1 on the tile, which read red-new values of
+//           planes t-2, t-1 (incl. ring) and t --
+//   two independent dependency chains between consecutive barriers.  The
+//   update is evaluated in lambda-form (below), so alpha is never read.
 //
 // Out of place (xin -> xout): the 2-ring reads of xin must see OLD values
 // whatever neighbouring CTAs have written, so the pair writes a second buffer
 // and the level swaps U <-> TMP.
 //
-// Data movement (Blackwell): every operand plane -- x (tile + 2-ring), alpha,
-// Dinv, rhs, beta_i, beta_j (tile + 1-ring) and beta_k -- arrives by TMA
+// Data movement (Blackwell): every operand plane -- x (tile + 2-ring), Dinv,
+// rhs, beta_i, beta_j (tile + 1-ring) and beta_k -- arrives by TMA
 // (cp.async.bulk.tensor.3d) into shared memory, completion tracked by an
-// mbarrier per plane "bundle", two planes ahead of use (~85 KB in flight per
-// SM).  One elected thread issues; all 8 warps compute from shared memory
-// (16-byte pair loads + warp shuffles for the x-neighbours); the output pair
-// is stored with coalesced 16-byte stores.  Persistent CTAs (one per SM, 190
-// KB smem) walk (tile, z-chunk) items in chunk-major order so neighbouring
-// tiles stream the same planes at the same time (ring/halo reads hit L2).
+// mbarrier per plane "bundle", PF bundles ahead of use (5 in the 32x16 build,
+// ~170 KB in flight per SM).  One elected thread issues; all warps compute
+// from shared memory (16-byte pair loads); the output pair is stored with
+// coalesced 16-byte streaming stores.  Persistent CTAs walk (tile, z-chunk)
+// items in chunk-major order so neighbouring tiles stream the same planes at
+// the same time (ring/halo reads hit L2).
 //
-// Dirichlet BC is folded in: a neighbour across a global face reads -x(c)
-// (PAPER.md:336-341).  Part (slab) interfaces read exchanged halo planes
+// Variants (template flags): RESID reduces the red part of max|rhs - A x| of
+// the input, BRES the black part of the output's (the split convergence check,
+// mg.cu), INTERP applies x_in += P0(e_coarse) to each x plane in shared memory
+// one step before its first read (A8 of the V-cycle fused into the first
+// post-smoothing pair).  Launches can be restricted to the interior or the
+// boundary z-chunks of a part (halo exchange overlapped, comm.cu).
+//
+// Dirichlet BC is folded in: a neighbour across a global face contributes 0 to
+// the lambda-form sum (its -x(c) ghost term is part of the diagonal,
+// PAPER.md:336-341).  Part (slab) interfaces read exchanged halo planes
 // (x depth 2, coefficients depth 2, rhs depth 1).
 #include <cuda.h>
 #include <cudaTypedefs.h>
@@ -40,11 +51,11 @@
 
 namespace {
 
-// Tile = 512 cells handled by 8 warps, one red/black pair per thread.  32x16
-// (default) carries ~22% less halo per cell than 64x8 and 48 instead of 72
-// redundant ring cells; its smaller bundle leaves room for 4-deep prefetch.
-// Compiled twice by build.py: 32x16 with 4-deep prefetch (suffix _t32) and
-// 64x8 with 3-deep prefetch (_t64, used when ny % 16 != 0).
+// One red/black pair per thread.  32x16 (8 warps) carries ~22% less halo per
+// cell than 64x8 and 48 instead of 72 redundant ring cells.  Compiled three
+// times by build.py: 32x16 with 5-deep prefetch (_t32), 64x8 with 4-deep
+// (_t64, when ny % 16 != 0) and 32x8 / 4 warps / 3-deep with two CTAs per SM
+// (_t32w4, levels up to 256^3).
 #ifndef SF_GSRB_TX
 #define SF_GSRB_TX 32
 #endif
