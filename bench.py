@@ -122,24 +122,46 @@ def ncu_traffic():
 
 
 # ------------------------------------------------------------------ oracle (cpu)
-def oracle_vcycle_sample(shape, reps=1):
-    """Time the CPU oracle's V-cycle on the same HPGMG-shaped workload.
-    Returns (seconds per V-cycle, cores used, description)."""
-    from oracle import oracle as O
-    from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
-    nx, ny, nz = shape
-    h = I.level_h(nx, ny, nz)
-    coeffs = I.hpgmg_coeffs(nx, ny, nz, h)
-    _, f = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
-    mg = O.MG(nx, ny, nz, h, 1.0, 1.0, *coeffs)
-    del coeffs
-    u = __import__("numpy").zeros(f.shape)
-    ts = []
-    for _ in range(reps):
+def oracle_threads():
+    """Host cores this process may use (the oracle's OpenMP build runs on all)."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+class OracleSampler:
+    """The CPU oracle's V-cycle on the same HPGMG-shaped workload, with its
+    OpenMP build on all host cores (the plane loops of oracle.c; same
+    arithmetic as the single-thread build, which the parity tests use)."""
+
+    def __init__(self, shape):
+        from oracle import oracle as O
+        from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
+        import numpy as np
+        O.use_openmp(True)
+        self.cores = O.lib().or_set_threads(oracle_threads())   # the threads it actually runs
+        nx, ny, nz = shape
+        h = I.level_h(nx, ny, nz)
+        coeffs = I.hpgmg_coeffs(nx, ny, nz, h)
+        _, self.f = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
+        self.mg = O.MG(nx, ny, nz, h, 1.0, 1.0, *coeffs)
+        del coeffs
+        self.u = np.zeros(self.f.shape)
+        self.desc = (f"oracle V-cycle (2+2 GSRB pairs, P0, exact bottom) on {nx}x{ny}x{nz}, "
+                     f"OpenMP build on {self.cores} host cores")
+
+    def vcycle_seconds(self):
         t0 = time.perf_counter()
-        u = mg.vcycle(u, f)
-        ts.append(time.perf_counter() - t0)
-    return min(ts), 1, f"oracle V-cycle (2+2 GSRB pairs, P0, exact bottom) on {nx}x{ny}x{nz}"
+        self.u = self.mg.vcycle(self.u, self.f)
+        return time.perf_counter() - t0
+
+
+def oracle_vcycle_sample(shape, reps=1):
+    """(seconds per V-cycle (min of reps), cores used, description)."""
+    s = OracleSampler(shape)
+    t = min(s.vcycle_seconds() for _ in range(reps))
+    return t, s.cores, s.desc
 
 
 def oracle_shape(shape):
@@ -161,9 +183,11 @@ def run_reference(args):
         return
     nx, ny, nz = dims_for(args.side, 1)
     shp, scale = oracle_shape((nx, ny, nz))
+    smp = OracleSampler(shp)
+    cores, desc = smp.cores, smp.desc
     steps = []
     for s in range(args.warmup + args.steps):
-        t, cores, desc = oracle_vcycle_sample(shp)
+        t = smp.vcycle_seconds()
         if s >= args.warmup:
             steps.append(t * scale)
     tv = sum(steps) / len(steps)
@@ -530,7 +554,7 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
         G.close()
         if world == 1 and not args.no_cpu_baseline:
             shp, scale = oracle_shape((nx, ny, nz))
-            tv, cores, desc = oracle_vcycle_sample(shp)
+            tv, cores, desc = oracle_vcycle_sample(shp, reps=2)
             tv *= scale
             t_solve = tv * (F_OVER_V + (cyc - 1))
             out["cpu_baseline"] = {

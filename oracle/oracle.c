@@ -9,7 +9,12 @@
  * constant with the CUDA path.
  *
  * Built with  gcc -O2 -ffp-contract=off  (no FMA contraction), IEEE fp64,
- * single thread.  Triple loops, one ghost layer, separate arrays.
+ * single thread.  Triple loops, one ghost layer, separate arrays.  The
+ * "omp parallel for" pragmas over the outer plane loop are inert in that
+ * build; bench.py's cpu_baseline / --impl reference legs time a second build
+ * with -fopenmp on the host's cores: every
+ * parallel loop writes disjoint cells (colour sweeps are order-independent),
+ * so only the L2 norm's summation order differs between the two builds.
  *
  * Citations are PAPER.md line numbers (/root/reference/PAPER.md, text of the
  * paper) plus the DESIGN.md reading (R-n) where the paper is silent.
@@ -26,6 +31,9 @@
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 typedef struct {
     int nx, ny, nz;
@@ -36,6 +44,17 @@ typedef struct {
 #define SY(g) ((size_t)(g)->ny + 2)
 #define OIDX(g, i, j, k) \
     ((((size_t)((k) + 1)) * SY(g) + (size_t)((j) + 1)) * SX(g) + (size_t)((i) + 1))
+
+/* threads of the timing build (1 in the single-thread build) */
+int or_set_threads(int n) {
+#ifdef _OPENMP
+    if (n > 0) omp_set_num_threads(n);
+    return omp_get_max_threads();
+#else
+    (void)n;
+    return 1;
+#endif
+}
 
 size_t or_size(int nx, int ny, int nz) {
     return ((size_t)nx + 2) * ((size_t)ny + 2) * ((size_t)nz + 2);
@@ -50,6 +69,7 @@ size_t or_size(int nx, int ny, int nz) {
 /* outside of, i.e. value = (-1)^m * x(mirror).                              */
 /* ------------------------------------------------------------------------ */
 void or_apply_bc(const or_grid* g, double* x) {
+#pragma omp parallel for schedule(static)
     for (int k = -1; k <= g->nz; k++)
         for (int j = -1; j <= g->ny; j++)
             for (int i = -1; i <= g->nx; i++) {
@@ -94,6 +114,7 @@ void or_apply_op(const or_grid* g, double a, double b, const double* alpha,
                  const double* bi, const double* bj, const double* bk,
                  double* x, double* out) {
     or_apply_bc(g, x);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++)
@@ -105,6 +126,7 @@ void or_residual(const or_grid* g, double a, double b, const double* alpha,
                  const double* bi, const double* bj, const double* bk,
                  double* x, const double* rhs, double* res) {
     or_apply_bc(g, x);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++)
@@ -121,6 +143,7 @@ void or_residual(const or_grid* g, double a, double b, const double* alpha,
 void or_dinv(const or_grid* g, double a, double b, const double* alpha,
              const double* bi, const double* bj, const double* bk, double* dinv) {
     double hm2 = 1.0 / (g->h * g->h);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) {
@@ -149,6 +172,7 @@ void or_gsrb_sweep(const or_grid* g, double a, double b, const double* alpha,
                    const double* bi, const double* bj, const double* bk,
                    const double* dinv, double* x, const double* rhs, int colour) {
     or_apply_bc(g, x);                                   /* "boundary" stencils */
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) {
@@ -176,6 +200,7 @@ void or_smooth(const or_grid* g, double a, double b, const double* alpha,
 /* ------------------------------------------------------------------------ */
 void or_restrict_cell(const or_grid* gc, double* coarse, const or_grid* gf,
                       const double* fine) {
+#pragma omp parallel for schedule(static)
     for (int K = 0; K < gc->nz; K++)
         for (int J = 0; J < gc->ny; J++)
             for (int I = 0; I < gc->nx; I++) {
@@ -192,6 +217,7 @@ void or_restrict_cell(const or_grid* gc, double* coarse, const or_grid* gf,
 void or_restrict_face(const or_grid* gc, double* coarse, const or_grid* gf,
                       const double* fine, int dir) {
     int ex = dir == 0, ey = dir == 1, ez = dir == 2;
+#pragma omp parallel for schedule(static)
     for (int K = 0; K < gc->nz + ez; K++)
         for (int J = 0; J < gc->ny + ey; J++)
             for (int I = 0; I < gc->nx + ex; I++) {
@@ -215,6 +241,7 @@ void or_restrict_face(const or_grid* gc, double* coarse, const or_grid* gf,
 /* ------------------------------------------------------------------------ */
 void or_interp_p0(const or_grid* gf, double* fine, double prescale,
                   const or_grid* gc, const double* coarse) {
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < gf->nz; k++)
         for (int j = 0; j < gf->ny; j++)
             for (int i = 0; i < gf->nx; i++) {
@@ -230,6 +257,7 @@ void or_interp_p0(const or_grid* gf, double* fine, double prescale,
 void or_interp_pl(const or_grid* gf, double* fine, double prescale,
                   const or_grid* gc, double* coarse) {
     or_apply_bc(gc, coarse);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < gf->nz; k++)
         for (int j = 0; j < gf->ny; j++)
             for (int i = 0; i < gf->nx; i++) {
@@ -252,6 +280,7 @@ void or_interp_pl(const or_grid* gf, double* fine, double prescale,
 /* A10: norms over the interior */
 double or_norm_max(const or_grid* g, const double* x) {
     double m = 0.0;
+#pragma omp parallel for reduction(max : m) schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) {
@@ -263,6 +292,7 @@ double or_norm_max(const or_grid* g, const double* x) {
 
 double or_norm_l2(const or_grid* g, const double* x) {
     double s = 0.0;
+#pragma omp parallel for reduction(+ : s) schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) {
@@ -594,6 +624,7 @@ static double lap_at(const or_grid* g, const double* x, int i, int j, int k) {
 
 void or_laplacian_cc(const or_grid* g, double* x, double* out) {
     or_apply_bc(g, x);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) out[OIDX(g, i, j, k)] = lap_at(g, x, i, j, k);
@@ -602,6 +633,7 @@ void or_laplacian_cc(const or_grid* g, double* x, double* out) {
 void or_jacobi_cc(const or_grid* g, double omega, double* x, const double* f, double* out) {
     double hm2 = 1.0 / (g->h * g->h);
     or_apply_bc(g, x);
+#pragma omp parallel for schedule(static)
     for (int k = 0; k < g->nz; k++)
         for (int j = 0; j < g->ny; j++)
             for (int i = 0; i < g->nx; i++) {

@@ -22,16 +22,32 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
 GCC_FLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-std=c99"]
+# The pins and every parity test use the single-thread build.  The -fopenmp
+# build (same source: the plane loops' "omp parallel for" pragmas become live)
+# is only for timing the oracle on all host cores (bench.py's cpu_baseline and
+# --impl reference legs); select it with use_openmp() before the first call.
+_use_omp = False
 
 
-def build(force=False):
-    """Compile liboracle.so with gcc (plain C, no contraction)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *GCC_FLAGS, "-o", tmp, _SRC, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+def use_openmp(on=True):
+    global _use_omp
+    if _lib is not None and on != _use_omp:
+        raise RuntimeError("oracle library already loaded with the other build")
+    _use_omp = on
+
+
+def build(force=False, omp=None):
+    """Compile liboracle.so (and liboracle_omp.so) with gcc (plain C, no contraction)."""
+    omp = _use_omp if omp is None else omp
+    out = _LIB_OMP if omp else _LIB
+    if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(_SRC):
+        tmp = out + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *GCC_FLAGS, *(["-fopenmp"] if omp else []), "-o", tmp, _SRC,
+                               "-lm"])
+        os.replace(tmp, out)
+    return out
 
 
 _lib = None
@@ -50,6 +66,7 @@ def lib():
         G = C.POINTER(_Grid)
         d = C.c_double
         sig = {
+            "or_set_threads": (C.c_int, [C.c_int]),
             "or_apply_bc": (None, [G, _P]),
             "or_apply_op": (None, [G, d, d, _P, _P, _P, _P, _P, _P]),
             "or_residual": (None, [G, d, d, _P, _P, _P, _P, _P, _P, _P]),
