@@ -15,6 +15,9 @@
 //
 // The operator is evaluated in exactly the term order of op_at (kernels.cu)
 // and the oracle; the Dirichlet fold reads -x(c) across global faces.
+#include <algorithm>
+#include <cstdlib>
+
 #include "sf_internal.h"
 
 namespace {
@@ -125,6 +128,101 @@ __global__ void __launch_bounds__(PX* PY) residual_restrict_kernel(PV f, const d
                 s += r.y - axb;
             }
         cx[sf_ix(c, I, J, K + zoff)] = s / 8.0;
+    }
+}
+
+// A x at the pair of row j from operands already in registers (op_pair's term
+// order and roundings; xs/xn/xb/xt carry the row's y/z neighbours, BC folded by
+// the caller's flags).
+__device__ __forceinline__ void op_pair_r(const PV& v, const double* __restrict__ x, int i, long c,
+                                          double2 xc, double2 xs, double2 xn, double2 xb,
+                                          double2 xt, double2 bjs, double2 bjn, double2 bkb,
+                                          double2 bkt, double a, double bh2, double& axa,
+                                          double& axb) {
+    const double xw = (i == 0) ? -xc.x : x[c - 1];
+    const double xe = (i + 1 == v.nx - 1) ? -xc.y : x[c + 2];
+    const double2 bi = ld2(v.f[SF_BETA_I] + c);
+    const double bie = v.f[SF_BETA_I][c + 2];
+    const double2 al = ld2(v.f[SF_ALPHA] + c);
+    double fa = bi.y * (xc.y - xc.x);
+    fa += bi.x * (xw - xc.x);
+    fa += bjn.x * (xn.x - xc.x);
+    fa += bjs.x * (xs.x - xc.x);
+    fa += bkt.x * (xt.x - xc.x);
+    fa += bkb.x * (xb.x - xc.x);
+    double fb = bie * (xe - xc.y);
+    fb += bi.y * (xc.x - xc.y);
+    fb += bjn.y * (xn.y - xc.y);
+    fb += bjs.y * (xs.y - xc.y);
+    fb += bkt.y * (xt.y - xc.y);
+    fb += bkb.y * (xb.y - xc.y);
+    axa = a * al.x * xc.x - bh2 * fa;
+    axb = a * al.y * xc.y - bh2 * fb;
+}
+
+__device__ __forceinline__ double2 neg2(double2 u) { return make_double2(-u.x, -u.y); }
+
+// residual_restrict, persistent and z-streamed: items = (32x4 coarse columns
+// tile, chunk of `depth` coarse planes), walked by an occupancy-sized grid; a
+// thread keeps the x planes 2K-1 .. 2K+2 and beta_k planes 2K .. 2K+2 of its
+// 2x2 fine columns in registers, so each coarse step loads two new x planes
+// and two beta_k planes (42 loads per 8 fine cells instead of 60).  Same
+// arithmetic, term order and roundings as residual_restrict_kernel.
+template <int MINB>
+__global__ void __launch_bounds__(PX* PY, MINB) residual_restrict_zs_kernel(
+    PV f, const double* __restrict__ x, const double* __restrict__ rhs, double a, double bh2, PV c,
+    double* __restrict__ cx, int zoff, int depth, int tgx, int ntiles, int nitems) {
+    const int nK = f.nz / 2;
+    const double* bj = f.f[SF_BETA_J];
+    const double* bk = f.f[SF_BETA_K];
+    for (int item = blockIdx.x; item < nitems; item += gridDim.x) {
+        const int ch = item / ntiles, tile = item - ch * ntiles;
+        const int I = (tile % tgx) * PX + threadIdx.x, J = (tile / tgx) * PY + threadIdx.y;
+        if (2 * I >= f.nx || 2 * J >= f.ny) continue;
+        const int K0 = ch * depth, K1 = min(K0 + depth, nK);
+        const int i = 2 * I, j0 = 2 * J, j1 = j0 + 1;
+        const long js = f.js, ks = f.ks;
+        long q0 = sf_ix(f, i, j0, 2 * K0);   // row j0 of plane 2K
+        // carried: x(2K-1), x(2K) and beta_k(2K) of rows j0, j1
+        double2 xa0 = ld2(x + q0 - ks), xa1 = ld2(x + q0 - ks + js);
+        double2 xb0 = ld2(x + q0), xb1 = ld2(x + q0 + js);
+        double2 k00 = ld2(bk + q0), k01 = ld2(bk + q0 + js);
+        for (int K = K0; K < K1; K++, q0 += 2 * ks) {
+            const long q1 = q0 + ks;   // plane 2K+1
+            const double2 xc0 = ld2(x + q1), xc1 = ld2(x + q1 + js);
+            const double2 xd0 = ld2(x + q1 + ks), xd1 = ld2(x + q1 + ks + js);
+            const double2 k10 = ld2(bk + q1), k11 = ld2(bk + q1 + js);
+            const double2 k20 = ld2(bk + q1 + ks), k21 = ld2(bk + q1 + ks + js);
+            double s = 0.0;
+#pragma unroll
+            for (int d = 0; d < 2; d++) {
+                const long q = d ? q1 : q0;
+                const int gk = f.z0 + 2 * K + d;
+                const double2 c0 = d ? xc0 : xb0, c1 = d ? xc1 : xb1;
+                double2 b0 = d ? xb0 : xa0, b1 = d ? xb1 : xa1;
+                double2 t0 = d ? xd0 : xc0, t1 = d ? xd1 : xc1;
+                const double2 kb0 = d ? k10 : k00, kb1 = d ? k11 : k01;
+                const double2 kt0 = d ? k20 : k10, kt1 = d ? k21 : k11;
+                if (gk == 0) { b0 = neg2(c0); b1 = neg2(c1); }
+                if (gk == f.gnz - 1) { t0 = neg2(c0); t1 = neg2(c1); }
+                double2 ys = ld2(x + q - js), yn = ld2(x + q + 2 * js);
+                if (j0 == 0) ys = neg2(c0);
+                if (j1 == f.ny - 1) yn = neg2(c1);
+                const double2 bj0 = ld2(bj + q), bj1 = ld2(bj + q + js), bj2 = ld2(bj + q + 2 * js);
+                double axa, axb;
+                // row j0: north neighbour row j1 (an interior row: j0 + 1 < ny)
+                op_pair_r(f, x, i, q, c0, ys, c1, b0, t0, bj0, bj1, kb0, kt0, a, bh2, axa, axb);
+                double2 r = ld2(rhs + q);
+                s += r.x - axa;
+                s += r.y - axb;
+                op_pair_r(f, x, i, q + js, c1, c0, yn, b1, t1, bj1, bj2, kb1, kt1, a, bh2, axa, axb);
+                r = ld2(rhs + q + js);
+                s += r.x - axa;
+                s += r.y - axb;
+            }
+            cx[sf_ix(c, I, J, K + zoff)] = s / 8.0;
+            xa0 = xc0; xa1 = xc1; xb0 = xd0; xb1 = xd1; k00 = k20; k01 = k21;
+        }
     }
 }
 
@@ -335,6 +433,30 @@ inline dim3 pair_grid(int nx, int ny, int nz, int* depth) {
     return dim3(gx, gy, zc);
 }
 
+// SF_RR_ZS = 0 selects the one-pass-per-launch residual_restrict (A/B runs)
+int rr_zs() {
+    static const int v = getenv("SF_RR_ZS") ? atoi(getenv("SF_RR_ZS")) : 1;
+    return v;
+}
+
+// resident CTAs of the z-streamed residual_restrict on this device
+int rr_zs_resident() {
+    static int g = 0;
+    if (!g) {
+        int dev = 0, sms = 148, per = 1;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (rr_zs() == 2)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, residual_restrict_zs_kernel<6>, PX * PY, 0);
+        else if (rr_zs() == 3)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, residual_restrict_zs_kernel<8>, PX * PY, 0);
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, residual_restrict_zs_kernel<4>, PX * PY, 0);
+        g = sms * std::max(per, 1);
+    }
+    return g;
+}
+
 }  // namespace
 
 bool pair_ok(const sf_level* L) { return L->nx % 2 == 0; }
@@ -369,11 +491,33 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
     for (int p = 0; p < F->nlocal; p++) {
         PV f = sf_view(F, p);
         PV c = sf_view(C, rep ? 0 : p);
-        int depth;
-        dim3 g = pair_grid(f.nx, f.ny / 2, f.nz / 2, &depth);  // thread per coarse (I,J)
-        residual_restrict_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[x], f.f[rhs], a, bh2, c,
-                                                                    c.f[cf], rep ? f.z0 / 2 : 0,
-                                                                    depth);
+        if (rr_zs()) {
+            // persistent z-streamed kernel: chunk depth D minimising rounds * (D + 1)
+            // (one plane of prologue) over the resident CTAs
+            const int tgx = (f.nx / 2 + PX - 1) / PX, tgy = (f.ny / 2 + PY - 1) / PY;
+            const int tiles = tgx * tgy, nK = f.nz / 2, G = rr_zs_resident();
+            int best_d = nK;
+            double best = 1e30;
+            for (int d = nK; d >= 1; d--) {
+                const long items = (long)tiles * ((nK + d - 1) / d);
+                const double cost = (double)((items + G - 1) / G) * (d + 1.0);
+                if (cost < best - 1e-9) { best = cost; best_d = d; }
+            }
+            const int items = tiles * ((nK + best_d - 1) / best_d);
+#define SF_RRZS(MB)                                                                              \
+    residual_restrict_zs_kernel<MB><<<std::min(items, G), dim3(PX, PY), 0, F->stream>>>(          \
+        f, f.f[x], f.f[rhs], a, bh2, c, c.f[cf], rep ? f.z0 / 2 : 0, best_d, tgx, tiles, items)
+            if (rr_zs() == 2) SF_RRZS(6);
+            else if (rr_zs() == 3) SF_RRZS(8);
+            else SF_RRZS(4);
+#undef SF_RRZS
+        } else {
+            int depth;
+            dim3 g = pair_grid(f.nx, f.ny / 2, f.nz / 2, &depth);  // thread per coarse (I,J)
+            residual_restrict_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[x], f.f[rhs], a, bh2,
+                                                                        c, c.f[cf],
+                                                                        rep ? f.z0 / 2 : 0, depth);
+        }
         SF_LAUNCHED();
     }
     SF_TRY(sf_check_launch("residual_restrict"));

@@ -392,6 +392,8 @@ extern "C" sf_status sf_smooth_residual_restrict(sf_level* F, int x, int rhs, do
         return SF_OK;
     }
     SF_TRY(sf_smooth_gsrb(F, x, rhs, a, b, 1, SF_SMOOTH_AUTO));
+    if (pair_ok(F))   // residual never stored (A6 + A7, 49 B/cell)
+        return k_residual_restrict(F, x, rhs, a, b, C, cf);
     SF_TRY(k_residual(F, SF_R, x, rhs, a, b));
     return k_restrict(C, cf, F, SF_R, SF_RESTRICT_CELL);
 }
