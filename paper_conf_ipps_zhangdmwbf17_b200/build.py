@@ -26,7 +26,7 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            ("gsrb_fused.cu", "gsrb_fused_t64.o",
             ["-DSF_GSRB_TX=64", "-DSF_GSRB_PF=4", "-DSF_GSRB_SUFFIX=_t64"]),
            ("gsrb_fused.cu", "gsrb_fused_t32w4.o",
-            ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=3", "-DSF_GSRB_NWARP=4", "-DSF_GSRB_MINB=2",
+            ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=2", "-DSF_GSRB_NWARP=4", "-DSF_GSRB_MINB=3",
              "-DSF_GSRB_SUFFIX=_t32w4"]),
            ("gsrb_rr.cu", "gsrb_rr.o", []),
            ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []),

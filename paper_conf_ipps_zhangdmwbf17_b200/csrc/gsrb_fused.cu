@@ -54,8 +54,10 @@ namespace {
 // One red/black pair per thread.  32x16 (8 warps) carries ~22% less halo per
 // cell than 64x8 and 48 instead of 72 redundant ring cells.  Compiled three
 // times by build.py: 32x16 with 5-deep prefetch (_t32), 64x8 with 4-deep
-// (_t64, when ny % 16 != 0) and 32x8 / 4 warps / 3-deep with two CTAs per SM
-// (_t32w4, levels up to 256^3).
+// (_t64, when ny % 16 != 0) and 32x8 / 4 warps / 2-deep with three CTAs per
+// SM (_t32w4, levels up to 256^3: three independent z-step chains per SM hide
+// each other's per-item pipeline fill; 6 % faster than two CTAs with 3-deep
+// prefetch at 256^3, profiles/r01/ab_256_ctas_per_sm.txt).
 #ifndef SF_GSRB_TX
 #define SF_GSRB_TX 32
 #endif

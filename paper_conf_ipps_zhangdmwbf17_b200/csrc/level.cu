@@ -404,9 +404,9 @@ bool gsrb_fused_supported(const sf_level* L) {
 
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
                             double* rmax, sf_level* C, int cf, int phase, int reserve, int rmode) {
-    // 32x8 tiles with two CTAs per SM measured 1.5-2 % faster up to 256^3 and
-    // 1.7 % slower at 512^3 than 32x16 with one (profiles/r01/ncu_variants_ab.txt);
-    // SF_GSRB_W4 = 0 / 1 forces the choice
+    // 32x8 tiles with three CTAs per SM: 7.5 % faster than 32x16 with one at
+    // 256^3 and equal at 512^3 (profiles/r01/ab_256_ctas_per_sm.txt,
+    // ab_w4_512.txt); SF_GSRB_W4 = 0 / 1 forces the choice
     static const int w4 = getenv("SF_GSRB_W4") ? atoi(getenv("SF_GSRB_W4")) : -1;
     const bool small = (long)L->nx * L->ny * L->lnz <= (1L << 24);
     if ((w4 == 1 || (w4 < 0 && small)) && gsrb_fused_supported_t32w4(L))

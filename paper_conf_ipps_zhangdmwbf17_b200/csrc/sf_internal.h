@@ -150,7 +150,7 @@ sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double 
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
                                 int rmode = 0);
-// 32x8 tiles, 4 warps, 2 CTAs per SM (two independent z-step chains per SM)
+// 32x8 tiles, 4 warps, 3 CTAs per SM (three independent z-step chains per SM)
 bool gsrb_fused_supported_t32w4(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32w4(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                   double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
