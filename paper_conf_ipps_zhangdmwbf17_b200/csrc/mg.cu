@@ -13,6 +13,22 @@
 
 #include "sf_internal.h"
 
+// Device-resident solve loop (sf_solve with graphs): termination is decided on
+// the device and drives a CUDA-graph WHILE node, so a whole solve is one graph
+// launch and one host synchronisation.
+#define SF_LOOP_HIST 256
+struct LoopCtl {    // device memory
+    double fn, rtol;
+    int max_cycles, done, status, nbody;
+    double hist[SF_LOOP_HIST];
+};
+struct LoopHost {   // mapped pinned memory: rtol / max_cycles in, results out
+    double rtol;
+    int max_cycles, done, status, nbody;
+    double hist[SF_LOOP_HIST];
+};
+enum { LS_RUN = 0, LS_CONVERGED = 1, LS_NUMERIC = 2, LS_NOT_CONVERGED = 3, LS_ZERO = 4, LS_RHS_NAN = 5 };
+
 struct sf_mg {
     std::vector<sf_level*> lv;
     std::vector<bool> own;
@@ -22,6 +38,12 @@ struct sf_mg {
     cudaGraphExec_t gexec[5] = {};  // V+check, F+check, F, first pair+check, rest of V
     long long gnodes[5] = {};
     bool graph_failed = false;
+    cudaGraphExec_t gloop[2] = {};  // device-resident solve, V-only / F first
+    long long loop_nodes[2][2] = {};   // launches in prologue+epilogue / in one loop body
+    bool loop_failed = false;
+    LoopCtl* lctl = nullptr;
+    LoopHost* lhost = nullptr;
+    LoopHost* lhost_dev = nullptr;
     std::vector<double> lmax;   // SF_SMOOTH_CHEBY: lambda_max(D^-1 A) per level
 };
 
@@ -59,6 +81,10 @@ extern "C" sf_status sf_mg_destroy(sf_mg* m) {
     if (!m->lv.empty()) cudaStreamSynchronize(m->lv[0]->stream);
     for (auto& g : m->gexec)
         if (g) cudaGraphExecDestroy(g);
+    for (auto& g : m->gloop)
+        if (g) cudaGraphExecDestroy(g);
+    if (m->lctl) cudaFree(m->lctl);
+    if (m->lhost) cudaFreeHost(m->lhost);
     if (m->ainv) cudaFree(m->ainv);
     destroy_levels(m);
     delete m;
@@ -434,6 +460,227 @@ static sf_status run(sf_mg* m, int kind) {
     return body_of(m, kind);
 }
 
+// ---------------------------------------------------------------- device loop
+static __global__ void loop_init_kernel(LoopCtl* c, const LoopHost* h, const double* fn, int done0) {
+    c->rtol = h->rtol;
+    c->max_cycles = h->max_cycles;
+    c->fn = *fn;
+    c->done = done0;
+    c->status = LS_RUN;
+    c->nbody = 0;
+}
+
+// After a first pair's fused check: rmax = max|F - A U| of the iterate after
+// `done` cycles (the same decision as sf_solve's host loop, made on the device).
+static __global__ void loop_check_kernel(LoopCtl* c, const double* rmax, cudaGraphConditionalHandle h) {
+    const int d = c->done;
+    unsigned cont = 1;
+    const double fn = c->fn;
+    if (!(fn == fn) || isinf(fn)) {
+        c->status = LS_RHS_NAN;
+        cont = 0;
+    } else if (fn == 0.0) {
+        c->status = LS_ZERO;
+        cont = 0;
+    } else if (d >= 1) {
+        const double rel = *rmax / fn;
+        if (d <= SF_LOOP_HIST) c->hist[d - 1] = rel;
+        if (!(rel == rel) || isinf(rel)) {
+            c->status = LS_NUMERIC;
+            cont = 0;
+        } else if (rel < c->rtol) {
+            c->status = LS_CONVERGED;
+            cont = 0;
+        } else if (d >= c->max_cycles) {
+            c->status = LS_NOT_CONVERGED;
+            cont = 0;
+        }
+    }
+    if (cont) {   // the loop body completes cycle d + 1
+        c->done = d + 1;
+        c->nbody++;
+    }
+    cudaGraphSetConditional(h, cont);
+}
+
+// results -> mapped host memory (posted writes: nothing queues behind bulk copies)
+static __global__ void loop_publish_kernel(const LoopCtl* c, LoopHost* h) {
+    const int n = min(c->done, SF_LOOP_HIST);
+    for (int i = threadIdx.x; i < n; i += blockDim.x) h->hist[i] = c->hist[i];
+    if (threadIdx.x == 0) {
+        h->done = c->done;
+        h->status = c->status;
+        h->nbody = c->nbody;
+    }
+}
+
+static sf_status first_pair(sf_mg* m) {   // first_pair_check without the host copy
+    sf_level* L = m->lv[0];
+    SF_TRY(sf_halo(L, SF_F, 1));
+    SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch, nullptr, 0,
+                            SF_RM_INPUT_RED));
+    sf_swap_fields(L, SF_U, SF_TMP);
+    if (L->comm && L->comm->kind != 0 && L->nparts > 1)
+        SF_TRY(sf_allreduce_scalar(L, L->comm, L->dscratch, 0));
+    return SF_OK;
+}
+
+static bool loop_allowed(const sf_mg* m) {
+    return !m->loop_failed && graphs_allowed(m) && fused_check_ok(m) &&
+           !(m->lv[0]->comm && m->lv[0]->comm->kind == 1);   // NCCL: host-side proxies
+}
+
+// Build the solve graph:
+//   [max|F| -> fn] [init] [F-cycle]? [first pair + check] WHILE(cont) { [rest of the
+//   V-cycle] [first pair of the next + check] } [publish]
+// The loop body holds 4 U/TMP swaps on the finest level (even on every level),
+// so every iteration reads the buffers the capture saw; the iterate a stop
+// leaves behind is the input of the last first pair, i.e. the buffer U named
+// before the solve.  Any failure leaves the device loop off for this hierarchy.
+static sf_status build_loop(sf_mg* m, int fc) {
+    sf_level* L = m->lv[0];
+    cudaStream_t st = L->stream;
+    std::vector<std::vector<SfPart>> saved;
+    for (sf_level* lv : m->lv) saved.push_back(lv->parts);
+    long long c0, c1, c2, c3;
+    cudaGraph_t g = nullptr;
+    cudaGraphExec_t ge = nullptr;
+    bool ok = true;
+    auto fail = [&]() {
+        cudaStreamCaptureStatus cs;
+        if (cudaStreamIsCapturing(st, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
+            cudaGraph_t junk = nullptr;
+            cudaStreamEndCapture(st, &junk);
+            if (junk && junk != g) cudaGraphDestroy(junk);
+        }
+        cudaGetLastError();
+        ok = false;
+    };
+    if (!m->lctl) {
+        if (cudaMalloc(&m->lctl, sizeof(LoopCtl)) != cudaSuccess ||
+            cudaHostAlloc(&m->lhost, sizeof(LoopHost), cudaHostAllocMapped) != cudaSuccess ||
+            cudaHostGetDevicePointer(&m->lhost_dev, m->lhost, 0) != cudaSuccess) {
+            cudaGetLastError();
+            m->loop_failed = true;
+            return SF_OK;
+        }
+    }
+    sf_launch_count(&c0, 0);
+    cudaGraphConditionalHandle h = 0;
+    cudaGraphNode_t last = nullptr, wnode = nullptr;
+    if (cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) != cudaSuccess) fail();
+    if (ok && sf_norm_async(L, SF_F, SF_NORM_MAX, L->dscratch + 2) != SF_OK) fail();
+    if (ok) {
+        loop_init_kernel<<<1, 1, 0, st>>>(m->lctl, m->lhost_dev, L->dscratch + 2, fc ? 1 : 0);
+        SF_LAUNCHED();
+    }
+    if (ok && fc && fcyc(m) != SF_OK) fail();
+    if (ok && first_pair(m) != SF_OK) fail();
+    if (ok) {
+        cudaStreamCaptureStatus cs;
+        cudaGraph_t cg = nullptr;
+        if (cudaStreamGetCaptureInfo(st, &cs, nullptr, &cg, nullptr, nullptr) != cudaSuccess ||
+            cs != cudaStreamCaptureStatusActive ||
+            cudaGraphConditionalHandleCreate(&h, cg, 0, cudaGraphCondAssignDefault) != cudaSuccess)
+            fail();
+    }
+    if (ok) {
+        loop_check_kernel<<<1, 1, 0, st>>>(m->lctl, L->dscratch, h);
+        SF_LAUNCHED();
+        cudaStreamCaptureStatus cs;
+        const cudaGraphNode_t* deps = nullptr;
+        size_t nd = 0;
+        if (cudaStreamGetCaptureInfo(st, &cs, nullptr, nullptr, &deps, &nd) != cudaSuccess || nd != 1)
+            fail();
+        else
+            last = deps[0];
+    }
+    if (ok && cudaStreamEndCapture(st, &g) != cudaSuccess) fail();
+    sf_launch_count(&c1, 0);
+    cudaGraph_t body = nullptr;
+    if (ok) {
+        cudaGraphNodeParams p = {};
+        p.type = cudaGraphNodeTypeConditional;
+        p.conditional.handle = h;
+        p.conditional.type = cudaGraphCondTypeWhile;
+        p.conditional.size = 1;
+        if (cudaGraphAddNode(&wnode, g, &last, 1, &p) != cudaSuccess) fail();
+        else body = p.conditional.phGraph_out[0];
+    }
+    if (ok && cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0,
+                                            cudaStreamCaptureModeThreadLocal) != cudaSuccess)
+        fail();
+    if (ok && vcyc(m, 0, true) != SF_OK) fail();
+    if (ok && first_pair(m) != SF_OK) fail();
+    if (ok) {
+        loop_check_kernel<<<1, 1, 0, st>>>(m->lctl, L->dscratch, h);
+        SF_LAUNCHED();
+        cudaGraph_t bo = nullptr;
+        if (cudaStreamEndCapture(st, &bo) != cudaSuccess) fail();
+    }
+    sf_launch_count(&c2, 0);
+    if (ok && cudaStreamBeginCaptureToGraph(st, g, &wnode, nullptr, 1,
+                                            cudaStreamCaptureModeThreadLocal) != cudaSuccess)
+        fail();
+    if (ok) {
+        loop_publish_kernel<<<1, 32, 0, st>>>(m->lctl, m->lhost_dev);
+        SF_LAUNCHED();
+        cudaGraph_t go = nullptr;
+        if (cudaStreamEndCapture(st, &go) != cudaSuccess) fail();
+    }
+    sf_launch_count(&c3, 0);
+    sf_count_launch(-(c3 - c0));   // captured, not launched
+    for (size_t i = 0; i < m->lv.size(); i++) m->lv[i]->parts = saved[i];
+    if (ok && cudaGraphInstantiate(&ge, g, 0) != cudaSuccess) fail();
+    if (g) cudaGraphDestroy(g);
+    if (!ok) {
+        if (ge) cudaGraphExecDestroy(ge);
+        m->loop_failed = true;
+        return SF_OK;
+    }
+    m->gloop[fc] = ge;
+    m->loop_nodes[fc][0] = (c1 - c0) + (c3 - c2);
+    m->loop_nodes[fc][1] = c2 - c1;
+    return SF_OK;
+}
+
+// One solve through the device loop.  *handled = false: not available, use the
+// host loop.
+static sf_status solve_loop(sf_mg* m, int fc, double rtol, int max_cycles, int* cycles,
+                            double* hist, bool* handled) {
+    *handled = false;
+    if (max_cycles > SF_LOOP_HIST || !loop_allowed(m)) return SF_OK;
+    if (!m->gloop[fc]) SF_TRY(build_loop(m, fc));
+    if (!m->gloop[fc]) return SF_OK;
+    sf_level* L = m->lv[0];
+    m->lhost->rtol = rtol;
+    m->lhost->max_cycles = max_cycles;
+    m->lhost->done = -1;
+    SF_CUDA(cudaGraphLaunch(m->gloop[fc], L->stream));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    *handled = true;
+    const LoopHost& r = *m->lhost;
+    if (r.done < 0) return sf_fail(SF_ERR_CUDA, "device solve loop did not publish");
+    sf_count_launch(m->loop_nodes[fc][0] + m->loop_nodes[fc][1] * r.nbody);
+    const int n = std::min(r.done, SF_LOOP_HIST);
+    if (r.status == LS_RHS_NAN) {
+        if (cycles) *cycles = 0;
+        return sf_fail(SF_ERR_NUMERIC, "rhs has NaN/Inf");
+    }
+    if (r.status == LS_ZERO) {
+        if (cycles) *cycles = 0;
+        SF_TRY(k_zero(L, SF_U));
+        return sf_sync(L);
+    }
+    if (cycles) *cycles = r.done;
+    if (hist)
+        for (int i = 0; i < n; i++) hist[i] = r.hist[i];
+    if (r.status == LS_NUMERIC) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
+    if (r.status == LS_NOT_CONVERGED)
+        return sf_fail(SF_ERR_NOT_CONVERGED, "no convergence to %g in %d cycles", rtol, max_cycles);
+    return SF_OK;
+}
+
 extern "C" sf_status sf_vcycle(sf_mg* m, int l) {
     if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
     if (l < 0 || l >= (int)m->lv.size()) return sf_fail(SF_ERR_INVALID, "bad level %d", l);
@@ -451,6 +698,11 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
     if (max_cycles < 1) max_cycles = m->o.max_cycles;
     if (!(rtol > 0)) rtol = m->o.rtol;
     sf_level* L = m->lv[0];
+    {
+        bool handled = false;
+        sf_status r = solve_loop(m, fcycle ? 1 : 0, rtol, max_cycles, cycles, hist, &handled);
+        if (handled || r != SF_OK) return r;
+    }
     double fn;
     SF_TRY(sf_norm(L, SF_F, SF_NORM_MAX, &fn));
     if (cycles) *cycles = 0;

@@ -508,6 +508,49 @@ def test_solve_eager_equals_graph(sf, oracle, fcycle):
     assert np.allclose(out[0][2], out[1][2], rtol=1e-12, atol=0)
 
 
+@pytest.mark.parametrize("fcycle", [False, True])
+@pytest.mark.parametrize("parts", [1, 2])
+def test_device_loop_equals_host_loop(sf, oracle, fcycle, parts):
+    """With graphs the whole solve is one graph launch whose WHILE node is
+    driven by the device-side convergence decision; it must reproduce the host
+    loop exactly: iterate, cycle count, every history entry (same IEEE
+    division) and the number of kernel launches."""
+    n = 32
+    out = {}
+    for g in (0, 1):
+        L, M, O = mg_pair(sf, oracle, n, parts=parts, use_graph=g)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        for rep in range(2):   # second solve: replay of the built loop
+            L.upload(sf.SF_U, np.zeros((n, n, n)))
+            sf.sf_launch_count(reset=True)
+            st, cyc, hist = M.solve(fcycle=fcycle, rtol=1e-10)
+            launches = sf.sf_launch_count(reset=True)
+        out[g] = (L.download(sf.SF_U), cyc, hist, launches)
+    assert out[0][1] == out[1][1] and out[0][2] == out[1][2]
+    assert np.array_equal(out[0][0], out[1][0])
+    # same kernels; the device loop adds its init + publish kernels and drops
+    # the host loop's copy of max|F| to the host
+    assert out[1][3] == out[0][3] + 1
+
+
+@pytest.mark.parametrize("use_graph", [0, 1])
+def test_solve_zero_and_nan_rhs(sf, oracle, use_graph):
+    """f = 0 gives u = 0 after zero cycles; a NaN in f is reported, not solved."""
+    n = 32
+    L, M, O = mg_pair(sf, oracle, n, use_graph=use_graph)
+    L.upload(sf.SF_U, I.random_field((n, n, n), 3))
+    L.upload(sf.SF_F, np.zeros((n, n, n)))
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, raise_on_error=False)
+    assert st == sf.SF_OK and cyc == 0
+    assert not L.download(sf.SF_U).any()
+    f = I.random_field((n, n, n), 1)
+    f[3, 4, 5] = np.nan
+    L.upload(sf.SF_F, f)
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, raise_on_error=False)
+    assert st == sf.SF_ERR_NUMERIC and cyc == 0
+
+
 @pytest.mark.parametrize("use_graph", [0, 1])
 def test_solve_max_cycles_keeps_last_cycle(sf, oracle, use_graph):
     """Stopping at max_cycles discards the speculative first pair of the next
