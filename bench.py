@@ -344,7 +344,7 @@ def main():
         }
         line.update({k: v for k, v in side.items() if k in (
             "e2e", "gsrb_c3", "vcycle", "fcycle", "fcycle_strong", "read_bw", "cpu_baseline", "fig7_256",
-            "gsrb_size_sweep", "dsl_256")})
+            "gsrb_size_sweep", "dsl_256", "c1_16", "c2_64")})
         print(json.dumps(line), flush=True)
     M.close()
     L.close()
@@ -552,6 +552,44 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
                           "colour_sweeps_ms_per_rb_pair": msc,
                           "note": "GStencil/s = point updates/s (each cell updated once per pair)"}
         G.close()
+        # BASELINE configs 1 and 2 (parity configs; latency-bound, timed for context):
+        # C1 16^3 CC Poisson, 2 RB pairs (4 sweeps) + residual; C2 64^3 VC Helmholtz,
+        # V-cycle solve from u = 0 to 1e-10 (one graph launch, device-side loop)
+        import numpy as np
+        from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
+        G1 = sf.Level(16, 16, 16, 1.0 / 16, stream=s)
+        G1.set_coeffs(*I.constant_coeffs(16, 16, 16))
+        sf.sf_rebuild_operator(G1.handle, 0.0, 1.0)
+
+        def c1():
+            sf.sf_smooth_gsrb(G1.handle, sf.SF_U, sf.SF_F, 0.0, 1.0, 2)
+            sf.sf_residual(G1.handle, sf.SF_R, sf.SF_U, sf.SF_F, 0.0, 1.0)
+        m1 = per_call(c1, 200)
+        G1.close()
+        G2 = sf.Level(64, 64, 64, 1.0 / 64, stream=s)
+        sf.sf_init_problem(G2.handle, 1, 1.0, 1.0, 1)
+        M2 = sf.MG(G2, 1.0, 1.0)
+        zeros = np.zeros((64, 64, 64))
+
+        def c2():
+            G2.upload(sf.SF_U, zeros)
+            return sf.sf_solve(M2.handle, False, 1e-10, 50)
+        c2()
+        s.synchronize()
+        t2 = time.perf_counter()
+        for _ in range(20):
+            _, cyc2, hist2 = c2()
+        m2 = (time.perf_counter() - t2) / 20 * 1e3
+        ue2, _ = I.manufactured(64, 64, 64, 1.0, 1.0, 1.0 / 64)
+        err2 = float(np.abs(G2.download(sf.SF_U) - ue2).max())
+        rho = (hist2[-1] / hist2[0]) ** (1.0 / max(1, len(hist2) - 1)) if len(hist2) > 1 else None
+        M2.close()
+        G2.close()
+        out["c1_16"] = {"ms": m1, "what": "2 RB pairs + residual, 16^3 CC Poisson (event-timed)"}
+        out["c2_64"] = {"ms_per_solve": m2, "cycles": cyc2, "final_relres": hist2[-1],
+                        "mean_rho": rho, "max_err_vs_manufactured": err2,
+                        "what": "64^3 VC Helmholtz V-cycle solve from u = 0 to 1e-10 (wall clock "
+                                "incl. the 2 MiB upload of u = 0 and the one host sync)"}
         if world == 1 and not args.no_cpu_baseline:
             shp, scale = oracle_shape((nx, ny, nz))
             tv, cores, desc = oracle_vcycle_sample(shp, reps=2)
