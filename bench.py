@@ -258,10 +258,25 @@ def main():
 
     nx, ny, nz = dims_for(args.side, world)
     comm = None
-    if world > 1:
-        comm = sf.Comm.p2p(host_group) if args.comm == "p2p" else sf.Comm.nccl()
+    transport = args.comm if world > 1 else "none"
     h = 1.0 / max(nx, ny, nz)
-    L = sf.Level(nx, ny, nz, h, comm=comm)
+    if world > 1 and args.comm == "p2p":
+        # device-initiated transport over CUDA IPC; if any rank cannot map its
+        # peers' buffers, every rank gets the same error (sf_ipc_register) and
+        # all fall back to NCCL together
+        comm = sf.Comm.p2p(host_group)
+        try:
+            L = sf.Level(nx, ny, nz, h, comm=comm)
+        except sf.SfError as e:
+            comm.close()
+            print(f"bench: p2p transport unavailable ({e}); using NCCL", file=sys.stderr)
+            comm = sf.Comm.nccl()
+            transport = "nccl (p2p unavailable)"
+            L = sf.Level(nx, ny, nz, h, comm=comm)
+    else:
+        if world > 1:
+            comm = sf.Comm.nccl()
+        L = sf.Level(nx, ny, nz, h, comm=comm)
     sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)       # HPGMG problem + manufactured f
     M = sf.MG(L, 1.0, 1.0)
     stream = L.stream
@@ -334,7 +349,7 @@ def main():
             "data": "synthetic (HPGMG-shaped VC Helmholtz, manufactured rhs, on-device init)",
             "config": {"workload": f"C5 HPGMG-FV VC Helmholtz {nx}x{ny}x{nz // world} per GPU",
                        "global": [nx, ny, nz], "parallelism": f"z-slab x{world}",
-                       "transport": (args.comm if world > 1 else "none"),
+                       "transport": transport,
                        "cycles_per_solve": cyc, "final_relres": hist[-1] if hist else None,
                        "max_err_vs_manufactured": err,
                        "smoother": "colour-fused GSRB, 2+2 pairs", "l2": "inputs >> L2, no flush"},

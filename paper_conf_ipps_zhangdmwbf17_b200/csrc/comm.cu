@@ -16,6 +16,7 @@
 #include <algorithm>
 
 #include <cstdlib>
+#include <cstring>
 
 #include "sf_internal.h"
 
@@ -300,20 +301,44 @@ sf_status sf_ipc_register(sf_level* L, const sf_comm* c) {
     struct Rec {
         cudaIpcMemHandle_t h;
         unsigned long long off;
+        int ok;
     } mine, all[64];
     if (c->nranks > 64) return sf_fail(SF_ERR_INVALID, "hostipc supports <= 64 ranks");
-    SF_CUDA(cudaIpcGetMemHandle(&mine.h, (void*)base));
+    // every rank reaches both all-gathers whatever fails locally, and all of
+    // them return the same error: a rank that cannot export or open a peer
+    // buffer must not leave the others waiting (callers fall back collectively)
+    memset(&mine, 0, sizeof(mine));
+    cudaError_t e = cudaIpcGetMemHandle(&mine.h, (void*)base);
+    mine.ok = e == cudaSuccess;
     mine.off = (unsigned long long)((char*)L->buf - (char*)base);
+    cudaGetLastError();
     SF_TRY(host_allgather(c, &mine, sizeof(Rec), all));
+    int ok = 1;
+    for (int r = 0; r < c->nranks; r++) ok &= all[r].ok;
+    if (const char* t = getenv("SF_TEST_IPC_FAIL_RANK"))   // tests: one rank cannot open
+        if (atoi(t) == c->rank) ok = 0;
     L->peer.assign(c->nranks, nullptr);
-    for (int r = 0; r < c->nranks; r++) {
+    for (int r = 0; r < c->nranks && ok; r++) {
         if (r == c->rank) continue;
         void* p = nullptr;
-        SF_CUDA(cudaIpcOpenMemHandle(&p, all[r].h, cudaIpcMemLazyEnablePeerAccess));   // NVLink P2P
+        e = cudaIpcOpenMemHandle(&p, all[r].h, cudaIpcMemLazyEnablePeerAccess);   // NVLink P2P
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            ok = 0;
+            break;
+        }
         L->ipc_opened.push_back(p);
         L->peer[r] = (char*)p + all[r].off;
     }
-    return host_barrier(c);
+    int oks[64];
+    SF_TRY(host_allgather(c, &ok, sizeof(int), oks));   // doubles as the barrier
+    for (int r = 0; r < c->nranks; r++)
+        if (!oks[r]) {
+            sf_ipc_close(L);
+            return sf_fail(SF_ERR_CUDA, "CUDA IPC: rank %d could not export or open a peer level buffer (%s)",
+                           r, cudaGetErrorString(e));
+        }
+    return SF_OK;
 }
 
 void sf_ipc_close(sf_level* L) {

@@ -132,3 +132,39 @@ def test_per_rank_matches_loopback(sf, world, transport):
             np.testing.assert_allclose(ranks[r][name][2], href, rtol=1e-9, atol=1e-13 * href[0])
         rel = np.linalg.norm((u - uref).ravel()) / np.linalg.norm(uref.ravel())
         assert rel < 1e-13, (name, rel)
+
+
+def _fail_worker(rank, world, port, out):
+    import os
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangdmwbf17_b200 import sf
+    os.environ["SF_TEST_IPC_FAIL_RANK"] = "1"
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
+                            world_size=world)
+    try:
+        comm = sf.Comm.p2p()
+        try:
+            sf.Level(32, 32, 48, comm=comm)
+            out[rank] = "created"
+        except sf.SfError as e:
+            out[rank] = str(e)
+        dist.barrier()
+        comm.close()
+    finally:
+        dist.destroy_process_group()
+
+
+def test_p2p_registration_fails_on_every_rank(sf):
+    """One rank cannot map its peers' buffers: every rank gets the same error
+    (no rank is left waiting in a barrier), so callers can fall back together
+    (bench.py switches to NCCL)."""
+    with mp.Manager() as m:
+        out = m.dict()
+        mp.spawn(_fail_worker, args=(3, _free_port(), out), nprocs=3, join=True)
+        res = dict(out)
+    assert len(res) == 3
+    assert all("rank 1 could not export or open" in v for v in res.values()), res
