@@ -250,7 +250,14 @@ sf_status sf_sync(sf_level* level);
  * sf_fcycle: one F-cycle from scratch for rhs F_0 into U_0, enqueued.
  * sf_solve: optional F-cycle, then V-cycles until ||F-AU||inf/||F||inf <
  *   rtol; fills *cycles and hist[0..*cycles-1] (may be NULL; caller array of
- *   max_cycles+1 doubles); syncs.
+ *   max_cycles+1 doubles); syncs.  F = 0 gives U = 0 and *cycles = 0; a NaN/Inf
+ *   in F returns SF_ERR_NUMERIC with *cycles = 0.  With use_graph and the
+ *   colour-fused smoother (max_cycles <= 256, no NCCL transport) the whole
+ *   solve is ONE CUDA graph launch whose WHILE node is driven by the
+ *   termination test evaluated on the device, and the call synchronises once;
+ *   otherwise the host tests after every cycle.  Both give the same iterate,
+ *   cycle count and history bits.  On SF_ERR_NOT_CONVERGED U holds the iterate
+ *   after exactly max_cycles cycles.
  */
 sf_status sf_mg_create(sf_mg** out, sf_level* finest, double a, double b, const sf_mg_opts* opts);
 /* Host-only (no device needed): the hierarchy sf_mg_create builds for a
