@@ -222,7 +222,7 @@ __device__ __forceinline__ void p2p_end(unsigned long long* my, const P2PPeers& 
 // halo: my ghosts <- the neighbours' boundary planes (peers 0 = lower, 1 = upper)
 __global__ void __launch_bounds__(256) p2p_halo_kernel(double* x, const double* lo_x, const double* hi_x,
                                                        unsigned long long* my, P2PPeers pe, long lo_dst,
-                                                       long hi_src, long hi_dst, long lo_src, long cnt) {
+                                                       long hi_src, long hi_dst, long lo_src, long cnt) { pdl_wait();
     const unsigned long long s = p2p_begin(my, pe, 2);
     const long stride = (long)gridDim.x * blockDim.x;
     for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) {
@@ -239,7 +239,7 @@ struct P2PPtrs {
 // all-reduce of one scalar: my slot <- v; every rank reduces all ranks' slots
 // in rank order (the same result on every rank)
 __global__ void p2p_allreduce_kernel(double* v, unsigned long long* my, P2PPeers pe, P2PPtrs slot,
-                                     int nranks, int op) {
+                                     int nranks, int op) { pdl_wait();
     // my slot is rewritten only after every peer consumed the previous op
     if (threadIdx.x == 0) *(double*)(my + 8) = *v;
     const unsigned long long s = p2p_begin(my, pe, nranks);
@@ -260,7 +260,7 @@ __global__ void p2p_allreduce_kernel(double* v, unsigned long long* my, P2PPeers
 __global__ void __launch_bounds__(256) p2p_gather_kernel(double* base, P2PPtrs peer_base,
                                                          unsigned long long* my, P2PPeers pe, int nranks,
                                                          int rank, long cnt, double* top,
-                                                         const double* peer_top, long topcnt) {
+                                                         const double* peer_top, long topcnt) { pdl_wait();
     const unsigned long long s = p2p_begin(my, pe, nranks);
     const long stride = (long)gridDim.x * blockDim.x;
     for (int q = 0; q < nranks; q++) {
@@ -396,7 +396,7 @@ sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t stream) {
         if (r > 0) { pe.sync[0] = peer_sync(L, r - 1); lo_x = peer_field(L, r - 1, x); }
         if (r < n - 1) { pe.sync[1] = peer_sync(L, r + 1); hi_x = peer_field(L, r + 1, x); }
         const int grid = (int)std::min<long>(max_ctas, ((long)cnt + 255) / 256);
-        p2p_halo_kernel<<<grid, 256, 0, stream>>>(x, lo_x, hi_x, L->dsync, pe, lo_dst, hi_src, hi_dst,
+        sf_launch(p2p_halo_kernel, grid, 256, 0, stream, x, lo_x, hi_x, L->dsync, pe, lo_dst, hi_src, hi_dst,
                                                      lo_src, (long)cnt);
         SF_LAUNCHED();
         return sf_check_launch("p2p_halo");
@@ -451,7 +451,7 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
         const double* ptop = (field == SF_BETA_K && cm->rank != parts - 1) ? peer_field(C, parts - 1, top)
                                                                            : nullptr;
         const int grid = (int)std::min<long>(148, (cnt + 255) / 256);
-        p2p_gather_kernel<<<grid, 256, 0, C->stream>>>(base, pb, C->dsync, pe, parts, cm->rank, cnt, top,
+        sf_launch(p2p_gather_kernel, grid, 256, 0, C->stream, base, pb, C->dsync, pe, parts, cm->rank, cnt, top,
                                                        ptop, C->ks);
         SF_LAUNCHED();
         return sf_check_launch("p2p_gather");
@@ -495,7 +495,7 @@ sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int o
             if (q != cm->rank) pe.sync[q] = peer_sync(L, q);
             sl.p[q] = (const double*)((q == cm->rank ? L->dsync : peer_sync(L, q)) + 8);
         }
-        p2p_allreduce_kernel<<<1, 32, 0, s>>>(dev, L->dsync, pe, sl, cm->nranks, op);
+        sf_launch(p2p_allreduce_kernel, 1, 32, 0, s, dev, L->dsync, pe, sl, cm->nranks, op);
         SF_LAUNCHED();
         return sf_check_launch("p2p_allreduce");
     }

@@ -238,7 +238,7 @@ template <bool RESID, bool INTERP, bool BRES>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
-                     CoarseView cv, int c0, int cstride) {
+                     CoarseView cv, int c0, int cstride) { pdl_wait();
     constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
@@ -539,7 +539,7 @@ bool SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(const sf_level* L) {
     return L->nx % TX == 0 && L->ny % TY == 0 && L->lnz >= 1;
 }
 
-static __global__ void zero_bits(double* p) { *p = 0.0; }
+static __global__ void zero_bits(double* p) { pdl_wait(); *p = 0.0; }
 
 template <bool R, bool I, bool B>
 static sf_status set_attrs() {
@@ -623,12 +623,12 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
             cvw = CoarseView{c.f[cf], C->js, C->ks, rep ? v.z0 / 2 : 0};
         }
         if (rmode == SF_RM_OUTPUT_BLACK && p == 0 && phase != 2) {
-            zero_bits<<<1, 1, 0, L->stream>>>(rmax);
+            sf_launch(zero_bits, 1, 1, 0, L->stream, rmax);
             SF_LAUNCHED();
         }
         double* xo = v.f[xout];
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
-    gsrb_pair_tma_kernel<R, I, B><<<grid, NT, SMEM, L->stream>>>(mp, g, xo, a, bh2, depth, ntx, tiles, \
+    sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride)
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);

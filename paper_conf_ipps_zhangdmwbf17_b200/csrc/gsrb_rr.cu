@@ -160,7 +160,7 @@ __device__ __forceinline__ double sum_at(const double* Xk, const double* Xm, con
 
 __global__ void __launch_bounds__(NT, 1)
 gsrb_rr_kernel(const __grid_constant__ Maps mp, const Ptrs pt, Geo g, double* __restrict__ xo,
-               double bh2, int depth, int ntx, int ntiles, int nitems) {
+               double bh2, int depth, int ntx, int ntiles, int nitems) { pdl_wait();
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][WX]
     double* Cs = Xs + NXS * XSLOT;                    // [NCS][NCA][CH][WC]
@@ -460,7 +460,7 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
     Ptrs pt{c.f[cf], C->js, C->ks};
     Geo g{v.nx, v.ny, v.nz, v.js, v.ks};
     const double bh2 = b / (L->h * L->h);
-    gsrb_rr_kernel<<<std::min(items, g_sms), NT, SMEM, L->stream>>>(mp, pt, g, v.f[xout], bh2, depth,
+    sf_launch(gsrb_rr_kernel, std::min(items, g_sms), NT, SMEM, L->stream, mp, pt, g, v.f[xout], bh2, depth,
                                                                      ntx, tiles, items);
     SF_LAUNCHED();
     return sf_check_launch("gsrb_rr");

@@ -51,7 +51,7 @@ __device__ __forceinline__ double op_at(const PV& v, const double* __restrict__ 
 
 __global__ void __launch_bounds__(BX* BY) apply_op_kernel(PV v, double* __restrict__ out,
                                                            const double* __restrict__ x, double a,
-                                                           double bh2) {
+                                                           double bh2) { pdl_wait();
     int i = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     if (i >= v.nx || j >= v.ny) return;
     out[sf_ix(v, i, j, k)] = op_at(v, x, i, j, k, a, bh2);
@@ -60,7 +60,7 @@ __global__ void __launch_bounds__(BX* BY) apply_op_kernel(PV v, double* __restri
 __global__ void __launch_bounds__(BX* BY) residual_kernel(PV v, double* __restrict__ res,
                                                            const double* __restrict__ x,
                                                            const double* __restrict__ rhs,
-                                                           double a, double bh2) {
+                                                           double a, double bh2) { pdl_wait();
     int i = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     if (i >= v.nx || j >= v.ny) return;
     long c = sf_ix(v, i, j, k);
@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(BX* BY) residual_kernel(PV v, double* __restri
 // (gi+gj+gk) % 2 == colour (reading R-2).  One thread per cell of the colour.
 __global__ void __launch_bounds__(BX* BY) gsrb_colour_kernel(PV v, double* __restrict__ x,
                                                               const double* __restrict__ rhs,
-                                                              double a, double bh2, int colour) {
+                                                              double a, double bh2, int colour) { pdl_wait();
     int t = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     int i = 2 * t + ((j + v.z0 + k + colour) & 1);
     if (i >= v.nx || j >= v.ny) return;
@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(BX* BY) gsrb_colour_kernel(PV v, double* __res
 }
 
 // A4: exact inverse diagonal with the Dirichlet fold.
-__global__ void __launch_bounds__(BX* BY) dinv_kernel(PV v, double a, double bh2) {
+__global__ void __launch_bounds__(BX* BY) dinv_kernel(PV v, double a, double bh2) { pdl_wait();
     int i = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     if (i >= v.nx || j >= v.ny) return;
     long c = sf_ix(v, i, j, k);
@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(BX* BY) dinv_kernel(PV v, double a, double bh2
 // where the cell is outside a GLOBAL boundary are reflected (odd reflection,
 // sign (-1)^m); z ghost planes at part interfaces are halos and are left as
 // exchanged (their x/y ghosts are still reflected).
-__global__ void bc_kernel(PV v, double* __restrict__ x) {
+__global__ void bc_kernel(PV v, double* __restrict__ x) { pdl_wait();
     int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
     int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
     int k = blockIdx.z - 1;
@@ -126,7 +126,7 @@ __global__ void bc_kernel(PV v, double* __restrict__ x) {
 // replicated coarse part (agglomeration), else 0.
 __global__ void __launch_bounds__(BX* BY) restrict_cell_kernel(PV c, double* __restrict__ cx,
                                                                 PV f, const double* __restrict__ x,
-                                                                int zoff) {
+                                                                int zoff) { pdl_wait();
     int I = blockIdx.x * BX + threadIdx.x, J = blockIdx.y * BY + threadIdx.y, K = blockIdx.z;
     if (I >= f.nx / 2 || J >= f.ny / 2) return;
     double s = 0.0;
@@ -142,7 +142,7 @@ __global__ void __launch_bounds__(BX* BY) restrict_cell_kernel(PV c, double* __r
 // A7 face (dir 0/1/2 = beta_i/j/k): average of the 4 fine faces covering the
 // coarse face.  Face index along dir runs to n (inclusive).
 __global__ void restrict_face_kernel(PV c, double* __restrict__ cx, PV f,
-                                     const double* __restrict__ x, int dir, int zoff, int ncz) {
+                                     const double* __restrict__ x, int dir, int zoff, int ncz) { pdl_wait();
     int I = blockIdx.x * blockDim.x + threadIdx.x, J = blockIdx.y * blockDim.y + threadIdx.y;
     int K = blockIdx.z;
     int ncx = f.nx / 2 + (dir == 0), ncy = f.ny / 2 + (dir == 1);
@@ -165,7 +165,7 @@ __global__ void restrict_face_kernel(PV c, double* __restrict__ cx, PV f,
 // plane inside the coarse part (replicated coarse levels), else 0.
 __global__ void __launch_bounds__(BX* BY) interp_p0_kernel(PV f, double* __restrict__ y, double s,
                                                             PV c, const double* __restrict__ x,
-                                                            int zoff) {
+                                                            int zoff) { pdl_wait();
     int i = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     if (i >= f.nx || j >= f.ny) return;
     long q = sf_ix(f, i, j, k);
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(BX* BY) interp_p0_kernel(PV f, double* __restr
 // valid.  Summation order matches the oracle (children in x, y, z order).
 __global__ void __launch_bounds__(BX* BY) interp_pl_kernel(PV f, double* __restrict__ y, double s,
                                                             PV c, const double* __restrict__ x,
-                                                            int zoff) {
+                                                            int zoff) { pdl_wait();
     int i = blockIdx.x * BX + threadIdx.x, j = blockIdx.y * BY + threadIdx.y, k = blockIdx.z;
     if (i >= f.nx || j >= f.ny) return;
     int gkf = f.z0 + k;                    // global fine plane -> parity of the child
@@ -203,7 +203,7 @@ __global__ void __launch_bounds__(BX* BY) interp_pl_kernel(PV f, double* __restr
 // pairs.  Each child's sum is the same ordered FMA chain as interp_pl_kernel.
 __global__ void __launch_bounds__(BX* BY) interp_pl_block_kernel(PV f, double* __restrict__ y, double s,
                                                                   PV c, const double* __restrict__ x,
-                                                                  int zoff) {
+                                                                  int zoff) { pdl_wait();
     const int I = blockIdx.x * BX + threadIdx.x, J = blockIdx.y * BY + threadIdx.y, Kl = blockIdx.z;
     if (2 * I >= f.nx || 2 * J >= f.ny) return;
     const int K = Kl + zoff;
@@ -252,7 +252,7 @@ __global__ void __launch_bounds__(BX* BY) interp_pl_block_kernel(PV f, double* _
 // for non-negative doubles the unsigned order of the bits is the numeric
 // order, and a (positive) NaN compares above +Inf, so NaN propagates.
 __global__ void __launch_bounds__(256) norm_kernel(PV v, const double* __restrict__ x, int kind,
-                                                   double* out) {
+                                                   double* out) { pdl_wait();
     __shared__ unsigned long long rmax[256];
     __shared__ double rsum[256];
     unsigned long long m = 0ull;
@@ -286,7 +286,7 @@ __global__ void __launch_bounds__(256) norm_kernel(PV v, const double* __restric
     }
 }
 
-__global__ void zero_scalar_kernel(double* p) { *p = 0.0; }
+__global__ void zero_scalar_kernel(double* p) { pdl_wait(); *p = 0.0; }
 
 // ----------------------------------------------------------------- problem init
 // HPGMG-shaped problem (the same recipe as
@@ -302,7 +302,7 @@ __device__ double dXf(double t) { return 12 * pow(t, 5) - 30 * pow(t, 4) + 20 * 
 __device__ double d2Xf(double t) { return 60 * pow(t, 4) - 120 * pow(t, 3) + 60 * t * t - 2; }
 
 __global__ void init_problem_kernel(PV v, int gnx, int gny, double h, int problem, double a,
-                                    double b, int want_rhs) {
+                                    double b, int want_rhs) { pdl_wait();
     int i = blockIdx.x * blockDim.x + threadIdx.x, j = blockIdx.y * blockDim.y + threadIdx.y;
     int k = blockIdx.z;  // 0..nz  (face planes run to nz)
     if (i > v.nx || j > v.ny || k > v.nz) return;
@@ -353,7 +353,7 @@ constexpr int BOT_MAX = 64;
 constexpr int BOT_LD = 2 * BOT_MAX + 1;
 constexpr size_t BOT_SMEM = sizeof(double) * BOT_MAX * BOT_LD;
 
-__global__ void bottom_setup_kernel(PV v, double a, double bh2, double* ainv) {
+__global__ void bottom_setup_kernel(PV v, double a, double bh2, double* ainv) { pdl_wait();
     extern __shared__ double Msh[];
     double(*M)[BOT_LD] = reinterpret_cast<double(*)[BOT_LD]>(Msh);
     int n = v.nx * v.ny * v.nz;
@@ -402,7 +402,7 @@ __global__ void bottom_setup_kernel(PV v, double a, double bh2, double* ainv) {
 }
 
 __global__ void bottom_solve_kernel(PV v, double* __restrict__ x, const double* __restrict__ rhs,
-                                    const double* __restrict__ ainv) {
+                                    const double* __restrict__ ainv) { pdl_wait();
     __shared__ double rr[BOT_MAX];
     int n = v.nx * v.ny * v.nz;
     int r = threadIdx.x;
@@ -427,7 +427,7 @@ sf_status k_apply_op(sf_level* L, int out, int x, double a, double b) {
     SF_TRY(sf_halo(L, x, 1));
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
-        apply_op_kernel<<<cell_grid(v), dim3(BX, BY), 0, L->stream>>>(v, v.f[out], v.f[x], a, bh2);
+        sf_launch(apply_op_kernel, cell_grid(v), dim3(BX, BY), 0, L->stream, v, v.f[out], v.f[x], a, bh2);
         SF_LAUNCHED();
     }
     return sf_check_launch("apply_op");
@@ -439,7 +439,7 @@ sf_status k_residual(sf_level* L, int res, int x, int rhs, double a, double b) {
     SF_TRY(sf_halo(L, x, 1));
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
-        residual_kernel<<<cell_grid(v), dim3(BX, BY), 0, L->stream>>>(v, v.f[res], v.f[x], v.f[rhs],
+        sf_launch(residual_kernel, cell_grid(v), dim3(BX, BY), 0, L->stream, v, v.f[res], v.f[x], v.f[rhs],
                                                                       a, bh2);
         SF_LAUNCHED();
     }
@@ -452,7 +452,7 @@ sf_status k_gsrb_colour(sf_level* L, int x, int rhs, double a, double b, int col
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         dim3 g(((v.nx + 1) / 2 + BX - 1) / BX, (v.ny + BY - 1) / BY, v.nz);
-        gsrb_colour_kernel<<<g, dim3(BX, BY), 0, L->stream>>>(v, v.f[x], v.f[rhs], a, bh2, colour);
+        sf_launch(gsrb_colour_kernel, g, dim3(BX, BY), 0, L->stream, v, v.f[x], v.f[rhs], a, bh2, colour);
         SF_LAUNCHED();
     }
     return sf_check_launch("gsrb_colour");
@@ -462,7 +462,7 @@ sf_status k_dinv(sf_level* L, double a, double b) {
     double bh2 = b / (L->h * L->h);
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
-        dinv_kernel<<<cell_grid(v), dim3(BX, BY), 0, L->stream>>>(v, a, bh2);
+        sf_launch(dinv_kernel, cell_grid(v), dim3(BX, BY), 0, L->stream, v, a, bh2);
         SF_LAUNCHED();
     }
     return sf_check_launch("dinv");
@@ -473,7 +473,7 @@ sf_status k_bc(sf_level* L, int field) {
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         dim3 g((v.nx + 2 + BX - 1) / BX, (v.ny + 2 + BY - 1) / BY, v.nz + 2);
-        bc_kernel<<<g, dim3(BX, BY), 0, L->stream>>>(v, v.f[field]);
+        sf_launch(bc_kernel, g, dim3(BX, BY), 0, L->stream, v, v.f[field]);
         SF_LAUNCHED();
     }
     return sf_check_launch("bc");
@@ -493,14 +493,14 @@ sf_status k_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind) {
         int zoff = rep ? f.z0 / 2 : 0;
         if (kind == SF_RESTRICT_CELL) {
             dim3 g((f.nx / 2 + BX - 1) / BX, (f.ny / 2 + BY - 1) / BY, f.nz / 2);
-            restrict_cell_kernel<<<g, dim3(BX, BY), 0, F->stream>>>(c, c.f[cf], f, f.f[ff], zoff);
+            sf_launch(restrict_cell_kernel, g, dim3(BX, BY), 0, F->stream, c, c.f[cf], f, f.f[ff], zoff);
         } else {
             int dir = kind - SF_RESTRICT_FACE_I;
             // beta_k: the top face of a part (index lnz/2) is written by every
             // part (it duplicates the next part's face 0, as uploaded).
             int ncz = f.nz / 2 + (dir == 2);
             dim3 g((f.nx / 2 + 1 + BX - 1) / BX, (f.ny / 2 + 1 + BY - 1) / BY, ncz);
-            restrict_face_kernel<<<g, dim3(BX, BY), 0, F->stream>>>(c, c.f[cf], f, f.f[ff], dir, zoff,
+            sf_launch(restrict_face_kernel, g, dim3(BX, BY), 0, F->stream, c, c.f[cf], f, f.f[ff], dir, zoff,
                                                                     ncz);
         }
         SF_LAUNCHED();
@@ -519,13 +519,12 @@ sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind)
         PV c = sf_view(C, rep ? 0 : p);
         int zoff = rep ? f.z0 / 2 : 0;
         if (kind == SF_INTERP_P0)
-            interp_p0_kernel<<<cell_grid(f), dim3(BX, BY), 0, F->stream>>>(f, f.f[ff], s, c, c.f[cf],
+            sf_launch(interp_p0_kernel, cell_grid(f), dim3(BX, BY), 0, F->stream, f, f.f[ff], s, c, c.f[cf],
                                                                            zoff);
         else if (f.nx % 2 == 0 && f.ny % 2 == 0 && f.nz % 2 == 0)
-            interp_pl_block_kernel<<<dim3((f.nx / 2 + BX - 1) / BX, (f.ny / 2 + BY - 1) / BY, f.nz / 2),
-                                     dim3(BX, BY), 0, F->stream>>>(f, f.f[ff], s, c, c.f[cf], zoff);
+            sf_launch(interp_pl_block_kernel, dim3((f.nx / 2 + BX - 1) / BX, (f.ny / 2 + BY - 1) / BY, f.nz / 2), dim3(BX, BY), 0, F->stream, f, f.f[ff], s, c, c.f[cf], zoff);
         else
-            interp_pl_kernel<<<cell_grid(f), dim3(BX, BY), 0, F->stream>>>(f, f.f[ff], s, c, c.f[cf],
+            sf_launch(interp_pl_kernel, cell_grid(f), dim3(BX, BY), 0, F->stream, f, f.f[ff], s, c, c.f[cf],
                                                                            zoff);
         SF_LAUNCHED();
     }
@@ -534,13 +533,13 @@ sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind)
 
 sf_status k_norm(sf_level* L, int field, int kind, double* dst) {
     if (pair_ok(L)) return k_norm_pair(L, field, kind, dst);
-    zero_scalar_kernel<<<1, 1, 0, L->stream>>>(dst);
+    sf_launch(zero_scalar_kernel, 1, 1, 0, L->stream, dst);
     SF_LAUNCHED();
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         long n = (long)v.nx * v.ny * v.nz;
         int blocks = (int)std::min<long>((n + 255) / 256, 148L * 8);
-        norm_kernel<<<blocks, 256, 0, L->stream>>>(v, v.f[field], kind, dst);
+        sf_launch(norm_kernel, blocks, 256, 0, L->stream, v, v.f[field], kind, dst);
         SF_LAUNCHED();
     }
     return sf_check_launch("norm");
@@ -549,7 +548,7 @@ sf_status k_norm(sf_level* L, int field, int kind, double* dst) {
 // packed host-layout buffer (nzh, nyh, nxh) <-> strided field interior of one part
 __global__ void __launch_bounds__(256) pack_kernel(double* __restrict__ field, long js, long ks,
                                                    double* __restrict__ buf, int nxh, int nyh,
-                                                   int nzh, int up) {
+                                                   int nzh, int up) { pdl_wait();
     const long rows = (long)nyh * nzh;
     for (long r = blockIdx.x; r < rows; r += gridDim.x) {
         const int j = (int)(r % nyh), k = (int)(r / nyh);
@@ -574,7 +573,7 @@ sf_status k_pack(sf_level* L, int field, double* buf, bool up) {
         double* b = buf + (size_t)q * L->lnz * nyh * nxh;
         const long rows = (long)nyh * nzh;
         const int grid = (int)std::min<long>(rows, 148L * 16);
-        pack_kernel<<<grid, 256, 0, L->stream>>>(L->parts[q].f[field], L->js, L->ks, b, nxh, nyh,
+        sf_launch(pack_kernel, grid, 256, 0, L->stream, L->parts[q].f[field], L->js, L->ks, b, nxh, nyh,
                                                  nzh, up ? 1 : 0);
         SF_LAUNCHED();
     }
@@ -591,7 +590,7 @@ sf_status k_init_problem(sf_level* L, int problem, double a, double b, int want_
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         dim3 g((v.nx + 1 + BX - 1) / BX, (v.ny + 1 + BY - 1) / BY, v.nz + 1);
-        init_problem_kernel<<<g, dim3(BX, BY), 0, L->stream>>>(v, L->gnx, L->gny, L->h, problem,
+        sf_launch(init_problem_kernel, g, dim3(BX, BY), 0, L->stream, v, L->gnx, L->gny, L->h, problem,
                                                                a, b, want_rhs);
         SF_LAUNCHED();
     }
@@ -605,14 +604,14 @@ sf_status k_bottom_setup(sf_level* L, double a, double b, double* ainv) {
     if (n > BOT_MAX) return sf_fail(SF_ERR_SHAPE, "bottom level has %d cells (> %d)", n, BOT_MAX);
     SF_CUDA(cudaFuncSetAttribute(bottom_setup_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)BOT_SMEM));
-    bottom_setup_kernel<<<1, BOT_MAX, BOT_SMEM, L->stream>>>(v, a, b / (L->h * L->h), ainv);
+    sf_launch(bottom_setup_kernel, 1, BOT_MAX, BOT_SMEM, L->stream, v, a, b / (L->h * L->h), ainv);
     SF_LAUNCHED();
     return sf_check_launch("bottom_setup");
 }
 
 sf_status k_bottom_solve(sf_level* L, int x, int rhs, const double* ainv) {
     PV v = sf_view(L, 0);
-    bottom_solve_kernel<<<1, BOT_MAX, 0, L->stream>>>(v, v.f[x], v.f[rhs], ainv);
+    sf_launch(bottom_solve_kernel, 1, BOT_MAX, 0, L->stream, v, v.f[x], v.f[rhs], ainv);
     SF_LAUNCHED();
     return sf_check_launch("bottom_solve");
 }

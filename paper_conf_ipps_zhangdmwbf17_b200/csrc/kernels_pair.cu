@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(PX* PY) residual_pair_kernel(PV v, double* __r
                                                                 const double* __restrict__ x,
                                                                 const double* __restrict__ rhs,
                                                                 double a, double bh2, int depth,
-                                                                double* nout) {
+                                                                double* nout) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     unsigned long long m = 0ull;
@@ -109,7 +109,7 @@ __global__ void __launch_bounds__(PX* PY) residual_restrict_kernel(PV f, const d
                                                                     const double* __restrict__ rhs,
                                                                     double a, double bh2, PV c,
                                                                     double* __restrict__ cx,
-                                                                    int zoff, int depth) {
+                                                                    int zoff, int depth) { pdl_wait();
     const int I = blockIdx.x * PX + threadIdx.x, J = blockIdx.y * PY + threadIdx.y;
     const int K0 = blockIdx.z * depth, K1 = min(K0 + depth, f.nz / 2);
     if (2 * I >= f.nx || 2 * J >= f.ny) return;
@@ -171,7 +171,7 @@ __device__ __forceinline__ double2 neg2(double2 u) { return make_double2(-u.x, -
 template <int MINB>
 __global__ void __launch_bounds__(PX* PY, MINB) residual_restrict_zs_kernel(
     PV f, const double* __restrict__ x, const double* __restrict__ rhs, double a, double bh2, PV c,
-    double* __restrict__ cx, int zoff, int depth, int tgx, int ntiles, int nitems) {
+    double* __restrict__ cx, int zoff, int depth, int tgx, int ntiles, int nitems) { pdl_wait();
     const int nK = f.nz / 2;
     const double* bj = f.f[SF_BETA_J];
     const double* bk = f.f[SF_BETA_K];
@@ -229,7 +229,7 @@ __global__ void __launch_bounds__(PX* PY, MINB) residual_restrict_zs_kernel(
 // fine pair (2I', 2I'+1) shares its coarse parent
 __global__ void __launch_bounds__(PX* PY) interp_p0_pair_kernel(PV f, double* __restrict__ y, double s,
                                                                  PV c, const double* __restrict__ x,
-                                                                 int zoff, int depth) {
+                                                                 int zoff, int depth) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, f.nz);
     if (i >= f.nx || j >= f.ny) return;
@@ -249,7 +249,7 @@ __global__ void __launch_bounds__(PX* PY) interp_p0_pair_kernel(PV f, double* __
 }
 
 __global__ void __launch_bounds__(PX* PY) norm_pair_kernel(PV v, const double* __restrict__ x,
-                                                            int kind, int depth, double* out) {
+                                                            int kind, int depth, double* out) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     unsigned long long m = 0ull;
@@ -285,7 +285,7 @@ template <bool JACOBI>
 __global__ void __launch_bounds__(PX* PY) cc_pair_kernel(PV v, double* __restrict__ out,
                                                           const double* __restrict__ x,
                                                           const double* __restrict__ f,
-                                                          double hm2, double h2w, int depth) {
+                                                          double hm2, double h2w, int depth) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     if (i >= v.nx || j >= v.ny) return;
@@ -342,7 +342,7 @@ __global__ void __launch_bounds__(PX* PY) cheby_pair_kernel(PV v, double* __rest
                                                              const double* __restrict__ xp,
                                                              const double* __restrict__ rhs,
                                                              double c1, double c2, double a,
-                                                             double bh2, int depth) {
+                                                             double bh2, int depth) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     if (i >= v.nx || j >= v.ny) return;
@@ -362,7 +362,7 @@ __global__ void __launch_bounds__(PX* PY) cheby_pair_kernel(PV v, double* __rest
 // power-iteration helpers for lambda_max(D^-1 A): w *= Dinv with sum w^2 (atomic),
 // and v = w * scale[0]
 __global__ void __launch_bounds__(PX* PY) dinv_scale_pair_kernel(PV v, double* __restrict__ w,
-                                                                  int depth, double* sumsq) {
+                                                                  int depth, double* sumsq) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     double acc = 0.0;
@@ -392,7 +392,7 @@ __global__ void __launch_bounds__(PX* PY) dinv_scale_pair_kernel(PV v, double* _
 // test builds the same formula independently):
 // v(i,j,k) = 1 + ((7 gi + 13 gj + 29 gk) mod 17) / 17
 __global__ void __launch_bounds__(PX* PY) start_vector_kernel(PV v, double* __restrict__ y,
-                                                               int depth) {
+                                                               int depth) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     if (i >= v.nx || j >= v.ny) return;
@@ -407,7 +407,7 @@ __global__ void __launch_bounds__(PX* PY) start_vector_kernel(PV v, double* __re
 
 __global__ void __launch_bounds__(PX* PY) scale_pair_kernel(PV v, double* __restrict__ y,
                                                              const double* __restrict__ src,
-                                                             const double* sumsq, int depth) {
+                                                             const double* sumsq, int depth) { pdl_wait();
     const int i = 2 * (blockIdx.x * PX + threadIdx.x), j = blockIdx.y * PY + threadIdx.y;
     const int k0 = blockIdx.z * depth, k1 = min(k0 + depth, v.nz);
     if (i >= v.nx || j >= v.ny) return;
@@ -421,7 +421,7 @@ __global__ void __launch_bounds__(PX* PY) scale_pair_kernel(PV v, double* __rest
     }
 }
 
-__global__ void zero_scalar(double* p) { *p = 0.0; }
+__global__ void zero_scalar(double* p) { pdl_wait(); *p = 0.0; }
 
 // grid over pairs: (ceil(nx/64), ceil(ny/4), z-chunks) with ~16 blocks per SM
 inline dim3 pair_grid(int nx, int ny, int nz, int* depth) {
@@ -465,7 +465,7 @@ sf_status k_residual_pair(sf_level* L, int res, int x, int rhs, double a, double
     const double bh2 = b / (L->h * L->h);
     SF_TRY(sf_halo(L, x, 1));
     if (nout) {
-        zero_scalar<<<1, 1, 0, L->stream>>>(nout);
+        sf_launch(zero_scalar, 1, 1, 0, L->stream, nout);
         SF_LAUNCHED();
     }
     for (int p = 0; p < L->nlocal; p++) {
@@ -474,11 +474,11 @@ sf_status k_residual_pair(sf_level* L, int res, int x, int rhs, double a, double
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
         double* r = res >= 0 ? v.f[res] : nullptr;
         if (r && nout)
-            residual_pair_kernel<true, true><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+            sf_launch(residual_pair_kernel<true, true>, g, dim3(PX, PY), 0, L->stream, v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
         else if (r)
-            residual_pair_kernel<true, false><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+            sf_launch(residual_pair_kernel<true, false>, g, dim3(PX, PY), 0, L->stream, v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
         else
-            residual_pair_kernel<false, true><<<g, dim3(PX, PY), 0, L->stream>>>(v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
+            sf_launch(residual_pair_kernel<false, true>, g, dim3(PX, PY), 0, L->stream, v, r, v.f[x], v.f[rhs], a, bh2, depth, nout);
         SF_LAUNCHED();
     }
     return sf_check_launch("residual_pair");
@@ -505,7 +505,7 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
             }
             const int items = tiles * ((nK + best_d - 1) / best_d);
 #define SF_RRZS(MB)                                                                              \
-    residual_restrict_zs_kernel<MB><<<std::min(items, G), dim3(PX, PY), 0, F->stream>>>(          \
+    sf_launch(residual_restrict_zs_kernel<MB>, std::min(items, G), dim3(PX, PY), 0, F->stream,           \
         f, f.f[x], f.f[rhs], a, bh2, c, c.f[cf], rep ? f.z0 / 2 : 0, best_d, tgx, tiles, items)
             if (rr_zs() == 2) SF_RRZS(6);
             else if (rr_zs() == 3) SF_RRZS(8);
@@ -514,7 +514,7 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
         } else {
             int depth;
             dim3 g = pair_grid(f.nx, f.ny / 2, f.nz / 2, &depth);  // thread per coarse (I,J)
-            residual_restrict_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[x], f.f[rhs], a, bh2,
+            sf_launch(residual_restrict_kernel, g, dim3(PX, PY), 0, F->stream, f, f.f[x], f.f[rhs], a, bh2,
                                                                         c, c.f[cf],
                                                                         rep ? f.z0 / 2 : 0, depth);
         }
@@ -532,7 +532,7 @@ sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf) {
         PV c = sf_view(C, rep ? 0 : p);
         int depth;
         dim3 g = pair_grid(f.nx, f.ny, f.nz, &depth);
-        interp_p0_pair_kernel<<<g, dim3(PX, PY), 0, F->stream>>>(f, f.f[ff], s, c, c.f[cf],
+        sf_launch(interp_p0_pair_kernel, g, dim3(PX, PY), 0, F->stream, f, f.f[ff], s, c, c.f[cf],
                                                                  rep ? f.z0 / 2 : 0, depth);
         SF_LAUNCHED();
     }
@@ -548,10 +548,10 @@ sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi) {
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
         if (jacobi)
-            cc_pair_kernel<true><<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], v.f[f], hm2,
+            sf_launch(cc_pair_kernel<true>, g, dim3(PX, PY), 0, L->stream, v, v.f[out], v.f[x], v.f[f], hm2,
                                                                      h2w, depth);
         else
-            cc_pair_kernel<false><<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], nullptr,
+            sf_launch(cc_pair_kernel<false>, g, dim3(PX, PY), 0, L->stream, v, v.f[out], v.f[x], nullptr,
                                                                       hm2, h2w, depth);
         SF_LAUNCHED();
     }
@@ -567,7 +567,7 @@ sf_status k_cheby_step(sf_level* L, int out, int x, int xp, int rhs, double c1, 
         PV v = sf_view(L, p);
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
-        cheby_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[out], v.f[x], v.f[xp], v.f[rhs],
+        sf_launch(cheby_pair_kernel, g, dim3(PX, PY), 0, L->stream, v, v.f[out], v.f[x], v.f[xp], v.f[rhs],
                                                              c1, c2, a, bh2, depth);
         SF_LAUNCHED();
     }
@@ -579,7 +579,7 @@ sf_status k_start_vector(sf_level* L, int field) {
         PV v = sf_view(L, p);
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
-        start_vector_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[field], depth);
+        sf_launch(start_vector_kernel, g, dim3(PX, PY), 0, L->stream, v, v.f[field], depth);
         SF_LAUNCHED();
     }
     return sf_check_launch("start_vector");
@@ -589,13 +589,13 @@ sf_status k_start_vector(sf_level* L, int field) {
 sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, double* sumsq) {
     if (!pair_ok(L)) return sf_fail(SF_ERR_SHAPE, "power iteration needs an even nx");
     SF_TRY(k_apply_op(L, w_id, v_id, a, b));
-    zero_scalar<<<1, 1, 0, L->stream>>>(sumsq);
+    sf_launch(zero_scalar, 1, 1, 0, L->stream, sumsq);
     SF_LAUNCHED();
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
-        dinv_scale_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[w_id], depth, sumsq);
+        sf_launch(dinv_scale_pair_kernel, g, dim3(PX, PY), 0, L->stream, v, v.f[w_id], depth, sumsq);
         SF_LAUNCHED();
     }
     if (L->comm && L->comm->kind != 0 && L->nparts > 1)
@@ -604,20 +604,20 @@ sf_status k_power_step(sf_level* L, int v_id, int w_id, double a, double b, doub
         PV v = sf_view(L, p);
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
-        scale_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[v_id], v.f[w_id], sumsq, depth);
+        sf_launch(scale_pair_kernel, g, dim3(PX, PY), 0, L->stream, v, v.f[v_id], v.f[w_id], sumsq, depth);
         SF_LAUNCHED();
     }
     return sf_check_launch("power_step");
 }
 
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst) {
-    zero_scalar<<<1, 1, 0, L->stream>>>(dst);
+    sf_launch(zero_scalar, 1, 1, 0, L->stream, dst);
     SF_LAUNCHED();
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         int depth;
         dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
-        norm_pair_kernel<<<g, dim3(PX, PY), 0, L->stream>>>(v, v.f[field], kind, depth, dst);
+        sf_launch(norm_pair_kernel, g, dim3(PX, PY), 0, L->stream, v, v.f[field], kind, depth, dst);
         SF_LAUNCHED();
     }
     return sf_check_launch("norm_pair");

@@ -486,10 +486,10 @@ sf_status sf_norm_async(sf_level* L, int field, int kind, double* dst) {
 // A device scalar -> hscratch[slot] through mapped pinned memory, written by a
 // one-thread kernel: no copy-engine transfer, so the per-cycle convergence
 // scalar never queues behind bulk PCIe copies (sf_solve_stream).
-static __global__ void scalar_to_host_kernel(const double* src, double* dst) { *dst = *src; }
+static __global__ void scalar_to_host_kernel(const double* src, double* dst) { pdl_wait(); *dst = *src; }
 
 sf_status sf_scalar_to_host(sf_level* L, const double* src, int slot) {
-    scalar_to_host_kernel<<<1, 1, 0, L->stream>>>(src, L->hscratch_dev + slot);
+    sf_launch(scalar_to_host_kernel, 1, 1, 0, L->stream, src, L->hscratch_dev + slot);
     SF_LAUNCHED();
     return sf_check_launch("scalar_to_host");
 }
@@ -504,4 +504,10 @@ extern "C" sf_status sf_norm(sf_level* L, int field, int kind, double* out) {
     double v = L->hscratch[0];
     *out = (kind == SF_NORM_L2) ? sqrt(v) : v;
     return SF_OK;
+}
+
+// programmatic stream serialisation on every launch unless SF_PDL=0 (sf_internal.h)
+bool sf_pdl_on() {
+    static const int v = getenv("SF_PDL") ? atoi(getenv("SF_PDL")) : 1;
+    return v != 0;
 }

@@ -461,7 +461,7 @@ static sf_status run(sf_mg* m, int kind) {
 }
 
 // ---------------------------------------------------------------- device loop
-static __global__ void loop_init_kernel(LoopCtl* c, const LoopHost* h, const double* fn, int done0) {
+static __global__ void loop_init_kernel(LoopCtl* c, const LoopHost* h, const double* fn, int done0) { pdl_wait();
     c->rtol = h->rtol;
     c->max_cycles = h->max_cycles;
     c->fn = *fn;
@@ -472,7 +472,7 @@ static __global__ void loop_init_kernel(LoopCtl* c, const LoopHost* h, const dou
 
 // After a first pair's fused check: rmax = max|F - A U| of the iterate after
 // `done` cycles (the same decision as sf_solve's host loop, made on the device).
-static __global__ void loop_check_kernel(LoopCtl* c, const double* rmax, cudaGraphConditionalHandle h) {
+static __global__ void loop_check_kernel(LoopCtl* c, const double* rmax, cudaGraphConditionalHandle h) { pdl_wait();
     const int d = c->done;
     unsigned cont = 1;
     const double fn = c->fn;
@@ -504,7 +504,7 @@ static __global__ void loop_check_kernel(LoopCtl* c, const double* rmax, cudaGra
 }
 
 // results -> mapped host memory (posted writes: nothing queues behind bulk copies)
-static __global__ void loop_publish_kernel(const LoopCtl* c, LoopHost* h) {
+static __global__ void loop_publish_kernel(const LoopCtl* c, LoopHost* h) { pdl_wait();
     const int n = min(c->done, SF_LOOP_HIST);
     for (int i = threadIdx.x; i < n; i += blockDim.x) h->hist[i] = c->hist[i];
     if (threadIdx.x == 0) {
@@ -571,7 +571,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
     if (cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) != cudaSuccess) fail();
     if (ok && sf_norm_async(L, SF_F, SF_NORM_MAX, L->dscratch + 2) != SF_OK) fail();
     if (ok) {
-        loop_init_kernel<<<1, 1, 0, st>>>(m->lctl, m->lhost_dev, L->dscratch + 2, fc ? 1 : 0);
+        sf_launch(loop_init_kernel, 1, 1, 0, st, m->lctl, m->lhost_dev, L->dscratch + 2, fc ? 1 : 0);
         SF_LAUNCHED();
     }
     if (ok && fc && fcyc(m) != SF_OK) fail();
@@ -585,7 +585,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
             fail();
     }
     if (ok) {
-        loop_check_kernel<<<1, 1, 0, st>>>(m->lctl, L->dscratch, h);
+        sf_launch(loop_check_kernel, 1, 1, 0, st, m->lctl, L->dscratch, h);
         SF_LAUNCHED();
         cudaStreamCaptureStatus cs;
         const cudaGraphNode_t* deps = nullptr;
@@ -613,7 +613,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
     if (ok && vcyc(m, 0, true) != SF_OK) fail();
     if (ok && first_pair(m) != SF_OK) fail();
     if (ok) {
-        loop_check_kernel<<<1, 1, 0, st>>>(m->lctl, L->dscratch, h);
+        sf_launch(loop_check_kernel, 1, 1, 0, st, m->lctl, L->dscratch, h);
         SF_LAUNCHED();
         cudaGraph_t bo = nullptr;
         if (cudaStreamEndCapture(st, &bo) != cudaSuccess) fail();
@@ -623,7 +623,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
                                             cudaStreamCaptureModeThreadLocal) != cudaSuccess)
         fail();
     if (ok) {
-        loop_publish_kernel<<<1, 32, 0, st>>>(m->lctl, m->lhost_dev);
+        sf_launch(loop_publish_kernel, 1, 32, 0, st, m->lctl, m->lhost_dev);
         SF_LAUNCHED();
         cudaGraph_t go = nullptr;
         if (cudaStreamEndCapture(st, &go) != cudaSuccess) fail();

@@ -102,6 +102,36 @@ sf_status sf_fail(sf_status s, const char* fmt, ...);
         if (s_ != SF_OK) return s_;                 \
     } while (0)
 #define SF_LAUNCHED() sf_count_launch()
+
+// ------------------------------------------------------------------ launches
+// Every kernel is launched with programmatic stream serialisation (PDL): the
+// next kernel of the stream may be scheduled onto SMs the previous one has
+// left while that one drains, and runs its prologue up to pdl_wait(), which
+// blocks until the previous grid has completed and its writes are visible.
+// Every kernel calls pdl_wait() before touching global memory, so stream
+// order semantics are unchanged; only launch latency is hidden.  SF_PDL=0
+// launches without the attribute (A/B).
+__device__ __forceinline__ void pdl_wait() {
+#if defined(__CUDA_ARCH__) && __CUDA_ARCH__ >= 900
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+}
+bool sf_pdl_on();
+template <typename... K, typename... A>
+inline cudaError_t sf_launch(void (*k)(K...), dim3 g, dim3 b, size_t smem, cudaStream_t s,
+                             A&&... args) {
+    cudaLaunchConfig_t c = {};
+    c.gridDim = g;
+    c.blockDim = b;
+    c.dynamicSmemBytes = smem;
+    c.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    c.attrs = at;
+    c.numAttrs = sf_pdl_on() ? 1 : 0;
+    return cudaLaunchKernelEx(&c, k, static_cast<A&&>(args)...);
+}
 void sf_count_launch(long long n = 1);
 sf_status sf_check_launch(const char* what);
 
