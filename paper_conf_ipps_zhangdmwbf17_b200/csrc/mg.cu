@@ -10,6 +10,7 @@
 // so a whole V-cycle (+ its convergence residual and norm) is captured once as
 // a CUDA graph and replayed: levels <= 64^3 are launch-latency bound.
 #include <cmath>
+#include <cstdlib>
 
 #include "sf_internal.h"
 
@@ -525,8 +526,21 @@ static sf_status first_pair(sf_mg* m) {   // first_pair_check without the host c
     return SF_OK;
 }
 
+// Kernel nodes inside a graph with conditional nodes are invisible to Nsight
+// Compute ("not supported for profiling"), so under a profiler's injection
+// (the variables Nsight tools set in the target process) the solve uses the
+// host loop: the same kernels in the same order, one graph per cycle half.
+// SF_DEVICE_LOOP=0 forces the host loop.
+static bool device_loop_env() {
+    static const bool on = !getenv("CUDA_INJECTION64_PATH") &&
+                           !getenv("NV_COMPUTE_PROFILER_PERFWORKS_DIR") &&
+                           !getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE") &&
+                           !(getenv("SF_DEVICE_LOOP") && atoi(getenv("SF_DEVICE_LOOP")) == 0);
+    return on;
+}
+
 static bool loop_allowed(const sf_mg* m) {
-    return !m->loop_failed && graphs_allowed(m) && fused_check_ok(m) &&
+    return device_loop_env() && !m->loop_failed && graphs_allowed(m) && fused_check_ok(m) &&
            !(m->lv[0]->comm && m->lv[0]->comm->kind == 1);   // NCCL: host-side proxies
 }
 
