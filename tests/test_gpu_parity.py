@@ -386,6 +386,26 @@ def test_c2_solve_parity(sf, oracle, fcycle):
     assert abs(np.abs(u - ue).max() - 5.19e-7) < 0.05e-6
 
 
+@pytest.mark.parametrize("shape", [(32, 16, 64), (64, 32, 32), (32, 64, 32)])
+@pytest.mark.parametrize("use_graph", [0, 1])
+def test_noncube_solve_parity(sf, oracle, shape, use_graph):
+    """Non-cube boxes (C5's per-GPU shapes are not cubes): F-cycle + V-cycles to
+    1e-10 through the host loop and the device loop, same cycle count as the
+    oracle, u within 1e-10.  (Hierarchies whose coarsest box would exceed 64
+    cells are rejected with SF_ERR_SHAPE by sf_mg_plan -- reading R-8.)"""
+    nz, ny, nx = shape
+    L, M, O = mg_pair(sf, oracle, None, shape=shape, use_graph=use_graph)
+    _, f = I.manufactured(nx, ny, nz, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    st, cyc, hist = M.solve(fcycle=True, rtol=1e-10)
+    u_o, hist_o = O.solve(f, fcycle=True, rtol=1e-10)
+    assert cyc == len(hist_o)
+    assert hist[-1] < 1e-10
+    # relres entries agree to rounding of max|f - Au| (~1e-16 of max|f|)
+    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-14)
+    assert rel(L.download(sf.SF_U), u_o) < 1e-10
+
+
 def test_solve_graph_replay_stable(sf, oracle):
     """Repeated solves through the captured CUDA graphs give identical results."""
     n = 32
