@@ -557,7 +557,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
     std::vector<std::vector<SfPart>> saved;
     for (sf_level* lv : m->lv) saved.push_back(lv->parts);
     long long c0, c1, c2, c3;
-    cudaGraph_t g = nullptr;
+    cudaGraph_t g = nullptr, body = nullptr;   // body: owned by the WHILE node
     cudaGraphExec_t ge = nullptr;
     bool ok = true;
     auto fail = [&]() {
@@ -565,7 +565,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
         if (cudaStreamIsCapturing(st, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
             cudaGraph_t junk = nullptr;
             cudaStreamEndCapture(st, &junk);
-            if (junk && junk != g) cudaGraphDestroy(junk);
+            if (junk && junk != g && junk != body) cudaGraphDestroy(junk);
         }
         cudaGetLastError();
         ok = false;
@@ -611,7 +611,6 @@ static sf_status build_loop(sf_mg* m, int fc) {
     }
     if (ok && cudaStreamEndCapture(st, &g) != cudaSuccess) fail();
     sf_launch_count(&c1, 0);
-    cudaGraph_t body = nullptr;
     if (ok) {
         cudaGraphNodeParams p = {};
         p.type = cudaGraphNodeTypeConditional;
