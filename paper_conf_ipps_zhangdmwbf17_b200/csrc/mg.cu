@@ -623,6 +623,7 @@ static sf_status build_loop(sf_mg* m, int fc) {
     if (ok && cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0,
                                             cudaStreamCaptureModeThreadLocal) != cudaSuccess)
         fail();
+    if (ok && getenv("SF_TEST_LOOP_FAIL")) fail();   // tests: a capture failing mid-body
     if (ok && vcyc(m, 0, true) != SF_OK) fail();
     if (ok && first_pair(m) != SF_OK) fail();
     if (ok) {

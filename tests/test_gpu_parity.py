@@ -554,6 +554,27 @@ def test_device_loop_equals_host_loop(sf, oracle, fcycle, parts):
     assert out[1][3] == out[0][3] + 1
 
 
+def test_device_loop_capture_failure_falls_back(sf, oracle, monkeypatch):
+    """A device-loop capture that fails inside the WHILE body leaves the level
+    mappings intact and the solve runs the host loop: same iterate and cycles
+    as a hierarchy that never tried."""
+    n = 32
+    out = []
+    for fail in (False, True):
+        if fail:
+            monkeypatch.setenv("SF_TEST_LOOP_FAIL", "1")
+        L, M, O = mg_pair(sf, oracle, n)
+        _, f = I.manufactured(n, n, n, 1.0, 1.0)
+        L.upload(sf.SF_F, f)
+        st, cyc, hist = M.solve(fcycle=True, rtol=1e-10)
+        L.upload(sf.SF_U, np.zeros((n, n, n)))
+        st, cyc2, hist2 = M.solve(fcycle=True, rtol=1e-10)   # replay / host loop again
+        out.append((L.download(sf.SF_U), cyc, hist, cyc2))
+    assert out[0][1] == out[1][1] == out[0][3] == out[1][3]
+    assert out[0][2] == out[1][2]
+    assert np.array_equal(out[0][0], out[1][0])
+
+
 @pytest.mark.parametrize("use_graph", [0, 1])
 def test_solve_zero_and_nan_rhs(sf, oracle, use_graph):
     """f = 0 gives u = 0 after zero cycles; a NaN in f is reported, not solved."""
