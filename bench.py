@@ -288,6 +288,10 @@ def main():
     for _ in range(args.warmup):
         st, cyc, hist = step()
     sf.sf_launch_count(reset=True)
+    # live duration of the dominant kernel inside the timed region: the fused
+    # pair stamps %globaltimer per launch on the finest level (CUDA events cannot
+    # bracket a kernel node of a graph)
+    sf.sf_level_pair_timing(L.handle, 1)
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     prof = os.environ.get("SF_PROFILE_TIMED") == "1"   # ncu --profile-from-start off
@@ -302,6 +306,7 @@ def main():
         if prof:
             torch.cuda.cudart().cudaProfilerStop()
     launches = sf.sf_launch_count(reset=True)
+    live_pair_ms, live_pairs = sf.sf_level_pair_timing(L.handle, 0)
     t = max_over_ranks(e0.elapsed_time(e1) / 1e3)
     value = dof_local * world * args.steps / t
     ms_step = t / args.steps * 1e3
@@ -325,22 +330,35 @@ def main():
         pk, pk_src = peaks()
         fine_pair = side.get("fine_pair_ms")
         roof = None
-        if fine_pair:
+        if live_pairs:
+            # at N > 1 every fine pair is two launches (interior z-chunks beside the
+            # halo exchange, then the boundary chunks): time per complete pair
+            n_pairs = live_pairs // 2 if world > 1 else live_pairs
+            pair_ms = live_pairs * live_pair_ms / max(1, n_pairs)
             alg = GSRB_BYTES_PER_CELL * dof_local
-            ach = alg / (fine_pair / 1e3) / 1e9
+            ach = alg / (pair_ms / 1e3) / 1e9
             tr = ncu_traffic().get(f"{nx}x{ny}x{nz // world}")
             kb = GSRB_KERNEL_BYTES_PER_CELL * dof_local
             roof = {"bound": "hbm", "achieved": ach, "peak": pk, "unit": "GB/s",
                     "frac": ach / pk, "traffic": tr,
-                    "kernel": "gsrb_pair_tma_kernel (colour-fused RB pair, finest level)",
+                    "kernel": "gsrb_pair_tma_kernel (colour-fused RB pair, finest level; all four "
+                              "variants: plain, check-fused RESID/BRES, P0-fused INTERP)",
                     "algorithmic_bytes_per_launch": alg,
                     "algorithmic_basis": "64 B/cell per RB pair (PAPER.md:669-672, SURVEY 8d)",
                     "kernel_compulsory_bytes_per_launch": kb,
-                    "frac_of_kernel_compulsory": kb / (fine_pair / 1e3) / 1e9 / pk,
+                    "frac_of_kernel_compulsory": kb / (pair_ms / 1e3) / 1e9 / pk,
                     "note": "lambda-form update reads 56 of the paper's 64 B/cell (alpha enters "
-                            "only through lambda = 1/diag(A)); traffic = ncu DRAM bytes per launch",
-                    "launch_ms": fine_pair, "peak_source": pk_src,
-                    "share_of_step": side.get("fine_pair_share")}
+                            "only through lambda = 1/diag(A)); traffic = ncu DRAM bytes per launch "
+                            "(plain variant)",
+                    "launch_ms": pair_ms,
+                    "launch_ms_how": "mean per RB pair over the finest level's fused-pair "
+                                     "launches inside the timed region (in-kernel %globaltimer, "
+                                     "first CTA start to last CTA end; sf_level_pair_timing)",
+                    "launches_in_timed_region": live_pairs, "peak_source": pk_src,
+                    "share_of_step": live_pairs * live_pair_ms / (t * 1e3),
+                    "isolated_plain_pair_ms": fine_pair,
+                    "isolated_plain_pair_frac": (alg / (fine_pair / 1e3) / 1e9 / pk
+                                                 if fine_pair else None)}
         line = {
             "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
             "value": value, "unit": "DOF/s", "n_gpus": world, "steps": args.steps,

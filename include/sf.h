@@ -239,6 +239,13 @@ sf_status sf_lambda_max(sf_level* level, int v, double a, double b, int iters, i
 /* A10: norm of the interior over all parts/ranks; syncs. */
 sf_status sf_norm(sf_level* level, int field, int kind, double* out);
 sf_status sf_sync(sf_level* level);
+/* Live duration of the colour-fused RB-pair kernel (A5) on this level, for the
+ * roofline measured inside a timed region: op 1 resets and arms an in-kernel
+ * timer (per launch: first CTA start to last CTA end on the global timer,
+ * booked by the last CTA), op 0 disarms it and returns the mean ms per launch
+ * and the launch count since arming.  Both ops synchronise the level's stream;
+ * the timer works inside captured graphs (it lives in the level's scratch). */
+sf_status sf_level_pair_timing(sf_level* level, int op, double* mean_ms, long long* count);
 
 /* -------------------------------------------------------------- multigrid (A9)
  * sf_mg_create: builds the hierarchy below `finest` (which must hold ALPHA and

@@ -238,7 +238,14 @@ template <bool RESID, bool INTERP, bool BRES>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
-                     CoarseView cv, int c0, int cstride) { pdl_wait();
+                     CoarseView cv, int c0, int cstride, unsigned long long* ts) { pdl_wait();
+    // live timing (sf_level_pair_timing): thread 0 of every CTA stamps its start
+    // and end on the global timer; the last CTA to finish books end - start
+    bool timing = false;
+    if (threadIdx.x == 0 && *(volatile unsigned long long*)ts != 0ull) {
+        timing = true;
+        atomicMin(&ts[1], gtimer());
+    }
     constexpr int RING_PER_WARP = (NRING + NWARP - 1) / NWARP;   // 6 (32x16) / 9 (64x8)
     extern __shared__ __align__(128) double sm[];
     double* Xs = sm;                                  // [NXS][XH][W]
@@ -480,6 +487,19 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
     }
+    if (timing) {
+        atomicMax(&ts[2], gtimer());
+        __threadfence();
+        if (atomicAdd(&ts[3], 1ull) == gridDim.x - 1) {   // every CTA has stamped
+            __threadfence();
+            const unsigned long long t0 = atomicAdd(&ts[1], 0ull), t1 = atomicAdd(&ts[2], 0ull);
+            ts[5] += t1 - t0;
+            ts[4] += 1;
+            ts[1] = ~0ull;
+            ts[2] = 0ull;
+            ts[3] = 0ull;
+        }
+    }
     if (RESID || BRES) {   // CTA max -> one atomic (bit order = numeric order for |r|; NaN wins)
         __shared__ unsigned long long wmax[NWARP];
         for (int o2 = 16; o2 > 0; o2 >>= 1) {
@@ -629,7 +649,8 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         double* xo = v.f[xout];
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
     sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
-                                                                items, rmax, cvw, c0, cstride)
+                                                                items, rmax, cvw, c0, cstride, \
+              (unsigned long long*)(L->dscratch + SF_TS_OFF))
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);
         else if (rmode == SF_RM_OUTPUT_BLACK) SF_LAUNCH_PAIR(false, false, true);

@@ -511,3 +511,25 @@ bool sf_pdl_on() {
     static const int v = getenv("SF_PDL") ? atoi(getenv("SF_PDL")) : 1;
     return v != 0;
 }
+
+// Live duration of the colour-fused pair kernel on this level (SF_TS_OFF slots
+// of the level's device scratch; gsrb_fused.cu stamps them when armed).
+extern "C" sf_status sf_level_pair_timing(sf_level* L, int op, double* mean_ms, long long* count) {
+    if (!L || (op != 0 && op != 1)) return sf_fail(SF_ERR_INVALID, "NULL level or bad op");
+    unsigned long long* ts = (unsigned long long*)(L->dscratch + SF_TS_OFF);
+    if (op == 1) {
+        static const unsigned long long arm[6] = {1ull, ~0ull, 0ull, 0ull, 0ull, 0ull};
+        SF_CUDA(cudaMemcpyAsync(ts, arm, sizeof(arm), cudaMemcpyHostToDevice, L->stream));
+        SF_CUDA(cudaStreamSynchronize(L->stream));
+        return SF_OK;
+    }
+    unsigned long long h[6];
+    SF_CUDA(cudaMemcpyAsync(h, ts, sizeof(h), cudaMemcpyDeviceToHost, L->stream));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    static const unsigned long long off = 0ull;
+    SF_CUDA(cudaMemcpyAsync(ts, &off, sizeof(off), cudaMemcpyHostToDevice, L->stream));
+    SF_CUDA(cudaStreamSynchronize(L->stream));
+    if (count) *count = (long long)h[4];
+    if (mean_ms) *mean_ms = h[4] ? (double)h[5] / (double)h[4] * 1e-6 : 0.0;
+    return SF_OK;
+}

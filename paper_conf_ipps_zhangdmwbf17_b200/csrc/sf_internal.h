@@ -24,6 +24,10 @@
 // [8, 8 + SF_P2P_MAX_RANKS) all-reduce slots (doubles)
 #define SF_P2P_MAX_RANKS 64
 #define SF_SCRATCH_BYTES (256 + 8 * (8 + SF_P2P_MAX_RANKS))
+// dscratch slots: [0] fused-check max residual, [1] power-iteration sum, [2] max|F|
+// of the device solve loop, [8..13] live timing of the colour-fused pair
+// (u64: armed, min start, max end, finished CTAs, launches, sum of ns)
+#define SF_TS_OFF 8
 
 struct sf_comm {
     int kind;          // 0 = local (all parts in this process), 1 = NCCL, 2 = host+IPC (tests),

@@ -48,6 +48,12 @@ __device__ __forceinline__ void fence_proxy_async() {
 
 __device__ __forceinline__ int md(int k, int m) { return ((k % m) + m) % m; }
 
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
 // Gauss-Seidel update in lambda-form.  With lambda = Dinv the EXACT inverse
 // diagonal of A including the Dirichlet fold (reading R-4),
 //     x + lambda (rhs - A x)  ==  lambda (rhs + b h^-2 S),

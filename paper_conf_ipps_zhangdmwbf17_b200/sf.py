@@ -45,7 +45,7 @@ EXPORTS = [
     "sf_apply_laplacian", "sf_jacobi", "sf_smooth_chebyshev", "sf_lambda_max",
     "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
-    "sf_comm_create_p2p", "sf_smooth_residual_restrict",
+    "sf_comm_create_p2p", "sf_smooth_residual_restrict", "sf_level_pair_timing",
 ]
 
 
@@ -135,6 +135,7 @@ def lib():
         "sf_interpolate": (_i, [_vp, _i, _d, _vp, _i, _i]),
         "sf_norm": (_i, [_vp, _i, _i, _P]),
         "sf_sync": (_i, [_vp]),
+        "sf_level_pair_timing": (_i, [_vp, _i, _P, C.POINTER(C.c_longlong)]),
         "sf_mg_create": (_i, [C.POINTER(_vp), _vp, _d, _d, C.POINTER(MgOpts)]),
         "sf_mg_num_levels": (_i, [_vp, C.POINTER(_i)]),
         "sf_mg_level": (_i, [_vp, _i, C.POINTER(_vp)]),
@@ -356,6 +357,14 @@ def sf_norm(level, field, kind=SF_NORM_MAX):
 
 def sf_sync(level):
     _check(lib().sf_sync(level))
+
+
+def sf_level_pair_timing(level, op):
+    """op 1: arm the in-kernel timer of the colour-fused pair on this level;
+    op 0: disarm, returns (mean ms per launch, launches since arming)."""
+    ms, n = C.c_double(), C.c_longlong()
+    _check(lib().sf_level_pair_timing(level, int(op), C.byref(ms), C.byref(n)))
+    return ms.value, n.value
 
 
 def sf_mg_create(level, a, b, opts=None):
