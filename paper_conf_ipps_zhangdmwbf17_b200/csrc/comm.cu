@@ -14,6 +14,7 @@
 #include <mutex>
 
 #include <algorithm>
+#include <cmath>
 
 #include <cstdlib>
 #include <cstring>
@@ -527,8 +528,25 @@ sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int o
 sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, double b, double* rmax,
                            sf_level* C, int cf, int rmode) {
     const char* ev = getenv("SF_HALO_OVERLAP");
-    const int ov = ev ? atoi(ev) : 1;
-    const bool split = ov && L->nparts > 1 && L->comm && L->comm->kind != 2 && L->lnz >= 24;
+    const int ov = ev ? atoi(ev) : -1;   // 1 always split, 0 never, -1 (default) by cost
+    bool split = ov != 0 && L->nparts > 1 && L->comm && L->comm->kind != 2 && L->lnz >= 24;
+    if (split && ov < 0) {
+        // Overlap pays when the exchange it hides costs more than the boundary
+        // launch it adds: that launch walks 2 * tiles two-plane items (5 z steps
+        // each) over the resident CTAs, ~G * 512 cells * 56 B per step at
+        // ~5.5 TB/s; the exchange moves 2 neighbours x 2 planes, ~10 us of flag
+        // synchronisation plus the bytes at ~600 GB/s over NVLink (a copy
+        // engine on one device: ~3 us + 2.5 TB/s).  With NVLink both grow with
+        // the plane area at similar rates (bench's 512^2..1024^2 slabs: no split),
+        // the fixed synchronisation cost makes small planes split.
+        const double plane = (double)L->nx * L->ny;
+        const bool local = L->comm->kind == 0;
+        const double t_halo = (local ? 3e-6 : 10e-6) + 4.0 * plane * 8.0 / (local ? 2.5e12 : 6e11);
+        const double tiles = plane / 512.0, G = 148.0;
+        const double t_step = G * 512.0 * 56.0 / 5.5e12;
+        const double t_split = std::ceil(2.0 * tiles / G) * 5.0 * t_step;
+        split = t_halo > t_split;
+    }
     if (!split) {
         SF_TRY(sf_halo(L, xin, 2));
         return k_gsrb_pair_fused(L, xin, xout, rhs, a, b, rmax, C, cf, 0, 0, rmode);

@@ -238,7 +238,8 @@ template <bool RESID, bool INTERP, bool BRES>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
-                     CoarseView cv, int c0, int cstride, unsigned long long* ts) { pdl_wait();
+                     CoarseView cv, int c0, int cstride, unsigned long long* ts, int bd,
+                     int nch) { pdl_wait();
     // live timing (sf_level_pair_timing): thread 0 of every CTA stamps its start
     // and end on the global timer; the last CTA to finish books end - start
     bool timing = false;
@@ -266,7 +267,24 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         const int ci = item / ntiles, tile = item - ci * ntiles;
         const int chunk = c0 + ci * cstride;  // z-chunks of this launch (all / interior / boundary)
         const int x0 = (tile % ntx) * TX, y0 = (tile / ntx) * TY;
-        const int z0 = chunk * depth, z1 = min(z0 + depth, g.nz);
+        // bd = 0: uniform chunks of `depth` planes.  bd > 0 (split launches beside
+        // a halo exchange): chunks 0 and nch-1 are the bd planes at either end
+        // (the only ones whose stencils read ghost planes), the interior chunks
+        // cover the rest in `depth`-plane pieces
+        int z0, z1;
+        if (bd == 0) {
+            z0 = chunk * depth;
+            z1 = min(z0 + depth, g.nz);
+        } else if (chunk == 0) {
+            z0 = 0;
+            z1 = bd;
+        } else if (chunk == nch - 1) {
+            z0 = g.nz - bd;
+            z1 = g.nz;
+        } else {
+            z0 = bd + (chunk - 1) * depth;
+            z1 = min(z0 + depth, g.nz - bd);
+        }
         const int cx = SF_OX + x0 - 2;        // TMA x coordinate of the box
         const int cyx = y0, cyc = y0 + 1;     // TMA y coordinates (x box, coef box)
         const unsigned seq0 = seq;            // pre-bundle; bundle q -> seq0 + 2 + q - z0
@@ -618,12 +636,32 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     }
     const char* ed = getenv("SF_GSRB_DEPTH");   // tuning override
     if (ed && atoi(ed) > 0) best_d = std::min(L->lnz, atoi(ed));
-    if (phase) best_d = std::min(best_d, L->lnz / 3);
-    const int depth = best_d, nch = (L->lnz + depth - 1) / depth;
+    const int Gl = phase == 1 ? std::max(1, g_num_sms - reserve) * MINB : G;
+    // split launches (phase 1 interior beside the halo exchange, phase 2 the two
+    // boundary chunks after it): thin boundary chunks of bd planes, so the part
+    // that waits for the halo is small; the interior depth from the same cost
+    // model over the resident CTAs phase 1 gets
+    int bd = 0;
+    if (phase) {
+        const char* eb = getenv("SF_SPLIT_BD");
+        bd = std::max(2, std::min(eb && atoi(eb) > 0 ? atoi(eb) : 2, L->lnz / 3));
+        const int P = L->lnz - 2 * bd;
+        best = 1e30;
+        best_d = P;
+        for (int nc = 1; nc <= P; nc++) {
+            const int d = (P + nc - 1) / nc;
+            if (d < 8 && nc > 1) break;
+            const long it = (long)tiles * ((P + d - 1) / d);
+            const double cost = (double)((it + Gl - 1) / Gl) * (d + 3.0);
+            if (cost < best - 1e-9) { best = cost; best_d = d; }
+        }
+        if (ed && atoi(ed) > 0) best_d = std::min(P, atoi(ed));
+    }
+    const int depth = best_d;
+    const int nch = phase ? 2 + (L->lnz - 2 * bd + depth - 1) / depth : (L->lnz + depth - 1) / depth;
     const int c0 = phase == 1 ? 1 : 0;
     const int cstride = phase == 2 ? nch - 1 : 1;
     const int items = tiles * (phase == 0 ? nch : phase == 1 ? nch - 2 : 2);
-    const int Gl = phase == 1 ? std::max(1, g_num_sms - reserve) * MINB : G;
     const double bh2 = b / (L->h * L->h);
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
@@ -650,7 +688,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
     sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride, \
-              (unsigned long long*)(L->dscratch + SF_TS_OFF))
+              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch)
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);
         else if (rmode == SF_RM_OUTPUT_BLACK) SF_LAUNCH_PAIR(false, false, true);
