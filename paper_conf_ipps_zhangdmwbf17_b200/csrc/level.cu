@@ -405,11 +405,13 @@ bool gsrb_fused_supported(const sf_level* L) {
 sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, double b,
                             double* rmax, sf_level* C, int cf, int phase, int reserve, int rmode) {
     // 32x8 tiles with three CTAs per SM: 7.5 % faster than 32x16 with one at
-    // 256^3 and equal at 512^3 (profiles/r01/ab_256_ctas_per_sm.txt,
-    // ab_w4_512.txt); SF_GSRB_W4 = 0 / 1 forces the choice
-    static const int w4 = getenv("SF_GSRB_W4") ? atoi(getenv("SF_GSRB_W4")) : -1;
-    const bool small = (long)L->nx * L->ny * L->lnz <= (1L << 24);
-    if ((w4 == 1 || (w4 < 0 && small)) && gsrb_fused_supported_t32w4(L))
+    // 256^3, equal at 512^3 timed alone and 2 % faster inside the power-capped
+    // solve (profiles/r01/ab_256_ctas_per_sm.txt, ab_w4_512.txt,
+    // ab_w4_instep.txt): the default wherever the shape allows.  SF_GSRB_W4=0
+    // selects the 32x16 / 64x8 one-CTA builds (read per call: tests switch it)
+    const char* ew = getenv("SF_GSRB_W4");
+    const int w4 = ew ? atoi(ew) : -1;
+    if (w4 != 0 && gsrb_fused_supported_t32w4(L))
         return k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve, rmode);
     if (gsrb_fused_supported_t32(L))
         return k_gsrb_pair_fused_t32(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve, rmode);

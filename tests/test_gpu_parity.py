@@ -116,6 +116,33 @@ def test_gsrb_per_pair(sf, oracle, shape, kind):
         assert rel(L.download(sf.SF_U), x) < TOL
 
 
+@pytest.mark.parametrize("shape", [(24, 16, 64), (20, 8, 128), (12, 48, 96)])
+def test_fused_builds_agree(sf, oracle, shape, monkeypatch):
+    """The three builds of the fused pair (32x8 / 3 CTAs per SM, the default;
+    32x16 and 64x8 with one CTA, SF_GSRB_W4=0) match the oracle per pair and
+    each other bit for bit (explicit contractions shared by all builds)."""
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    coeffs = I.random_coeffs(nx, ny, nz, 5)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.0, 1.0, *coeffs)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    d = P.dinv()
+    outs = []
+    for mode in ("1", "0"):
+        monkeypatch.setenv("SF_GSRB_W4", mode)
+        L = make_level(sf, shape, coeffs)
+        sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+        L.upload(sf.SF_U, x)
+        L.upload(sf.SF_F, f)
+        xo = x
+        for _ in range(2):
+            sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED)
+            xo = P.smooth(xo, f, 1, dinv=d)
+            assert rel(L.download(sf.SF_U), xo) < TOL
+        outs.append(L.download(sf.SF_U))
+    assert np.array_equal(outs[0], outs[1])
+
+
 def test_fused_equals_colour(sf):
     shape = (48, 32, 128)
     nz, ny, nx = shape
