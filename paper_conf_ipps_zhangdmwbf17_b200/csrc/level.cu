@@ -410,7 +410,14 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
     // ab_w4_instep.txt): the default wherever the shape allows.  SF_GSRB_W4=0
     // selects the 32x16 / 64x8 one-CTA builds (read per call: tests switch it)
     const char* ew = getenv("SF_GSRB_W4");
-    const int w4 = ew ? atoi(ew) : -1;
+    int w4 = ew ? atoi(ew) : -1;
+    // the P0-fused variant keeps 5-deep prefetch on big levels (its end-of-step
+    // correction waits one bundle ahead): 32x16 build there, 0.25 % faster
+    // solve (r01/ab_interp_t32.txt); SF_INTERP_T32=0 disables
+    const char* ei = getenv("SF_INTERP_T32");
+    if (C && !(ei && atoi(ei) == 0) && w4 < 0 && (long)L->nx * L->ny * L->lnz > (1L << 24) &&
+        gsrb_fused_supported_t32(L))
+        w4 = 0;
     if (w4 != 0 && gsrb_fused_supported_t32w4(L))
         return k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, rmax, C, cf, phase, reserve, rmode);
     if (gsrb_fused_supported_t32(L))
