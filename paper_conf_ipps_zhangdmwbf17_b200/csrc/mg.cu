@@ -527,15 +527,20 @@ static sf_status first_pair(sf_mg* m) {   // first_pair_check without the host c
 }
 
 // Kernel nodes inside a graph with conditional nodes are invisible to Nsight
-// Compute ("not supported for profiling"), so under a profiler's injection
-// (the variables Nsight tools set in the target process) the solve uses the
+// Compute ("not supported for profiling"), and compute-sanitizer's racecheck /
+// synccheck abort the conditional graph ("unspecified launch failure"; memcheck
+// and initcheck run it clean), so under a profiler's or sanitizer's injection
+// (the variables those tools set in the target process) the solve uses the
 // host loop: the same kernels in the same order, one graph per cycle half.
-// SF_DEVICE_LOOP=0 forces the host loop.
+// SF_DEVICE_LOOP=0 forces the host loop, =1 the device loop even under a tool.
 static bool device_loop_env() {
-    static const bool on = !getenv("CUDA_INJECTION64_PATH") &&
-                           !getenv("NV_COMPUTE_PROFILER_PERFWORKS_DIR") &&
-                           !getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE") &&
-                           !(getenv("SF_DEVICE_LOOP") && atoi(getenv("SF_DEVICE_LOOP")) == 0);
+    static const bool on = [] {
+        const char* e = getenv("SF_DEVICE_LOOP");
+        if (e) return atoi(e) != 0;
+        return !getenv("CUDA_INJECTION64_PATH") && !getenv("NV_COMPUTE_PROFILER_PERFWORKS_DIR") &&
+               !getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE") &&
+               !getenv("NV_SANITIZER_INJECTION_TRANSPORT_TYPE");
+    }();
     return on;
 }
 

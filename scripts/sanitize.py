@@ -25,6 +25,7 @@ for n, parts in ((32, 1), (64, 1), (64, 2)):
 
 # halo exchange beside the interior chunks (2 parts x 24 planes), the pair +
 # residual + restriction kernel (SF_RR=1) and the 32x16 build (SF_GSRB_W4=0)
+os.environ["SF_HALO_OVERLAP"] = "1"   # force the split (2-plane boundary chunks)
 comm = sf.Comm.local(2)
 L = sf.Level(64, 32, 48, 1.0 / 64, comm=comm)
 sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
@@ -43,3 +44,13 @@ sf.sf_smooth_residual_restrict(F.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, s
 sf.sf_sync(F.handle)
 print("ok rr", flush=True)
 F.close(); C.close()
+
+# graphs on: the device-resident solve loop (WHILE node) and PDL launches
+os.environ.pop("SF_RR", None)
+L = sf.Level(32, 32, 32, 1.0 / 32)
+sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
+M = sf.MG(L, 1.0, 1.0)
+st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, raise_on_error=False)
+sf.sf_sync(L.handle)
+print("ok graph solve", cyc, flush=True)
+M.close(); L.close()
