@@ -331,10 +331,9 @@ def main():
         fine_pair = side.get("fine_pair_ms")
         roof = None
         if live_pairs:
-            # at N > 1 every fine pair is two launches (interior z-chunks beside the
-            # halo exchange, then the boundary chunks): time per complete pair
-            n_pairs = live_pairs // 2 if world > 1 else live_pairs
-            pair_ms = live_pairs * live_pair_ms / max(1, n_pairs)
+            # a pair split around a halo exchange (interior + boundary launch) is
+            # booked once with both launches' durations: mean = time per pair
+            pair_ms = live_pair_ms
             alg = GSRB_BYTES_PER_CELL * dof_local
             ach = alg / (pair_ms / 1e3) / 1e9
             tr = ncu_traffic().get(f"{nx}x{ny}x{nz // world}")

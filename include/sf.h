@@ -242,8 +242,9 @@ sf_status sf_sync(sf_level* level);
 /* Live duration of the colour-fused RB-pair kernel (A5) on this level, for the
  * roofline measured inside a timed region: op 1 resets and arms an in-kernel
  * timer (per launch: first CTA start to last CTA end on the global timer,
- * booked by the last CTA), op 0 disarms it and returns the mean ms per launch
- * and the launch count since arming.  Both ops synchronise the level's stream;
+ * booked by the last CTA), op 0 disarms it and returns the mean ms per RB pair
+ * and the number of pairs since arming (a pair split into interior and
+ * boundary launches around a halo exchange counts once, with both durations).  Both ops synchronise the level's stream;
  * the timer works inside captured graphs (it lives in the level's scratch). */
 sf_status sf_level_pair_timing(sf_level* level, int op, double* mean_ms, long long* count);
 

@@ -239,7 +239,7 @@ __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
                      CoarseView cv, int c0, int cstride, unsigned long long* ts, int bd,
-                     int nch) { pdl_wait();
+                     int nch, int tcount) { pdl_wait();
     // live timing (sf_level_pair_timing): thread 0 of every CTA stamps its start
     // and end on the global timer; the last CTA to finish books end - start
     bool timing = false;
@@ -512,7 +512,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             __threadfence();
             const unsigned long long t0 = atomicAdd(&ts[1], 0ull), t1 = atomicAdd(&ts[2], 0ull);
             ts[5] += t1 - t0;
-            ts[4] += 1;
+            ts[4] += tcount;   // a split pair (interior + boundary launch) counts once
             ts[1] = ~0ull;
             ts[2] = 0ull;
             ts[3] = 0ull;
@@ -688,7 +688,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
     sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride, \
-              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch)
+              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1)
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);
         else if (rmode == SF_RM_OUTPUT_BLACK) SF_LAUNCH_PAIR(false, false, true);

@@ -143,6 +143,36 @@ def test_fused_builds_agree(sf, oracle, shape, monkeypatch):
     assert np.array_equal(outs[0], outs[1])
 
 
+@pytest.mark.parametrize("parts,overlap", [(1, None), (2, "1"), (2, "0")])
+def test_pair_timing_counts_pairs(sf, parts, overlap, monkeypatch):
+    """sf_level_pair_timing books one entry per RB pair and part -- also when
+    the pair is split into interior and boundary launches around the halo --
+    and its mean agrees with CUDA events around back-to-back pairs."""
+    import torch
+    if overlap is not None:
+        monkeypatch.setenv("SF_HALO_OVERLAP", overlap)
+    shape = (48 * parts, 32, 64)
+    nz, ny, nx = shape
+    L = make_level(sf, shape, I.hpgmg_coeffs(nx, ny, nz), parts=parts)
+    sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+    L.upload(sf.SF_F, I.random_field(shape, 1))
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, sf.SF_SMOOTH_FUSED)   # warm
+    sf.sf_level_pair_timing(L.handle, 1)
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(L.stream)
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 3, sf.SF_SMOOTH_FUSED)
+    b.record(L.stream)
+    ms, n = sf.sf_level_pair_timing(L.handle, 0)
+    assert n == 3 * parts
+    ev = a.elapsed_time(b) / n
+    assert 0 < ms <= ev * 1.05 + 0.02
+    # disarmed: nothing more is booked
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED)
+    sf.sf_level_pair_timing(L.handle, 1)
+    ms2, n2 = sf.sf_level_pair_timing(L.handle, 0)
+    assert n2 == 0 and ms2 == 0.0
+
+
 def test_fused_equals_colour(sf):
     shape = (48, 32, 128)
     nz, ny, nx = shape
