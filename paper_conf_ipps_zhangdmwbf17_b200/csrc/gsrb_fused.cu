@@ -191,16 +191,20 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
 // = rhs - A x at the black cell AFTER its update, q - x_new/dinv with q the
 // quantity the update just formed (its red neighbours are final: this is the
 // black part of the residual of the pair's output).
+// The black cell's in-pair partner and its neighbours below / above are the
+// red cells this thread updated itself in the last three steps (rn_same,
+// rn_below, rn_above: the values it stored to shared memory), so they come
+// from registers.
 template <int SEL, bool BRES>
 __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx, int gy,
                                               const Geo& g, int gkm, double bh2, const double* rb,
-                                              double& bres) {
-    const double2 q2 = *(const double2*)&s.Xm[xo_];  // (red-new, black-old) of plane p-1
+                                              double& bres, double rn_below, double rn_same,
+                                              double rn_above) {
     double xw, xe;
     if (SEL == 0) {
-        xw = s.Xm[xo_ - 1]; xe = q2.y;
+        xw = s.Xm[xo_ - 1]; xe = rn_same;
     } else {
-        xw = q2.x; xe = s.Xm[xo_ + 2];
+        xw = rn_same; xe = s.Xm[xo_ + 2];
     }
     const int gxb = gx + SEL;
     if (gxb == 0) xw = 0.0;
@@ -208,12 +212,12 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
     const int col = xo_ + SEL;
     const double xs = (gy == 0) ? 0.0 : s.Xm[col - W];
     const double xn = (gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
-    const double xb = (gkm == 0) ? 0.0 : s.Xmm[col];
-    const double xt = (gkm == g.gnz - 1) ? 0.0 : s.Xk[col];
+    const double xb = (gkm == 0) ? 0.0 : rn_below;
+    const double xt = (gkm == g.gnz - 1) ? 0.0 : rn_above;
     const double q = gs_q(rb[7], bh2, sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
     const double bnew = __dmul_rn(rb[6], q);
     if (BRES) bres = __fma_rn(-bnew, inv_fast(rb[6]), q);
-    return SEL ? make_double2(q2.x, bnew) : make_double2(bnew, q2.y);
+    return SEL ? make_double2(rn_same, bnew) : make_double2(bnew, rn_same);
 }
 
 // Ring red cell at smem offsets (xo_, co_) (scalar loads; bounds in flags)
@@ -414,6 +418,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             __syncthreads();
         }
 
+        double rn0 = 0.0, rn1 = 0.0, rn2 = 0.0;   // red-new of planes t, t-1, t-2 at step t
         auto step = [&](int t, double* stash) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
@@ -447,10 +452,10 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             double rres = 0.0, bres = 0.0;
             if (sel == 0) {
                 if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
-                if (bin) o = black_pair<1, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres);
+                if (bin) o = black_pair<1, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             } else {
                 if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
-                if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres);
+                if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             }
             if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
                 const unsigned long long m2 = abits(rres);
@@ -470,6 +475,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 if (rin) Xw[xoff + sel] = rn;
                 if (ring) Xw[ro] = rr;
             }
+            rn2 = rn1;   // this thread's red-new values of planes t-1, t, t+1
+            rn1 = rn0;
+            rn0 = rn;
             if (bin)   // streaming store: do not evict halo lines other tiles still need
                 __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
