@@ -140,11 +140,13 @@ struct StepCtx {
 // red-new value; leaves the black cell's coefficients of the plane in nb
 // (bw, be, bs, bn, bb, bt, dinv, rhs).  RESID: rres = rhs - A x_in at the red
 // cell (A x = x(c)/dinv - b h^-2 S): the red part of the INPUT's residual.
+// The thread's own pair at planes q-1, q, q+1 (pb, xp2, pt) comes from
+// registers: each step loads only the pair of the newest plane.
 template <int SEL, bool RESID>
 __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
                                            int gy, const Geo& g, bool zlo, bool zhi, double bh2,
-                                           double* nb, double& rres) {
-    const double2 xp2 = *(const double2*)&s.Xk[xo_];
+                                           double* nb, double& rres, double2 pb, double2 xp2,
+                                           double2 pt) {
     const double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
     const double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
     const double2 bi2 = *(const double2*)&s.C[CA_BI * CARR + co_];
@@ -165,8 +167,8 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     if (gxr == g.nx - 1) xe = 0.0;
     const double xs = (gy == 0) ? 0.0 : s.Xk[col - W];
     const double xn = (gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
-    const double xb = zlo ? 0.0 : s.Xm[col];
-    const double xt = zhi ? 0.0 : s.Xp[col];
+    const double xb = zlo ? 0.0 : (SEL ? pb.y : pb.x);
+    const double xt = zhi ? 0.0 : (SEL ? pt.y : pt.x);
     double r, S;
     if (SEL == 0) {
         S = sum6(xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x);
@@ -419,6 +421,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
 
         double rn0 = 0.0, rn1 = 0.0, rn2 = 0.0;   // red-new of planes t, t-1, t-2 at step t
+        // own pair of planes t and t+1 at step t (INTERP: after their correction)
+        double2 pq0 = *(const double2*)&Xs[ix_0 * XSLOT + xoff];
+        double2 pq1 = *(const double2*)&Xs[ix_p1 * XSLOT + xoff];
         auto step = [&](int t, double* stash) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
@@ -450,11 +455,12 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             // planes t+1 and t-1 have the same parity: the black cell of
             // plane t-1 is the pair's other cell (position 1-sel)
             double rres = 0.0, bres = 0.0;
+            const double2 pn = *(const double2*)&s.Xp[xoff];   // own pair, plane t+2
             if (sel == 0) {
-                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
+                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn);
                 if (bin) o = black_pair<1, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             } else {
-                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres);
+                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn);
                 if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             }
             if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
@@ -478,6 +484,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             rn2 = rn1;   // this thread's red-new values of planes t-1, t, t+1
             rn1 = rn0;
             rn0 = rn;
+            pq0 = pq1;   // own pair (old values) of planes t+1, t+2 for the next step
+            pq1 = pn;
             if (bin)   // streaming store: do not evict halo lines other tiles still need
                 __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
