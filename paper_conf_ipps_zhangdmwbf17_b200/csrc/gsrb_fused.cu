@@ -146,14 +146,13 @@ template <int SEL, bool RESID>
 __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, int lane, int gx,
                                            int gy, const Geo& g, bool zlo, bool zhi, double bh2,
                                            double* nb, double& rres, double2 pb, double2 xp2,
-                                           double2 pt) {
+                                           double2 pt, double2 bkl, double2& bkh) {
     const double2 dv2 = *(const double2*)&s.C[CA_DV * CARR + co_];
     const double2 rh2 = *(const double2*)&s.C[CA_RH * CARR + co_];
     const double2 bi2 = *(const double2*)&s.C[CA_BI * CARR + co_];
     const double2 bjl = *(const double2*)&s.C[CA_BJ * CARR + co_];
     const double2 bjh = *(const double2*)&s.C[CA_BJ * CARR + co_ + W];
-    const double2 bkl = *(const double2*)&s.Klo[co_];
-    const double2 bkh = *(const double2*)&s.Khi[co_];
+    bkh = *(const double2*)&s.Khi[co_];   // beta_k(q+1); beta_k(q) was the last step's
     const double bie = s.C[CA_BI * CARR + co_ + 2];   // east face of the odd cell
     const int col = xo_ + SEL;
     double xw, xe;
@@ -424,6 +423,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         // own pair of planes t and t+1 at step t (INTERP: after their correction)
         double2 pq0 = *(const double2*)&Xs[ix_0 * XSLOT + xoff];
         double2 pq1 = *(const double2*)&Xs[ix_p1 * XSLOT + xoff];
+        double2 bkc = *(const double2*)&Ks[ik1 * CARR + coff];   // beta_k(t+1) at step t
         auto step = [&](int t, double* stash) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
@@ -456,11 +456,12 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             // plane t-1 is the pair's other cell (position 1-sel)
             double rres = 0.0, bres = 0.0;
             const double2 pn = *(const double2*)&s.Xp[xoff];   // own pair, plane t+2
+            double2 bkn = make_double2(0.0, 0.0);   // beta_k(t+2) at the own pair (R loads it)
             if (sel == 0) {
-                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn);
+                if (rin) rn = red_pair<0, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn, bkc, bkn);
                 if (bin) o = black_pair<1, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             } else {
-                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn);
+                if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn, bkc, bkn);
                 if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             }
             if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
@@ -486,6 +487,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             rn0 = rn;
             pq0 = pq1;   // own pair (old values) of planes t+1, t+2 for the next step
             pq1 = pn;
+            bkc = rin ? bkn : *(const double2*)&s.Khi[coff];   // beta_k(t+2): next step's bottom face
             if (bin)   // streaming store: do not evict halo lines other tiles still need
                 __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
