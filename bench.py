@@ -130,51 +130,64 @@ def oracle_threads():
         return os.cpu_count() or 1
 
 
-class OracleSampler:
-    """The CPU oracle's V-cycle on the same HPGMG-shaped workload, with its
-    OpenMP build on all host cores (the plane loops of oracle.c; same
-    arithmetic as the single-thread build, which the parity tests use)."""
+class OracleSolver:
+    """The CPU oracle solving the workload's problem exactly as a bench step
+    does (F-cycle, then V-cycles with 2+2 GSRB pairs, P0, exact bottom, until
+    ||f - Au||inf / ||f||inf < 1e-10), with its OpenMP build on all host cores
+    (the plane loops of oracle.c; same arithmetic as the single-thread build,
+    which the pins and parity tests use)."""
 
     def __init__(self, shape):
         from oracle import oracle as O
         from paper_conf_ipps_zhangdmwbf17_b200 import inputs as I
-        import numpy as np
         O.use_openmp(True)
         self.cores = O.lib().or_set_threads(oracle_threads())   # the threads it actually runs
         nx, ny, nz = shape
+        self.shape = shape
         h = I.level_h(nx, ny, nz)
         coeffs = I.hpgmg_coeffs(nx, ny, nz, h)
         _, self.f = I.manufactured(nx, ny, nz, 1.0, 1.0, h)
         self.mg = O.MG(nx, ny, nz, h, 1.0, 1.0, *coeffs)
         del coeffs
-        self.u = np.zeros(self.f.shape)
-        self.desc = (f"oracle V-cycle (2+2 GSRB pairs, P0, exact bottom) on {nx}x{ny}x{nz}, "
+        self.desc = (f"one complete oracle solve (F-cycle + V-cycles, 2+2 GSRB pairs, P0, exact "
+                     f"bottom, to 1e-10) of the HPGMG VC Helmholtz problem at {nx}x{ny}x{nz}, "
                      f"OpenMP build on {self.cores} host cores")
 
-    def vcycle_seconds(self):
+    def solve_seconds(self):
+        """(seconds, cycles, final relres) of one measured solve from u = 0."""
         t0 = time.perf_counter()
-        self.u = self.mg.vcycle(self.u, self.f)
-        return time.perf_counter() - t0
+        _, hist = self.mg.solve(self.f, fcycle=True, rtol=1e-10)
+        return time.perf_counter() - t0, len(hist), hist[-1] if hist else None
 
 
-def oracle_vcycle_sample(shape, reps=1):
-    """(seconds per V-cycle (min of reps), cores used, description)."""
-    s = OracleSampler(shape)
-    t = min(s.vcycle_seconds() for _ in range(reps))
-    return t, s.cores, s.desc
-
-
-def oracle_shape(shape):
-    """Full workload if the host has the memory (~22 GB for 512^3), else 256^3."""
+def host_memory_allows(shape):
+    """The oracle hierarchy of `shape` needs ~40 doubles per cell of host RAM."""
     try:
         import psutil
         avail = psutil.virtual_memory().available
     except Exception:
         avail = 0
-    cells = shape[0] * shape[1] * shape[2]
-    if avail > cells * 8 * 40:
-        return shape, 1.0
-    return (256, 256, 256), cells / 256**3
+    return avail > shape[0] * shape[1] * shape[2] * 8 * 40
+
+
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+# The reference arm's step: one complete oracle solve of the workload's problem
+# at 256^3 (1/8 of the 512^3 per-GPU DOFs): a few seconds on a many-core host,
+# so --steps 20 --warmup 5 ends within minutes.  Multigrid work per DOF is
+# size-independent (11-12 cycles at 256^3 and 512^3), so DOF/s of the sample
+# is the CPU's rate on the workload; bench's default run also measures one
+# 512^3 oracle solve (cpu_baseline) when the host has the memory.
+REFERENCE_SAMPLE = (256, 256, 256)
 
 
 def run_reference(args):
@@ -182,37 +195,32 @@ def run_reference(args):
     if rank != 0:
         return
     nx, ny, nz = dims_for(args.side, 1)
-    shp, scale = oracle_shape((nx, ny, nz))
-    smp = OracleSampler(shp)
-    cores, desc = smp.cores, smp.desc
-    steps = []
+    shp = REFERENCE_SAMPLE if nx * ny * nz > 256**3 else (nx, ny, nz)
+    smp = OracleSolver(shp)
+    cells = shp[0] * shp[1] * shp[2]
+    steps, cyc, rr = [], None, None
     for s in range(args.warmup + args.steps):
-        t = smp.vcycle_seconds()
+        t, cyc, rr = smp.solve_seconds()
         if s >= args.warmup:
-            steps.append(t * scale)
-    tv = sum(steps) / len(steps)
-    cyc = solve_cycles_guess()
-    t_solve = tv * (F_OVER_V + cyc)
-    val = (nx * ny * nz) / t_solve          # per-GPU-equivalent workload, one host
-    sample = (f"{desc}{'' if scale == 1 else f' scaled x{scale:g} to {nx}^3'}; solve = 1 F-cycle "
-              f"(= {F_OVER_V:.3f} V) + {cyc} V-cycles, per GPU-equivalent workload")
+            steps.append(t)
+    t_solve = sum(steps) / len(steps)
+    val = cells / t_solve
+    sample = (f"{smp.desc}: {cyc} cycles, final relres {rr:.2e}, {t_solve:.2f} s per solve "
+              f"(mean of {len(steps)} measured solves); each step is one such solve -- a "
+              f"{shp[0]}^3 sample of the {nx}x{ny}x{nz} per-GPU workload (same problem, solver "
+              f"and tolerance; DOF/s of the sample)")
     line = {"impl": "reference", "metric": "HPGMG-FV DOF/s (F-cycle + V-cycles to 1e-10)",
             "value": val, "unit": "DOF/s", "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_solve * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"C5 HPGMG-FV VC Helmholtz {nx}x{ny}x{nz} per GPU",
                        "global": [nx, ny, nz]},
-            "cpu_baseline": {"value": val, "unit": "DOF/s", "cores": cores, "kind": "oracle",
-                             "sample": sample},
+            "cpu_baseline": {"value": val, "unit": "DOF/s", "cores": smp.cores, "kind": "oracle",
+                             "sample": sample, "cpu_model": cpu_model(),
+                             "sample_shape": list(shp), "cycles": cyc},
             "e2e": {"value": val, "unit": "DOF/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
-
-
-def solve_cycles_guess():
-    """V-cycles after the F-cycle for the 512^3 workload (measured on the GPU
-    arm, which prints `cycles`; kept here for the oracle-only arm)."""
-    return int(os.environ.get("SF_SOLVE_VCYCLES", "10"))
 
 
 # ------------------------------------------------------------------ GPU arm
@@ -457,6 +465,7 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
     M.solve_stream([host_f] * reps, [host_u[k % 2] for k in range(reps)])
     barrier()
     te = max_over_ranks((time.perf_counter() - t0) / reps)
+    h2d_ms, solve_ms, d2h_ms, wall_ms = sf.sf_solve_stream_stats(M.handle)
     # the same, one step at a time with no overlap (upload, solve, download)
     def e2e_step():
         sf.sf_level_upload(L.handle, sf.SF_F, host_f.data_ptr())
@@ -474,7 +483,11 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
                          "H2D of f[k+1] and D2H of u[k-1] overlap solve k (wall clock, host "
                          "timer, incl. pipeline fill and drain)",
                   "serial_ms_per_step": ts * 1e3,
-                  "serial_value": dof_local * world / ts}
+                  "serial_value": dof_local * world / ts,
+                  "phases_ms": {"h2d_f": h2d_ms, "solve_incl_pack": solve_ms, "d2h_u": d2h_ms,
+                                "wall_per_rhs": wall_ms,
+                                "how": "CUDA events on the H2D, level and D2H streams inside "
+                                       "sf_solve_stream (sf_solve_stream_stats), rank 0"}}
 
     # BASELINE config 3: 256^3 GSRB smoother throughput (rank 0's GPU only)
     if rank == 0:
@@ -623,16 +636,19 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
                         "what": "64^3 VC Helmholtz V-cycle solve from u = 0 to 1e-10 (wall clock "
                                 "incl. the 2 MiB upload of u = 0 and the one host sync)"}
         if world == 1 and not args.no_cpu_baseline:
-            shp, scale = oracle_shape((nx, ny, nz))
-            tv, cores, desc = oracle_vcycle_sample(shp, reps=2)
-            tv *= scale
-            t_solve = tv * (F_OVER_V + (cyc - 1))
+            # one measured oracle solve of the workload itself (512^3: ~25 s on
+            # 16 cores) when the host has the memory, else the 256^3 sample
+            shp = (nx, ny, nz) if host_memory_allows((nx, ny, nz)) else REFERENCE_SAMPLE
+            smp = OracleSolver(shp)
+            t_s, cyc_o, rr_o = smp.solve_seconds()
+            cells_o = shp[0] * shp[1] * shp[2]
             out["cpu_baseline"] = {
-                "value": nx * ny * nz / t_solve, "unit": "DOF/s", "cores": cores,
-                "kind": "oracle",
-                "sample": (f"{desc}{'' if scale == 1 else f' x{scale:g}'}: {tv:.2f} s; solve "
-                           f"extrapolated as 1 F-cycle ({F_OVER_V:.3f} V) + {cyc - 1} V-cycles, "
-                           "the cycle counts this GPU run measured")}
+                "value": cells_o / t_s, "unit": "DOF/s", "cores": smp.cores, "kind": "oracle",
+                "cpu_model": cpu_model(), "sample_shape": list(shp), "cycles": cyc_o,
+                "seconds": t_s,
+                "sample": f"{smp.desc}: {cyc_o} cycles, final relres {rr_o:.2e}, {t_s:.2f} s "
+                          f"(measured, not extrapolated)"}
+            del smp
     out["fine_pair_share"] = (4 * (cyc - 1) + 4 * 1) * fine_pair / (
         (out["vcycle"]["ms"]) * (F_OVER_V + cyc - 1)) if fine_pair else None
     return out

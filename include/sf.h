@@ -142,10 +142,25 @@ sf_status sf_comm_create_hostipc(sf_comm** out, int nranks, int rank, sf_host_al
  * all-reduces are kernels that read the peers' memory directly and
  * synchronise through flags in device memory (no NCCL, no host round trip;
  * CUDA-graph capturable).  The host all-gather is used only at level
- * creation to exchange the IPC handles; same contract as hostipc. */
+ * creation to exchange the IPC handles; same contract as hostipc.  Every wait
+ * on a peer's flag is bounded (environment SF_P2P_TIMEOUT_S, default 60 s, on
+ * the GPU's global timer): a dead or hung peer makes the waiting kernel trap,
+ * and the next synchronising call returns SF_ERR_CUDA naming the flag, peer
+ * slot and op ("p2p peer wait timed out") instead of blocking forever; the
+ * CUDA context is unusable afterwards (the process should exit).  With the
+ * NCCL transport, synchronising calls poll ncclCommGetAsyncError and abort the
+ * communicator on an asynchronous error or after SF_NCCL_TIMEOUT_S (default
+ * 600 s), returning SF_ERR_NCCL. */
 sf_status sf_comm_create_p2p(sf_comm** out, int nranks, int rank, sf_host_allgather_fn allgather,
                              void* user);
 sf_status sf_comm_destroy(sf_comm* comm);
+/* Transport self-test (collective): with the NCCL transport, runs once on a few
+ * device doubles every collective the slab path uses -- ncclAllReduce (max,
+ * sum), ncclBroadcast, ncclAllGather and, for nranks > 1, grouped ring
+ * ncclSend/ncclRecv -- on `stream` (cudaStream_t), checks the values on the
+ * host and returns SF_ERR_NCCL on any failure or wrong value.  Other transports
+ * have nothing to check without a level: SF_OK.  Synchronises. */
+sf_status sf_comm_check(const sf_comm* comm, void* stream);
 /* number of parts in the job, parts local to this process, first local part */
 sf_status sf_comm_info(const sf_comm* comm, int* nparts, int* nlocal, int* first);
 
@@ -189,7 +204,11 @@ sf_status sf_apply_op(sf_level* level, int out, int x, double a, double b);
 /* A5: rb_pairs x (BC, red, BC, black) in place on field x with rhs field rhs
  * and the level's DINV.  Red = (i+j+k) even in
  * global 0-based cell indices (R-2).  x must be SF_U or SF_TMP when the fused
- * smoother is used.  kind: enum sf_smoother_kind. */
+ * smoother is used: it writes each pair into the other of U / TMP and swaps the
+ * two ids, so with x = SF_TMP and kind SF_SMOOTH_FUSED the buffer U named before
+ * the call is overwritten.  SF_SMOOTH_AUTO takes the fused kernel only for
+ * x = SF_U (TMP is then the clobbered scratch), otherwise the colour sweeps.
+ * kind: enum sf_smoother_kind. */
 sf_status sf_smooth_gsrb(sf_level* level, int x, int rhs, double a, double b, int rb_pairs, int kind);
 /* A6: res = rhs - A x */
 sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double b);
@@ -198,7 +217,7 @@ sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double
  * coarse.c_field = R_cell(rhs - A x) of the smoothed x.  By default a pair, a
  * residual into SF_R and a restriction produce it.  With the environment
  * variable SF_RR=1, on single-part levels with nx % 32 == 0, ny % 16 == 0 and
- * x = SF_U or SF_TMP, one kernel does all three in a single HBM pass and the
+ * x = SF_U, one kernel does all three in a single HBM pass and the
  * residual is never stored (the U/TMP ids are swapped as by the fused
  * smoother); it is measured slower on B200, hence opt-in.
  * x must differ from rhs, SF_R and SF_DINV.  coarse dims must be fine dims / 2
@@ -206,6 +225,17 @@ sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double
  * stream; the coarse level must be idle on its own stream. */
 sf_status sf_smooth_residual_restrict(sf_level* fine, int x, int rhs, double a, double b,
                                       sf_level* coarse, int c_field);
+/* A8 + A5, the head of V(l)'s post-smoothing:
+ * fine.x += P0(coarse.c_field) (piecewise-constant interpolation, prescale 1),
+ * then one RB pair on fine.x with rhs -- exactly sf_interpolate(P0, 1.0)
+ * followed by sf_smooth_gsrb(rb_pairs = 1).  With x = SF_U, rhs != SF_TMP and a
+ * level the colour-fused smoother supports, the correction is applied inside
+ * the fused pair's single HBM pass (TMP is clobbered and the U/TMP ids are
+ * swapped, as by the fused smoother); otherwise P0 then the smoother.  coarse
+ * dims must be fine dims / 2 (SF_ERR_SHAPE).  Enqueued on the fine level's
+ * stream; the coarse level must be idle on its own stream. */
+sf_status sf_interpolate_smooth(sf_level* fine, int x, int rhs, double a, double b,
+                                sf_level* coarse, int c_field);
 /* A7: coarse.c_field = R(fine.f_field); coarse dims must be fine dims / 2
  * (PAPER.md:293-297, 466-468).  kind: enum sf_restrict_kind. */
 sf_status sf_restrict(sf_level* coarse, int c_field, sf_level* fine, int f_field, int kind);
@@ -258,7 +288,8 @@ sf_status sf_level_pair_timing(sf_level* level, int op, double* mean_ms, long lo
  * sf_fcycle: one F-cycle from scratch for rhs F_0 into U_0, enqueued.
  * sf_solve: optional F-cycle, then V-cycles until ||F-AU||inf/||F||inf <
  *   rtol; fills *cycles and hist[0..*cycles-1] (may be NULL; caller array of
- *   max_cycles+1 doubles); syncs.  F = 0 gives U = 0 and *cycles = 0; a NaN/Inf
+ *   max_cycles+1 doubles); max_cycles < 1 is SF_ERR_INVALID; rtol <= 0 takes
+ *   opts->rtol; syncs.  F = 0 gives U = 0 and *cycles = 0; a NaN/Inf
  *   in F returns SF_ERR_NUMERIC with *cycles = 0.  With use_graph and the
  *   colour-fused smoother (max_cycles <= 256, no NCCL transport) the whole
  *   solve is ONE CUDA graph launch whose WHILE node is driven by the
@@ -290,12 +321,17 @@ sf_status sf_mg_destroy(sf_mg* mg);
  * sf_level_upload/download; pinned memory makes the copies asynchronous).
  * The host->device copy of f_{k+1} and the device->host copy of u_{k-1} run
  * on their own streams while solve k runs, through two packed device staging
- * buffers allocated for the call (2 x one field).  cycles[k] (may be NULL)
+ * buffers (2 x one field, allocated on the first call and kept by the
+ * hierarchy until sf_mg_destroy).  cycles[k] (may be NULL)
  * receives each solve's cycle count.  Synchronises; returns the first failing
  * solve's status (later right-hand sides are not solved).  Leaves F = f_{last}
  * and U = u_{last} on the level. */
 sf_status sf_solve_stream(sf_mg* mg, int fcycle, double rtol, int max_cycles, int n,
                           const double* const* host_f, double* const* host_u, int* cycles);
+/* Phase times of the last sf_solve_stream call (CUDA events on the three
+ * streams): stats[0] mean H2D copy of one f, [1] mean solve incl. (un)packing,
+ * [2] mean D2H copy of one u (ms), [3] host wall ms per right-hand side. */
+sf_status sf_solve_stream_stats(const sf_mg* mg, double stats[4]);
 
 /* -------------------------------------------------------------- measurement
  * Number of kernels libsf launched since the counter was last reset (host-side

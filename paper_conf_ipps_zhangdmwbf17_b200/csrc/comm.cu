@@ -11,7 +11,9 @@
 
 #include <cuda.h>
 
+#include <chrono>
 #include <mutex>
+#include <thread>
 
 #include <algorithm>
 #include <cmath>
@@ -36,6 +38,8 @@ struct NcclApi {
     decltype(&ncclAllGather) allGather;
     decltype(&ncclBroadcast) broadcast;
     decltype(&ncclGetErrorString) errStr;
+    decltype(&ncclCommGetAsyncError) asyncErr;
+    decltype(&ncclCommAbort) abort;
 };
 
 NcclApi g_nccl;
@@ -61,6 +65,8 @@ sf_status nccl_load() {
     SYM(allGather, "ncclAllGather");
     SYM(broadcast, "ncclBroadcast");
     SYM(errStr, "ncclGetErrorString");
+    SYM(asyncErr, "ncclCommGetAsyncError");
+    SYM(abort, "ncclCommAbort");
 #undef SYM
     g_nccl.h = h;
     return SF_OK;
@@ -178,13 +184,42 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
-__device__ __forceinline__ void wait_ge(const unsigned long long* p, unsigned long long v) {
-    while (ld_acquire_sys(p) < v) __nanosleep(64);
+__device__ __forceinline__ unsigned long long p2p_clock() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
 }
 
 struct P2PPeers {
     const unsigned long long* sync[SF_P2P_MAX_RANKS];   // peers' sync blocks (nullptr: not involved)
+    unsigned long long* err;        // mapped host word written before a timed-out wait traps
+    unsigned long long timeout_ns;  // bound of every wait on a peer's flag
 };
+
+// Wait until *p >= v.  A peer that never gets there (dead, hung, or not
+// running the same op sequence) must not wedge this GPU forever: after
+// timeout_ns on the global timer the waiting thread records (what, peer, op)
+// in mapped host memory and traps, which fails the stream with a CUDA error
+// that sf_stream_sync reports as SF_ERR_CUDA with that description.
+__device__ __forceinline__ void wait_ge(const unsigned long long* p, unsigned long long v,
+                                        const P2PPeers& pe, int peer, int what) {
+    if (ld_acquire_sys(p) >= v) return;
+    const unsigned long long t0 = p2p_clock();
+    unsigned ns = 32;
+    while (ld_acquire_sys(p) < v) {
+        __nanosleep(ns);
+        if (ns < 1024) ns *= 2;
+        if (p2p_clock() - t0 > pe.timeout_ns) {
+            if (pe.err) {
+                *(volatile unsigned long long*)pe.err =
+                    (1ull << 63) | ((unsigned long long)what << 56) |
+                    ((unsigned long long)(peer & 0xffff) << 40) | (v & 0xffffffffffull);
+                __threadfence_system();
+            }
+            __trap();
+        }
+    }
+}
 
 // op start: every CTA learns s; CTA 0 publishes ready; thread 0 of each CTA
 // waits for the peers' ready
@@ -195,7 +230,7 @@ __device__ __forceinline__ unsigned long long p2p_begin(unsigned long long* my, 
         const unsigned long long s = *(volatile unsigned long long*)&my[2] + 1;
         if (blockIdx.x == 0) st_release_sys(&my[0], s);
         for (int q = 0; q < npeers; q++)
-            if (pe.sync[q]) wait_ge(&pe.sync[q][0], s);
+            if (pe.sync[q]) wait_ge(&pe.sync[q][0], s, pe, q, 1);
         s_seq = s;
     }
     __syncthreads();
@@ -214,7 +249,7 @@ __device__ __forceinline__ void p2p_end(unsigned long long* my, const P2PPeers& 
             my[3] = 0;
             st_release_sys(&my[1], s);
             for (int q = 0; q < npeers; q++)
-                if (pe.sync[q]) wait_ge(&pe.sync[q][1], s);
+                if (pe.sync[q]) wait_ge(&pe.sync[q][1], s, pe, q, 2);
             *(volatile unsigned long long*)&my[2] = s;
         }
     }
@@ -273,6 +308,81 @@ __global__ void __launch_bounds__(256) p2p_gather_kernel(double* base, P2PPtrs p
     if (peer_top)
         for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < topcnt; i += stride) top[i] = peer_top[i];
     p2p_end(my, pe, nranks, s);
+}
+
+// process-wide mapped host word for the p2p timeout diagnosis (see wait_ge)
+static unsigned long long* g_err_host = nullptr;
+static unsigned long long* g_err_dev = nullptr;
+static std::mutex g_err_mu;
+
+static P2PPeers peers_init() {
+    P2PPeers pe = {};
+    {
+        std::lock_guard<std::mutex> lk(g_err_mu);
+        if (!g_err_host) {
+            void* h = nullptr;
+            void* d = nullptr;
+            if (cudaHostAlloc(&h, 64, cudaHostAllocMapped) == cudaSuccess &&
+                cudaHostGetDevicePointer(&d, h, 0) == cudaSuccess) {
+                memset(h, 0, 64);
+                g_err_host = (unsigned long long*)h;
+                g_err_dev = (unsigned long long*)d;
+            } else {
+                cudaGetLastError();
+            }
+        }
+    }
+    pe.err = g_err_dev;
+    static const double secs = getenv("SF_P2P_TIMEOUT_S") ? atof(getenv("SF_P2P_TIMEOUT_S")) : 60.0;
+    pe.timeout_ns = (unsigned long long)(std::max(secs, 1e-3) * 1e9);
+    return pe;
+}
+
+// Status of a synchronisation that returned e; a timed-out peer wait is named.
+static sf_status sync_failure(cudaError_t e, const char* what) {
+    const unsigned long long w = g_err_host ? *(volatile unsigned long long*)g_err_host : 0ull;
+    if (w >> 63)
+        return sf_fail(SF_ERR_CUDA,
+                       "%s: p2p peer wait timed out (%s flag of peer slot %d, op %llu; the peer "
+                       "rank is dead, hung or off the op sequence): %s",
+                       what, ((w >> 56) & 0x7f) == 1 ? "ready" : "consumed", (int)((w >> 40) & 0xffff),
+                       w & 0xffffffffffull, cudaGetErrorString(e));
+    return sf_fail(SF_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+// Host synchronisation of a level's stream.  With the NCCL transport the wait
+// polls ncclCommGetAsyncError (a peer's failure aborts the communicator instead
+// of blocking forever; SF_NCCL_TIMEOUT_S bounds the wait, default 600 s).
+sf_status sf_stream_sync(sf_level* L) {
+    const sf_comm* c = L->comm ? L->comm : L->rep_comm;
+    if (c && c->kind == 1 && c->nccl && g_nccl.asyncErr) {
+        static const double secs =
+            getenv("SF_NCCL_TIMEOUT_S") ? atof(getenv("SF_NCCL_TIMEOUT_S")) : 600.0;
+        const auto t0 = std::chrono::steady_clock::now();
+        for (;;) {
+            cudaError_t e = cudaStreamQuery(L->stream);
+            if (e == cudaSuccess) return SF_OK;
+            if (e != cudaErrorNotReady) return sync_failure(e, "stream");
+            ncclResult_t ar = ncclSuccess;
+            if (g_nccl.asyncErr((ncclComm_t)c->nccl, &ar) != ncclSuccess ||
+                (ar != ncclSuccess && ar != ncclInProgress)) {
+                g_nccl.abort((ncclComm_t)c->nccl);
+                const_cast<sf_comm*>(c)->nccl = nullptr;
+                return sf_fail(SF_ERR_NCCL, "NCCL asynchronous error: %s",
+                               g_nccl.errStr ? g_nccl.errStr(ar) : "?");
+            }
+            if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > secs) {
+                g_nccl.abort((ncclComm_t)c->nccl);
+                const_cast<sf_comm*>(c)->nccl = nullptr;
+                return sf_fail(SF_ERR_NCCL, "NCCL wait exceeded %.0f s (SF_NCCL_TIMEOUT_S); "
+                               "communicator aborted", secs);
+            }
+            std::this_thread::sleep_for(std::chrono::microseconds(50));
+        }
+    }
+    cudaError_t e = cudaStreamSynchronize(L->stream);
+    if (e != cudaSuccess) return sync_failure(e, "stream");
+    return SF_OK;
 }
 
 static unsigned long long* peer_sync(const sf_level* L, int r) {
@@ -355,6 +465,62 @@ extern "C" sf_status sf_comm_destroy(sf_comm* c) {
     return SF_OK;
 }
 
+// Transport self-test: every NCCL collective the slab path uses, once, on a
+// few device doubles, results checked on the host.
+extern "C" sf_status sf_comm_check(const sf_comm* c, void* stream) {
+    if (!c) return sf_fail(SF_ERR_INVALID, "NULL comm");
+    if (c->kind != 1) return SF_OK;
+    if (!c->nccl) return sf_fail(SF_ERR_NCCL, "communicator was aborted");
+    cudaStream_t s = (cudaStream_t)stream;
+    ncclComm_t nc = (ncclComm_t)c->nccl;
+    const int n = c->nranks, r = c->rank;
+    const int G = 4;   // all-gather doubles per rank
+    std::vector<double> h(8 + (size_t)G * n + 4, 0.0);
+    h[0] = r;          // all-reduce max
+    h[1] = r + 1;      // all-reduce sum
+    h[2] = (r == n - 1) ? 1000.0 + r : -1.0;   // broadcast from the last rank
+    h[3] = 100.0 + r;  // ring send
+    for (int i = 0; i < G; i++) h[8 + (size_t)G * r + i] = 10.0 * r + i;
+    double* d = nullptr;
+    SF_CUDA(cudaMalloc(&d, h.size() * sizeof(double)));
+    sf_status st = SF_OK;
+    auto nccl = [&](ncclResult_t e, const char* what) {
+        if (e != ncclSuccess && st == SF_OK)
+            st = sf_fail(SF_ERR_NCCL, "%s: %s", what, g_nccl.errStr ? g_nccl.errStr(e) : "?");
+    };
+    if (cudaMemcpyAsync(d, h.data(), h.size() * sizeof(double), cudaMemcpyHostToDevice, s) != cudaSuccess)
+        st = sf_fail(SF_ERR_CUDA, "upload");
+    if (st == SF_OK) nccl(g_nccl.allReduce(d, d, 1, ncclDouble, ncclMax, nc, s), "ncclAllReduce(max)");
+    if (st == SF_OK) nccl(g_nccl.allReduce(d + 1, d + 1, 1, ncclDouble, ncclSum, nc, s), "ncclAllReduce(sum)");
+    if (st == SF_OK) nccl(g_nccl.broadcast(d + 2, d + 2, 1, ncclDouble, n - 1, nc, s), "ncclBroadcast");
+    if (st == SF_OK)
+        nccl(g_nccl.allGather(d + 8 + (size_t)G * r, d + 8, G, ncclDouble, nc, s), "ncclAllGather");
+    if (st == SF_OK && n > 1) {   // ring point-to-point, as the halo exchange groups it
+        nccl(g_nccl.groupStart(), "ncclGroupStart");
+        if (st == SF_OK) nccl(g_nccl.send(d + 3, 1, ncclDouble, (r + 1) % n, nc, s), "ncclSend");
+        if (st == SF_OK) nccl(g_nccl.recv(d + 4, 1, ncclDouble, (r + n - 1) % n, nc, s), "ncclRecv");
+        nccl(g_nccl.groupEnd(), "ncclGroupEnd");
+    }
+    if (st == SF_OK &&
+        cudaMemcpyAsync(h.data(), d, h.size() * sizeof(double), cudaMemcpyDeviceToHost, s) != cudaSuccess)
+        st = sf_fail(SF_ERR_CUDA, "download");
+    if (st == SF_OK) {
+        sf_level tmp;   // a level shell carrying the stream and the comm for the polled wait
+        tmp.comm = c;
+        tmp.rep_comm = nullptr;
+        tmp.stream = s;
+        st = sf_stream_sync(&tmp);
+    }
+    cudaFree(d);
+    if (st != SF_OK) return st;
+    bool ok = h[0] == n - 1 && h[1] == 0.5 * n * (n + 1) && h[2] == 1000.0 + (n - 1);
+    for (int q = 0; q < n; q++)
+        for (int i = 0; i < G; i++) ok = ok && h[8 + (size_t)G * q + i] == 10.0 * q + i;
+    if (n > 1) ok = ok && h[4] == 100.0 + (r + n - 1) % n;
+    if (!ok) return sf_fail(SF_ERR_NCCL, "NCCL self-test returned wrong values");
+    return SF_OK;
+}
+
 extern "C" sf_status sf_comm_info(const sf_comm* c, int* nparts, int* nlocal, int* first) {
     if (!c) return sf_fail(SF_ERR_INVALID, "NULL comm");
     if (nparts) *nparts = c->nparts;
@@ -391,7 +557,7 @@ sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t stream) {
         const sf_comm* c = L->comm;
         const int r = c->rank, n = c->nranks;
         double* x = L->parts[0].f[field];
-        P2PPeers pe = {};
+        P2PPeers pe = peers_init();
         const double* lo_x = nullptr;
         const double* hi_x = nullptr;
         if (r > 0) { pe.sync[0] = peer_sync(L, r - 1); lo_x = peer_field(L, r - 1, x); }
@@ -441,7 +607,7 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part) {
     if (cm->kind == 3) {  // device-initiated gather over peer memory
         double* base = C->parts[0].f[field] + (long)SF_GZ * C->ks;
         const long cnt = (long)lnz_per_part * C->ks;
-        P2PPeers pe = {};
+        P2PPeers pe = peers_init();
         P2PPtrs pb = {};
         for (int q = 0; q < parts; q++)
             if (q != cm->rank) {
@@ -490,7 +656,7 @@ sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* cm, double* dev, int o
     if (!cm || cm->kind == 0 || cm->nranks == 1) return SF_OK;
     cudaStream_t s = L->stream;
     if (cm->kind == 3) {
-        P2PPeers pe = {};
+        P2PPeers pe = peers_init();
         P2PPtrs sl = {};
         for (int q = 0; q < cm->nranks; q++) {
             if (q != cm->rank) pe.sync[q] = peer_sync(L, q);

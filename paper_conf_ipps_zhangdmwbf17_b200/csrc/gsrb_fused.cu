@@ -119,7 +119,14 @@ struct CoarseView {
 struct Geo {
     int nx, ny, nz, z0, gnz;
     long js, ks;
+    int zmask;   // measurement knob (SF_DBG_ZMASK): planes aliased to q & zmask, 0 = off
 };
+
+// storage plane (TMA coordinate / store row) of plane q; with the measurement
+// knob every plane aliases one of zmask+1 planes, so the whole working set is
+// L2-resident and the kernel's SM-side throughput is measured (results are
+// meaningless then)
+__device__ __forceinline__ int zplane(const Geo& g, int q) { return (g.zmask ? (q & g.zmask) : q) + SF_GZ; }
 
 // Per-step state shared by the templated step bodies.
 struct StepCtx {
@@ -306,13 +313,13 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const unsigned b = mb_u + 8u * (sq % NMB);
             if (part == 0) {
                 mbar_expect_u(b, BUNDLE_BYTES);
-                tma3u(xs_u + 8u * (md(q + 1, NXS) * XSLOT), &mp.x, cx, cyx, q + 1 + SF_GZ, b);
+                tma3u(xs_u + 8u * (md(q + 1, NXS) * XSLOT), &mp.x, cx, cyx, zplane(g, q + 1), b);
             } else if (part == 5) {
-                tma3u(ks_u + 8u * (md(q + 1, NKS) * CARR), &mp.bk, cx, cyc, q + 1 + SF_GZ, b);
+                tma3u(ks_u + 8u * (md(q + 1, NKS) * CARR), &mp.bk, cx, cyc, zplane(g, q + 1), b);
             } else {
                 const unsigned c = cs_u + 8u * (md(q, NCS) * CSLOT + (part - 1) * CARR);
                 const CUtensorMap* m = part == 1 ? &mp.dv : part == 2 ? &mp.rh : part == 3 ? &mp.bi : &mp.bj;
-                tma3u(c, m, cx, cyc, q + SF_GZ, b);
+                tma3u(c, m, cx, cyc, zplane(g, q), b);
             }
         };
         auto issue = [&](int q) {
@@ -322,9 +329,9 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             fence_proxy_async();  // generic smem writes of the previous item before TMA reuse
             unsigned long long* b = &mbar[seq0 % NMB];
             mbar_expect(b, 2 * XBYTES + CBYTES);
-            tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 2 + SF_GZ, b);
-            tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, z0 - 1 + SF_GZ, b);
-            tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, z0 - 1 + SF_GZ, b);
+            tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, zplane(g, z0 - 2), b);
+            tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, zplane(g, z0 - 1), b);
+            tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, zplane(g, z0 - 1), b);
             for (int q = z0 - 1; q <= min(z0 + PF - 2, z1); q++) issue(q);  // step t: t+PF+1
         }
 
@@ -489,7 +496,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             pq1 = pn;
             bkc = rin ? bkn : *(const double2*)&s.Khi[coff];   // beta_k(t+2): next step's bottom face
             if (bin)   // streaming store: do not evict halo lines other tiles still need
-                __stcs((double2*)(xo + (long)(t - 1 + SF_GZ) * g.ks + (long)(gy + SF_GY) * g.js +
+                __stcs((double2*)(xo + (long)zplane(g, t - 1) * g.ks + (long)(gy + SF_GY) * g.js +
                                   SF_OX + gxa), o);
 #pragma unroll
             for (int i = 0; i < 8; i++) stash[i] = nb[i];
@@ -690,7 +697,9 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY(encode(&mp.bi, L, v.f[SF_BETA_I], CHH));
         SF_TRY(encode(&mp.bj, L, v.f[SF_BETA_J], CHH));
         SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
-        Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks};
+        Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks, 0};
+        if (const char* ez = getenv("SF_DBG_ZMASK"))   // measurement only (see zplane)
+            if (atoi(ez) > 0 && v.nz > atoi(ez)) g.zmask = atoi(ez);
         int grid = std::min(items, Gl);
         CoarseView cvw{nullptr, 0, 0, 0};
         if (C) {

@@ -336,9 +336,13 @@ __global__ void init_problem_kernel(PV v, int gnx, int gny, double h, int proble
             double ch = cosh(BSHARP * (r - BRAD));
             double sc = 0.5 * (BMAX - BMIN) * BSHARP / (ch * ch);
             beta = beta_at(xc, yc, zc);
-            bx = sc * dx / r / Lx;
-            by = sc * dy / r / Ly;
-            bz = sc * dz / r / Lz;
+            // grad beta = beta'(r) (dx, dy, dz) / r; at r = 0 (the centre cell of
+            // an all-odd grid) the direction is undefined but bounded and beta'
+            // is finite: the limit of the flux term's gradient part is 0
+            const double ir = r > 0.0 ? 1.0 / r : 0.0;
+            bx = sc * dx * ir / Lx;
+            by = sc * dy * ir / Ly;
+            bz = sc * dz * ir / Lz;
         }
         v.f[SF_F][q] = a * 1.0 * u - b * (bx * ux + by * uy + bz * uz + beta * lap);
     }

@@ -503,9 +503,16 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
                 const double cost = (double)((items + G - 1) / G) * (d + 1.0);
                 if (cost < best - 1e-9) { best = cost; best_d = d; }
             }
+            // test / tuning overrides: chunk depth (coarse planes) and grid size,
+            // so small levels take the multi-plane, multi-item paths of 512^3
+            if (const char* e = getenv("SF_RR_DEPTH"))
+                if (atoi(e) > 0) best_d = std::min(nK, atoi(e));
             const int items = tiles * ((nK + best_d - 1) / best_d);
+            int grid = std::min(items, G);
+            if (const char* e = getenv("SF_RR_GRID"))
+                if (atoi(e) > 0) grid = std::min(items, atoi(e));
 #define SF_RRZS(MB)                                                                              \
-    sf_launch(residual_restrict_zs_kernel<MB>, std::min(items, G), dim3(PX, PY), 0, F->stream,           \
+    sf_launch(residual_restrict_zs_kernel<MB>, grid, dim3(PX, PY), 0, F->stream,                         \
         f, f.f[x], f.f[rhs], a, bh2, c, c.f[cf], rep ? f.z0 / 2 : 0, best_d, tgx, tiles, items)
             if (rr_zs() == 2) SF_RRZS(6);
             else if (rr_zs() == 3) SF_RRZS(8);

@@ -232,7 +232,7 @@ extern "C" sf_status sf_level_download(sf_level* L, int field, double* host) {
     if (!L || !host) return sf_fail(SF_ERR_INVALID, "NULL argument");
     SF_TRY(check_field(field));
     SF_TRY(copy3d(L, field, host, false));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     return SF_OK;
 }
 
@@ -250,7 +250,7 @@ extern "C" sf_status sf_level_field_ptr(sf_level* L, int part, int field, double
 
 extern "C" sf_status sf_sync(sf_level* L) {
     if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     SF_CUDA(cudaGetLastError());
     return SF_OK;
 }
@@ -349,7 +349,7 @@ sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, 
     for (int it = 0; it < iters; it++) SF_TRY(k_power_step(L, v, SF_R, a, b, sumsq));
     // last ratio ||D^-1 A v|| / ||v|| with ||v|| = 1 after normalisation
     SF_TRY(sf_scalar_to_host(L, sumsq, 1));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     *out = sqrt(L->hscratch[1]);
     return SF_OK;
 }
@@ -382,8 +382,7 @@ extern "C" sf_status sf_smooth_residual_restrict(sf_level* F, int x, int rhs, do
     if (x == rhs || x == SF_DINV || rhs == SF_DINV || x == SF_R || rhs == SF_R || cf == SF_DINV)
         return sf_fail(SF_ERR_INVALID, "x, rhs, R and DINV must be distinct fields");
     if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
-    if ((x == SF_U || x == SF_TMP) && rhs != SF_U && rhs != SF_TMP && gsrb_fused_supported(F) &&
-        gsrb_rr_supported(F, C)) {
+    if (x == SF_U && rhs != SF_TMP && gsrb_fused_supported(F) && gsrb_rr_supported(F, C)) {
         const int other = (x == SF_U) ? SF_TMP : SF_U;
         SF_TRY(sf_halo(F, rhs, 1));
         SF_TRY(sf_halo(F, x, 2));
@@ -396,6 +395,28 @@ extern "C" sf_status sf_smooth_residual_restrict(sf_level* F, int x, int rhs, do
         return k_residual_restrict(F, x, rhs, a, b, C, cf);
     SF_TRY(k_residual(F, SF_R, x, rhs, a, b));
     return k_restrict(C, cf, F, SF_R, SF_RESTRICT_CELL);
+}
+
+extern "C" sf_status sf_interpolate_smooth(sf_level* F, int x, int rhs, double a, double b,
+                                           sf_level* C, int cf) {
+    if (!F || !C) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(x));
+    SF_TRY(check_field(rhs));
+    SF_TRY(check_field(cf));
+    if (x == rhs || x == SF_DINV || rhs == SF_DINV)
+        return sf_fail(SF_ERR_INVALID, "x, rhs and DINV must be distinct fields");
+    if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
+    if (x == SF_U && rhs != SF_TMP && gsrb_fused_supported(F)) {
+        // e_l += P0 e_{l+1} applied to each x plane in shared memory inside the
+        // colour-fused pair (the V-cycle's first post-smoothing pair, mg.cu)
+        SF_TRY(sf_halo(C, cf, 1));
+        SF_TRY(sf_halo(F, rhs, 1));
+        SF_TRY(k_gsrb_pair_halo(F, SF_U, SF_TMP, rhs, a, b, nullptr, C, cf, SF_RM_NONE));
+        sf_swap_fields(F, SF_U, SF_TMP);
+        return SF_OK;
+    }
+    SF_TRY(k_interp(F, x, 1.0, C, cf, SF_INTERP_P0));
+    return sf_smooth_gsrb(F, x, rhs, a, b, 1, SF_SMOOTH_AUTO);
 }
 
 bool gsrb_fused_supported(const sf_level* L) {
@@ -415,7 +436,11 @@ sf_status k_gsrb_pair_fused(sf_level* L, int xin, int xout, int rhs, double a, d
     // correction waits one bundle ahead): 32x16 build there, 0.25 % faster
     // solve (r01/ab_interp_t32.txt); SF_INTERP_T32=0 disables
     const char* ei = getenv("SF_INTERP_T32");
-    if (C && !(ei && atoi(ei) == 0) && w4 < 0 && (long)L->nx * L->ny * L->lnz > (1L << 24) &&
+    // SF_INTERP_T32_CELLS: the level size above which it applies (tests lower it
+    // to compare that build with the oracle cell by cell on small levels)
+    const char* ec = getenv("SF_INTERP_T32_CELLS");
+    const long t32_cells = ec ? atol(ec) : (1L << 24);
+    if (C && !(ei && atoi(ei) == 0) && w4 < 0 && (long)L->nx * L->ny * L->lnz > t32_cells &&
         gsrb_fused_supported_t32(L))
         w4 = 0;
     if (w4 != 0 && gsrb_fused_supported_t32w4(L))
@@ -441,7 +466,10 @@ extern "C" sf_status sf_smooth_gsrb(sf_level* L, int x, int rhs, double a, doubl
                     rhs != SF_U;
     if (kind == SF_SMOOTH_FUSED && !fused_ok)
         return sf_fail(SF_ERR_SHAPE, "fused smoother unsupported for this level/fields");
-    bool fused = (kind == SF_SMOOTH_FUSED) || (kind == SF_SMOOTH_AUTO && fused_ok);
+    // the fused pair ping-pongs x through the other of U / TMP; AUTO only takes
+    // it when that other field is the scratch TMP (x = U), so a solution in U is
+    // never clobbered by a call that did not ask for the fused kernel
+    bool fused = (kind == SF_SMOOTH_FUSED) || (kind == SF_SMOOTH_AUTO && fused_ok && x == SF_U);
     if (rb_pairs == 0) return SF_OK;
     if (fused) {
         int other = (x == SF_U) ? SF_TMP : SF_U;
@@ -509,7 +537,7 @@ extern "C" sf_status sf_norm(sf_level* L, int field, int kind, double* out) {
     if (kind != SF_NORM_MAX && kind != SF_NORM_L2) return sf_fail(SF_ERR_INVALID, "bad norm kind");
     SF_TRY(sf_norm_async(L, field, kind, L->dscratch));
     SF_TRY(sf_scalar_to_host(L, L->dscratch, 0));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     double v = L->hscratch[0];
     *out = (kind == SF_NORM_L2) ? sqrt(v) : v;
     return SF_OK;
@@ -529,15 +557,15 @@ extern "C" sf_status sf_level_pair_timing(sf_level* L, int op, double* mean_ms, 
     if (op == 1) {
         static const unsigned long long arm[6] = {1ull, ~0ull, 0ull, 0ull, 0ull, 0ull};
         SF_CUDA(cudaMemcpyAsync(ts, arm, sizeof(arm), cudaMemcpyHostToDevice, L->stream));
-        SF_CUDA(cudaStreamSynchronize(L->stream));
+        SF_TRY(sf_stream_sync(L));
         return SF_OK;
     }
     unsigned long long h[6];
     SF_CUDA(cudaMemcpyAsync(h, ts, sizeof(h), cudaMemcpyDeviceToHost, L->stream));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     static const unsigned long long off = 0ull;
     SF_CUDA(cudaMemcpyAsync(ts, &off, sizeof(off), cudaMemcpyHostToDevice, L->stream));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     if (count) *count = (long long)h[4];
     if (mean_ms) *mean_ms = h[4] ? (double)h[5] / (double)h[4] * 1e-6 : 0.0;
     return SF_OK;

@@ -9,6 +9,7 @@
 // Every cycle only ENQUEUES work on the finest level's stream (no host sync),
 // so a whole V-cycle (+ its convergence residual and norm) is captured once as
 // a CUDA graph and replayed: levels <= 64^3 are launch-latency bound.
+#include <chrono>
 #include <cmath>
 #include <cstdlib>
 
@@ -46,7 +47,45 @@ struct sf_mg {
     LoopHost* lhost = nullptr;
     LoopHost* lhost_dev = nullptr;
     std::vector<double> lmax;   // SF_SMOOTH_CHEBY: lambda_max(D^-1 A) per level
+    // Field -> buffer mapping of every level when the cached graphs were
+    // captured: a graph names device pointers, so a public call that swaps
+    // U/TMP (sf_smooth_gsrb, sf_smooth_chebyshev, ...) between solves makes
+    // every cached graph stale; they are then destroyed and re-captured.
+    std::vector<double*> gsig;
+    // sf_solve_stream: staging buffers, copy streams and events kept across
+    // calls (a per-call 2 x 1 GiB cudaMalloc/cudaFree cost more than it hid)
+    double *stf = nullptr, *stu = nullptr;
+    size_t st_bytes = 0;
+    cudaStream_t sin = nullptr, sout = nullptr;
+    cudaEvent_t sev[4] = {};      // f_ready, f_free, u_ready, u_free
+    double stats[4] = {};         // last call: mean H2D, solve, D2H ms; wall ms per rhs
 };
+
+static std::vector<double*> field_map(const sf_mg* m) {
+    std::vector<double*> v;
+    for (const sf_level* l : m->lv)
+        for (const SfPart& P : l->parts) v.insert(v.end(), P.f, P.f + SF_NFIELDS);
+    return v;
+}
+
+// Drop every cached graph whose device pointers no longer match the levels'
+// field mapping; remember the mapping the next captures will see.
+static void refresh_graph_map(sf_mg* m) {
+    std::vector<double*> cur = field_map(m);
+    if (cur == m->gsig) return;
+    if (!m->lv.empty()) cudaStreamSynchronize(m->lv[0]->stream);
+    for (auto& g : m->gexec)
+        if (g) {
+            cudaGraphExecDestroy(g);
+            g = nullptr;
+        }
+    for (auto& g : m->gloop)
+        if (g) {
+            cudaGraphExecDestroy(g);
+            g = nullptr;
+        }
+    m->gsig.swap(cur);
+}
 
 // NEXT-3 reading R-16: Chebyshev interval [hi/8, hi], hi = 1.05 lambda_max(D^-1 A)
 // (power iteration, 30 steps from the fixed start vector, at setup)
@@ -86,6 +125,14 @@ extern "C" sf_status sf_mg_destroy(sf_mg* m) {
         if (g) cudaGraphExecDestroy(g);
     if (m->lctl) cudaFree(m->lctl);
     if (m->lhost) cudaFreeHost(m->lhost);
+    if (m->sin) cudaStreamSynchronize(m->sin);
+    if (m->sout) cudaStreamSynchronize(m->sout);
+    for (cudaEvent_t e : m->sev)
+        if (e) cudaEventDestroy(e);
+    if (m->sin) cudaStreamDestroy(m->sin);
+    if (m->sout) cudaStreamDestroy(m->sout);
+    cudaFree(m->stf);
+    cudaFree(m->stu);
     if (m->ainv) cudaFree(m->ainv);
     destroy_levels(m);
     delete m;
@@ -439,6 +486,7 @@ static sf_status capture(sf_mg* m, int kind) {
 // enqueue cycle piece `kind` (graph replay when possible)
 static sf_status run(sf_mg* m, int kind) {
     sf_level* L = m->lv[0];
+    if (graphs_allowed(m)) refresh_graph_map(m);
     if (graphs_allowed(m) && !m->gexec[kind]) {
         if (kind == G_FIRST || kind == G_REST) {
             // capture both halves back to back: together they hold an even
@@ -669,6 +717,7 @@ static sf_status solve_loop(sf_mg* m, int fc, double rtol, int max_cycles, int* 
                             double* hist, bool* handled) {
     *handled = false;
     if (max_cycles > SF_LOOP_HIST || !loop_allowed(m)) return SF_OK;
+    refresh_graph_map(m);
     if (!m->gloop[fc]) SF_TRY(build_loop(m, fc));
     if (!m->gloop[fc]) return SF_OK;
     sf_level* L = m->lv[0];
@@ -676,7 +725,7 @@ static sf_status solve_loop(sf_mg* m, int fc, double rtol, int max_cycles, int* 
     m->lhost->max_cycles = max_cycles;
     m->lhost->done = -1;
     SF_CUDA(cudaGraphLaunch(m->gloop[fc], L->stream));
-    SF_CUDA(cudaStreamSynchronize(L->stream));
+    SF_TRY(sf_stream_sync(L));
     *handled = true;
     const LoopHost& r = *m->lhost;
     if (r.done < 0) return sf_fail(SF_ERR_CUDA, "device solve loop did not publish");
@@ -714,7 +763,8 @@ extern "C" sf_status sf_fcycle(sf_mg* m) {
 extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles, int* cycles,
                               double* hist) {
     if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
-    if (max_cycles < 1) max_cycles = m->o.max_cycles;
+    // hist holds max_cycles entries (sf.h): a silent default cap would overrun it
+    if (max_cycles < 1) return sf_fail(SF_ERR_INVALID, "max_cycles must be >= 1");
     if (!(rtol > 0)) rtol = m->o.rtol;
     sf_level* L = m->lv[0];
     {
@@ -740,7 +790,7 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
     if (!fused) {
         for (int c = 1; c <= max_cycles; c++) {
             SF_TRY(run(m, (fcycle && c == 1) ? G_FCHECK : G_VCHECK));
-            SF_CUDA(cudaStreamSynchronize(L->stream));
+            SF_TRY(sf_stream_sync(L));
             int r = fin(L->hscratch[0] / fn, c);
             if (r < 0) return sf_fail(SF_ERR_NUMERIC, "residual is NaN/Inf");
             if (r > 0) return SF_OK;
@@ -756,7 +806,7 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
         // first pair of the next V-cycle + max|F - A U| of the iterate after `done` cycles
         const double* u0 = L->parts[0].f[SF_U];
         SF_TRY(run(m, G_FIRST));
-        SF_CUDA(cudaStreamSynchronize(L->stream));
+        SF_TRY(sf_stream_sync(L));
         if (done >= 1) {
             int r = fin(L->hscratch[0] / fn, done);
             if (r != 0 || done >= max_cycles) {
@@ -777,7 +827,8 @@ extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles,
 
 // Pipelined multi-RHS solve (include/sf.h): copies of f_{k+1} (H2D) and
 // u_{k-1} (D2H) run on their own streams under solve k; two packed staging
-// buffers decouple them from the level's F and U.
+// buffers (kept by the hierarchy) decouple them from the level's F and U.
+// Per-phase device times of the call are kept for sf_solve_stream_stats.
 extern "C" sf_status sf_solve_stream(sf_mg* m, int fcycle, double rtol, int max_cycles, int n,
                                      const double* const* host_f, double* const* host_u,
                                      int* cycles) {
@@ -785,28 +836,48 @@ extern "C" sf_status sf_solve_stream(sf_mg* m, int fcycle, double rtol, int max_
     if (n == 0) return SF_OK;
     sf_level* L = m->lv[0];
     const size_t bytes = (size_t)L->nlocal * L->lnz * L->ny * L->nx * sizeof(double);
-    double *stf = nullptr, *stu = nullptr;
-    cudaStream_t sin = nullptr, sout = nullptr;
-    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};   // f_ready, f_free, u_ready, u_free
+    if (m->st_bytes != bytes) {
+        cudaFree(m->stf);
+        cudaFree(m->stu);
+        m->stf = m->stu = nullptr;
+        m->st_bytes = 0;
+        SF_CUDA(cudaMalloc(&m->stf, bytes));
+        SF_CUDA(cudaMalloc(&m->stu, bytes));
+        m->st_bytes = bytes;
+    }
+    if (!m->sin) {
+        SF_CUDA(cudaStreamCreateWithFlags(&m->sin, cudaStreamNonBlocking));
+        SF_CUDA(cudaStreamCreateWithFlags(&m->sout, cudaStreamNonBlocking));
+        for (int i = 0; i < 4; i++) SF_CUDA(cudaEventCreateWithFlags(&m->sev[i], cudaEventDisableTiming));
+    }
+    double *stf = m->stf, *stu = m->stu;
+    cudaStream_t sin = m->sin, sout = m->sout;
+    cudaEvent_t* ev = m->sev;
+    // phase timing: [k][0..5] = H2D start/end, solve start/end, D2H start/end
+    std::vector<cudaEvent_t> te(6 * (size_t)n, nullptr);
+    for (auto& e : te) SF_CUDA(cudaEventCreate(&e));
+    auto tev = [&](int k, int i) { return te[6 * (size_t)k + i]; };
     sf_status st = SF_OK;
     auto cu = [&](cudaError_t e, const char* what) {
         if (e != cudaSuccess && st == SF_OK) st = sf_fail(SF_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
         return st == SF_OK;
     };
-    if (cu(cudaMalloc(&stf, bytes), "staging f") && cu(cudaMalloc(&stu, bytes), "staging u") &&
-        cu(cudaStreamCreateWithFlags(&sin, cudaStreamNonBlocking), "stream") &&
-        cu(cudaStreamCreateWithFlags(&sout, cudaStreamNonBlocking), "stream")) {
-        for (int i = 0; i < 4 && st == SF_OK; i++)
-            cu(cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming), "event");
-    }
-    if (st == SF_OK && cu(cudaMemcpyAsync(stf, host_f[0], bytes, cudaMemcpyDefault, sin), "H2D f") &&
-        cu(cudaEventRecord(ev[0], sin), "record")) {
+    const auto w0 = std::chrono::steady_clock::now();
+    int solved = 0;
+    // the u staging buffer is free at the start (no D2H pending)
+    cu(cudaEventRecord(ev[3], sout), "record");
+    if (cu(cudaEventRecord(tev(0, 0), sin), "record") &&
+        cu(cudaMemcpyAsync(stf, host_f[0], bytes, cudaMemcpyDefault, sin), "H2D f") &&
+        cu(cudaEventRecord(tev(0, 1), sin), "record") && cu(cudaEventRecord(ev[0], sin), "record")) {
         for (int k = 0; k < n && st == SF_OK; k++) {
             if (!cu(cudaStreamWaitEvent(L->stream, ev[0], 0), "wait")) break;
+            if (!cu(cudaEventRecord(tev(k, 2), L->stream), "record")) break;
             if ((st = k_pack(L, SF_F, stf, true)) != SF_OK) break;
             if (!cu(cudaEventRecord(ev[1], L->stream), "record")) break;
             if (k + 1 < n && !(cu(cudaStreamWaitEvent(sin, ev[1], 0), "wait") &&
+                               cu(cudaEventRecord(tev(k + 1, 0), sin), "record") &&
                                cu(cudaMemcpyAsync(stf, host_f[k + 1], bytes, cudaMemcpyDefault, sin), "H2D f") &&
+                               cu(cudaEventRecord(tev(k + 1, 1), sin), "record") &&
                                cu(cudaEventRecord(ev[0], sin), "record")))
                 break;
             if (!fcycle && (st = k_zero(L, SF_U)) != SF_OK) break;
@@ -816,22 +887,37 @@ extern "C" sf_status sf_solve_stream(sf_mg* m, int fcycle, double rtol, int max_
             if (st != SF_OK) break;
             if (!cu(cudaStreamWaitEvent(L->stream, ev[3], 0), "wait")) break;
             if ((st = k_pack(L, SF_U, stu, false)) != SF_OK) break;
-            if (!(cu(cudaEventRecord(ev[2], L->stream), "record") &&
+            if (!(cu(cudaEventRecord(tev(k, 3), L->stream), "record") &&
+                  cu(cudaEventRecord(ev[2], L->stream), "record") &&
                   cu(cudaStreamWaitEvent(sout, ev[2], 0), "wait") &&
+                  cu(cudaEventRecord(tev(k, 4), sout), "record") &&
                   cu(cudaMemcpyAsync(host_u[k], stu, bytes, cudaMemcpyDefault, sout), "D2H u") &&
+                  cu(cudaEventRecord(tev(k, 5), sout), "record") &&
                   cu(cudaEventRecord(ev[3], sout), "record")))
                 break;
+            solved = k + 1;
         }
     }
     sf_status keep = st;
-    if (sin) cudaStreamSynchronize(sin);
-    if (sout) cudaStreamSynchronize(sout);
+    cudaStreamSynchronize(sin);
+    cudaStreamSynchronize(sout);
     cudaStreamSynchronize(L->stream);
-    for (cudaEvent_t e : ev)
-        if (e) cudaEventDestroy(e);
-    if (sin) cudaStreamDestroy(sin);
-    if (sout) cudaStreamDestroy(sout);
-    cudaFree(stf);
-    cudaFree(stu);
+    const double wall = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - w0).count();
+    double acc[3] = {0, 0, 0};
+    for (int k = 0; k < solved; k++)
+        for (int p = 0; p < 3; p++) {
+            float ms = 0.f;
+            if (cudaEventElapsedTime(&ms, tev(k, 2 * p), tev(k, 2 * p + 1)) == cudaSuccess) acc[p] += ms;
+        }
+    cudaGetLastError();
+    for (auto& e : te) cudaEventDestroy(e);
+    for (int p = 0; p < 3; p++) m->stats[p] = solved ? acc[p] / solved : 0.0;
+    m->stats[3] = solved ? wall / solved : 0.0;
     return keep;
+}
+
+extern "C" sf_status sf_solve_stream_stats(const sf_mg* m, double stats[4]) {
+    if (!m || !stats) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    for (int i = 0; i < 4; i++) stats[i] = m->stats[i];
+    return SF_OK;
 }

@@ -218,5 +218,8 @@ sf_status sf_agglomerate(sf_level* C, int field, int parts, int lnz_per_part);
 // kind-2 comm: open the peers' buffers of level L (collective)
 sf_status sf_ipc_register(sf_level* L, const sf_comm* c);
 void sf_ipc_close(sf_level* L);
+// Host synchronisation of the level's stream: NCCL async errors polled, a
+// timed-out p2p peer wait reported by name (comm.cu).
+sf_status sf_stream_sync(sf_level* L);
 // Reduce a device scalar over ranks (op 0 = max, 1 = sum); in place.
 sf_status sf_allreduce_scalar(sf_level* L, const sf_comm* comm, double* dev, int op);

@@ -71,7 +71,10 @@ def _dbeta(xh, yh, zh):
     dx, dy, dz = xh - 0.5, yh - 0.5, zh - 0.5
     r = np.sqrt(dx * dx + dy * dy + dz * dz)
     s = 0.5 * (BMAX - BMIN) * BSHARP / np.cosh(BSHARP * (r - BRAD)) ** 2
-    return s * dx / r, s * dy / r, s * dz / r
+    # r = 0 only at the centre cell of an all-odd grid: the gradient's direction
+    # is undefined there but bounded, so its limit contribution is 0
+    ir = np.divide(1.0, r, out=np.zeros_like(r), where=r > 0)
+    return s * dx * ir, s * dy * ir, s * dz * ir
 
 
 def _X(t):

@@ -46,6 +46,7 @@ EXPORTS = [
     "sf_comm_create_hostipc", "sf_stencil_compile", "sf_stencil_source", "sf_stencil_apply",
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
     "sf_comm_create_p2p", "sf_smooth_residual_restrict", "sf_level_pair_timing",
+    "sf_interpolate_smooth", "sf_comm_check", "sf_solve_stream_stats",
 ]
 
 
@@ -127,6 +128,9 @@ def lib():
         "sf_smooth_gsrb": (_i, [_vp, _i, _i, _d, _d, _i, _i]),
         "sf_residual": (_i, [_vp, _i, _i, _i, _d, _d]),
         "sf_smooth_residual_restrict": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
+        "sf_interpolate_smooth": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
+        "sf_comm_check": (_i, [_vp, _vp]),
+        "sf_solve_stream_stats": (_i, [_vp, C.POINTER(C.c_double)]),
         "sf_apply_laplacian": (_i, [_vp, _i, _i]),
         "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
         "sf_smooth_chebyshev": (_i, [_vp, _i, _i, _d, _d, _i, _d, _d]),
@@ -318,6 +322,14 @@ def sf_smooth_residual_restrict(fine, x, rhs, a, b, coarse, c_field):
     _check(lib().sf_smooth_residual_restrict(fine, x, rhs, float(a), float(b), coarse, c_field))
 
 
+def sf_comm_check(comm, stream=None):
+    _check(lib().sf_comm_check(comm, stream))
+
+
+def sf_interpolate_smooth(fine, x, rhs, a, b, coarse, c_field):
+    _check(lib().sf_interpolate_smooth(fine, x, rhs, float(a), float(b), coarse, c_field))
+
+
 def sf_apply_laplacian(level, out, x):
     _check(lib().sf_apply_laplacian(level, out, x))
 
@@ -419,6 +431,14 @@ def sf_solve_stream(mg, host_f_ptrs, host_u_ptrs, fcycle=True, rtol=1e-10, max_c
 
 def sf_mg_destroy(mg):
     _check(lib().sf_mg_destroy(mg))
+
+
+def sf_solve_stream_stats(mg):
+    """(h2d_ms, solve_ms, d2h_ms, wall_ms) per right-hand side of the last
+    sf_solve_stream call."""
+    out = (C.c_double * 4)()
+    _check(lib().sf_solve_stream_stats(mg, out))
+    return tuple(out)
 
 
 def sf_mg_plan(gnx, gny, gnz, nparts=1, agglom_min_planes=8, max_levels=32):

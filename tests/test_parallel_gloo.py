@@ -91,3 +91,15 @@ def test_plan_rejects_bad_shapes():
     with pytest.raises(sf.SfError):
         sf.sf_mg_plan(512, 512, 30, 2, 16)        # 15 planes per slab cannot halve
     assert len(sf.sf_mg_plan(16, 16, 16)) == 4
+
+
+def test_mg_plan_matches_bench_n8():
+    """bench.py at N = 8: 1024^3 in 8 slabs of 128 planes stays distributed
+    down to 128^3 (16 planes per rank) and is agglomerated from 64^3 on; the
+    64x64x256 8-part GPU test (test_gpu_multigpu_readiness.py) has the same
+    pattern: distributed levels, then agglomerated ones down to the bottom."""
+    from paper_conf_ipps_zhangdmwbf17_b200 import sf
+    d8 = [d for _, d in sf.sf_mg_plan(1024, 1024, 1024, 8, 16)]
+    dt = [d for _, d in sf.sf_mg_plan(64, 64, 256, 8, 16)]
+    assert d8 == [True] * 4 + [False] * 6
+    assert dt == [True] * 2 + [False] * 4
