@@ -29,7 +29,7 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
             ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=2", "-DSF_GSRB_NWARP=4", "-DSF_GSRB_MINB=3",
              "-DSF_GSRB_SUFFIX=_t32w4"]),
            ("gsrb_rr.cu", "gsrb_rr.o", []),
-           ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []),
+           ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []), ("coarse.cu", "coarse.o", []),
            ("stencil.cu", "stencil.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -49,6 +49,7 @@ def _compile(spec, force):
     s = os.path.join(CSRC, src)
     o = os.path.join(BUILD, obj)
     deps = [s, os.path.join(CSRC, "sf_internal.h"), os.path.join(CSRC, "tma_common.cuh"),
+            os.path.join(CSRC, "cell_ops.cuh"),
             os.path.join(INCLUDE, "sf.h")]
     if not force and not _needs(o, deps):
         return o, ""

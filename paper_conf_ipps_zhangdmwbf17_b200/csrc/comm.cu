@@ -310,6 +310,8 @@ __global__ void __launch_bounds__(256) p2p_gather_kernel(double* base, P2PPtrs p
     p2p_end(my, pe, nranks, s);
 }
 
+static sf_status sync_failure(cudaError_t e, const char* what);
+
 // process-wide mapped host word for the p2p timeout diagnosis (see wait_ge)
 static unsigned long long* g_err_host = nullptr;
 static unsigned long long* g_err_dev = nullptr;
@@ -338,7 +340,10 @@ static P2PPeers peers_init() {
     return pe;
 }
 
-// Status of a synchronisation that returned e; a timed-out peer wait is named.
+// Status of a CUDA call that returned e; a timed-out peer wait is named (the
+// trap it caused is a sticky error, so whichever call sees it first reports it).
+sf_status sf_cuda_failure(cudaError_t e, const char* what) { return sync_failure(e, what); }
+
 static sf_status sync_failure(cudaError_t e, const char* what) {
     const unsigned long long w = g_err_host ? *(volatile unsigned long long*)g_err_host : 0ull;
     if (w >> 63)

@@ -23,31 +23,7 @@ inline dim3 cell_grid(const PV& v) {
     return dim3((v.nx + BX - 1) / BX, (v.ny + BY - 1) / BY, v.nz);
 }
 
-// A3 at cell (i,j,k) with the Dirichlet fold.  Summation order matches the
-// operator definition term by term (A3).
-__device__ __forceinline__ double op_at(const PV& v, const double* __restrict__ x, int i, int j,
-                                        int k, double a, double bh2) {
-    const double* al = v.f[SF_ALPHA];
-    const double* bi = v.f[SF_BETA_I];
-    const double* bj = v.f[SF_BETA_J];
-    const double* bk = v.f[SF_BETA_K];
-    long c = sf_ix(v, i, j, k);
-    double xc = x[c];
-    int gk = v.z0 + k;
-    double xw = (i == 0) ? -xc : x[c - 1];
-    double xe = (i == v.nx - 1) ? -xc : x[c + 1];
-    double xs = (j == 0) ? -xc : x[c - v.js];
-    double xn = (j == v.ny - 1) ? -xc : x[c + v.js];
-    double xb = (gk == 0) ? -xc : x[c - v.ks];
-    double xt = (gk == v.gnz - 1) ? -xc : x[c + v.ks];
-    double flux = bi[c + 1] * (xe - xc);
-    flux += bi[c] * (xw - xc);
-    flux += bj[c + v.js] * (xn - xc);
-    flux += bj[c] * (xs - xc);
-    flux += bk[c + v.ks] * (xt - xc);
-    flux += bk[c] * (xb - xc);
-    return a * al[c] * xc - bh2 * flux;
-}
+#include "cell_ops.cuh"
 
 __global__ void __launch_bounds__(BX* BY) apply_op_kernel(PV v, double* __restrict__ out,
                                                            const double* __restrict__ x, double a,

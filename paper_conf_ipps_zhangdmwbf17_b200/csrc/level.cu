@@ -23,7 +23,11 @@ void sf_count_launch(long long n) { g_launches.fetch_add(n, std::memory_order_re
 
 sf_status sf_check_launch(const char* what) {
     cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return sf_fail(SF_ERR_CUDA, "launch of %s: %s", what, cudaGetErrorString(e));
+    if (e != cudaSuccess) {
+        char w[160];
+        snprintf(w, sizeof(w), "launch of %s", what);
+        return sf_cuda_failure(e, w);
+    }
     return SF_OK;
 }
 

@@ -47,6 +47,7 @@ struct sf_mg {
     LoopHost* lhost = nullptr;
     LoopHost* lhost_dev = nullptr;
     std::vector<double> lmax;   // SF_SMOOTH_CHEBY: lambda_max(D^-1 A) per level
+    int coarse_l0 = -1;         // first level whose V-cycle runs as one cluster launch (-1: none)
     // Field -> buffer mapping of every level when the cached graphs were
     // captured: a graph names device pointers, so a public call that swaps
     // U/TMP (sf_smooth_gsrb, sf_smooth_chebyshev, ...) between solves makes
@@ -184,6 +185,29 @@ extern "C" sf_status sf_mg_plan(int gnx, int gny, int gnz, int nparts, int amin,
     return SF_OK;
 }
 
+// First level l >= 1 from which V(l) runs as ONE cluster launch (coarse.cu):
+// every level from l down is single-part and l has at most SF_COARSE_CELLS
+// cells (default 32^3); GSRB smoothers with P0 in the V-cycle only (the
+// kernel implements those).  SF_COARSE_KERNEL=0 keeps the per-phase launches.
+static int plan_coarse(const sf_mg* m) {
+    const char* e = getenv("SF_COARSE_KERNEL");
+    if (e && atoi(e) == 0) return -1;
+    if (m->o.smoother == SF_SMOOTH_CHEBY || m->o.vcycle_interp != SF_INTERP_P0) return -1;
+    const char* ec = getenv("SF_COARSE_CELLS");
+    const long maxc = ec ? atol(ec) : 32768L;
+    const int nl = (int)m->lv.size();
+    int l0 = -1;
+    for (int l = nl - 1; l >= 1; l--) {
+        const sf_level* L = m->lv[l];
+        if (L->nparts != 1 || L->nlocal != 1) break;
+        if ((long)L->nx * L->ny * L->lnz > maxc) break;
+        if (nl - l > coarse_vcycle_max_levels()) break;
+        l0 = l;
+    }
+    if (l0 < 0 || l0 >= nl - 1 || !coarse_vcycle_available()) return -1;
+    return l0;
+}
+
 extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double b,
                                   const sf_mg_opts* opts) {
     if (!out || !fine) return sf_fail(SF_ERR_INVALID, "NULL argument");
@@ -261,6 +285,7 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
         cudaError_t e = cudaStreamSynchronize(fine->stream);
         if (e != cudaSuccess) s = sf_fail(SF_ERR_CUDA, "mg setup: %s", cudaGetErrorString(e));
     }
+    if (s == SF_OK) m->coarse_l0 = plan_coarse(m);
     if (s != SF_OK) {
         sf_mg_destroy(m);
         return s;
@@ -313,6 +338,9 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
+    if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one cluster launch
+        return k_coarse_vcycle(&m->lv[l], (int)m->lv.size() - l, m->a, m->b, m->ainv,
+                               m->o.pre_pairs, m->o.post_pairs);
     sf_level* C = m->lv[l + 1];
     const int pre = m->o.pre_pairs - (skip_first ? 1 : 0);
     if (pre >= 1 && (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&

@@ -93,12 +93,12 @@ sf_status sf_copy_field(sf_level* L, int field, double* host, bool up, cudaStrea
 
 // ------------------------------------------------------------------ errors
 sf_status sf_fail(sf_status s, const char* fmt, ...);
+// SF_ERR_CUDA for e; names a timed-out p2p peer wait if that caused it (comm.cu)
+sf_status sf_cuda_failure(cudaError_t e, const char* what);
 #define SF_CUDA(call)                                                                  \
     do {                                                                               \
         cudaError_t e_ = (call);                                                       \
-        if (e_ != cudaSuccess)                                                         \
-            return sf_fail(SF_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,     \
-                           cudaGetErrorString(e_));                                    \
+        if (e_ != cudaSuccess) return sf_cuda_failure(e_, #call);                      \
     } while (0)
 #define SF_TRY(call)                                \
     do {                                            \
@@ -208,6 +208,12 @@ sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t s);
 bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
                          int cf);
+
+// coarse-level V-cycle in one thread-block-cluster launch (coarse.cu)
+bool coarse_vcycle_available();
+int coarse_vcycle_max_levels();
+sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
+                          int pre, int post);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.
