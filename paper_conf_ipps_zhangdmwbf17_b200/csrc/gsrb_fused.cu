@@ -649,9 +649,13 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     double best = 1e30;
     const int min_nch = phase ? 3 : 1;
     if (L->lnz < min_nch) return sf_fail(SF_ERR_SHAPE, "split fused pair needs >= 3 planes per part");
+    // shallowest chunk considered (SF_GSRB_MIND, A/B knob; 8 before r02): small
+    // levels whose items fit one round of resident CTAs want shallow chunks
+    // (fewer serial z steps per CTA); big levels pick deep ones anyway
+    static const int mind = getenv("SF_GSRB_MIND") ? std::max(1, atoi(getenv("SF_GSRB_MIND"))) : 1;
     for (int nch = min_nch; nch <= L->lnz; nch++) {
         int d = (L->lnz + nch - 1) / nch;
-        if (d < 8 && nch > min_nch) break;
+        if (d < mind && nch > min_nch) break;
         if ((L->lnz + d - 1) / d < min_nch) continue;
         int n = (L->lnz + d - 1) / d;
         long items = (long)tiles * n;

@@ -185,27 +185,19 @@ extern "C" sf_status sf_mg_plan(int gnx, int gny, int gnz, int nparts, int amin,
     return SF_OK;
 }
 
-// First level l >= 1 from which V(l) runs as ONE cluster launch (coarse.cu):
-// every level from l down is single-part and l has at most SF_COARSE_CELLS
-// cells (default 32^3); GSRB smoothers with P0 in the V-cycle only (the
-// kernel implements those).  SF_COARSE_KERNEL=0 keeps the per-phase launches.
-static int plan_coarse(const sf_mg* m) {
+// First level l >= 1 from which V(l) runs as ONE single-CTA launch with the
+// iterates in shared memory (coarse.cu): every level from l down is
+// single-part, l has at most 16^3 cells and the chain fits the kernel's
+// arrays; GSRB smoothers with P0 in the V-cycle only (what the kernel
+// implements).  SF_COARSE_KERNEL=0 keeps the per-phase launches.
+static int plan_coarse(sf_mg* m) {
     const char* e = getenv("SF_COARSE_KERNEL");
     if (e && atoi(e) == 0) return -1;
     if (m->o.smoother == SF_SMOOTH_CHEBY || m->o.vcycle_interp != SF_INTERP_P0) return -1;
-    const char* ec = getenv("SF_COARSE_CELLS");
-    const long maxc = ec ? atol(ec) : 32768L;
     const int nl = (int)m->lv.size();
-    int l0 = -1;
-    for (int l = nl - 1; l >= 1; l--) {
-        const sf_level* L = m->lv[l];
-        if (L->nparts != 1 || L->nlocal != 1) break;
-        if ((long)L->nx * L->ny * L->lnz > maxc) break;
-        if (nl - l > coarse_vcycle_max_levels()) break;
-        l0 = l;
-    }
-    if (l0 < 0 || l0 >= nl - 1 || !coarse_vcycle_available()) return -1;
-    return l0;
+    for (int l = 1; l < nl - 1; l++)
+        if (coarse_vcycle_fits(&m->lv[l], nl - l)) return l;
+    return -1;
 }
 
 extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double b,
@@ -338,7 +330,7 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
-    if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one cluster launch
+    if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one launch
         return k_coarse_vcycle(&m->lv[l], (int)m->lv.size() - l, m->a, m->b, m->ainv,
                                m->o.pre_pairs, m->o.post_pairs);
     sf_level* C = m->lv[l + 1];

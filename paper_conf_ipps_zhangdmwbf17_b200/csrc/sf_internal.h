@@ -209,8 +209,8 @@ bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
                          int cf);
 
-// coarse-level V-cycle in one thread-block-cluster launch (coarse.cu)
-bool coarse_vcycle_available();
+// coarse-level V-cycle in one single-CTA launch, iterates in shared memory (coarse.cu)
+bool coarse_vcycle_fits(sf_level* const* lv, int n);
 int coarse_vcycle_max_levels();
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
                           int pre, int post);

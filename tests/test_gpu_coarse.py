@@ -1,7 +1,8 @@
-"""The coarse-level V-cycle as one thread-block-cluster launch (coarse.cu):
-from the first single-part level of <= 32^3 cells down to the bottom and back,
+"""The coarse-level V-cycle as one single-CTA launch (coarse.cu, iterates in
+shared memory) from the first single-part level of <= 16^3 cells down to the
+bottom and back:
 every colour sweep, residual + restriction, P0 interpolation and the exact
-bottom solve run in one kernel with cluster barriers between phases.
+bottom solve run in one kernel, __syncthreads between phases.
 Compared with the oracle (1e-11 per cycle, same cycle counts per solve) and
 with the per-phase launches it replaces (SF_COARSE_KERNEL=0)."""
 import numpy as np
