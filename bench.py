@@ -315,6 +315,7 @@ def main():
             torch.cuda.cudart().cudaProfilerStop()
     launches = sf.sf_launch_count(reset=True)
     live_pair_ms, live_pairs = sf.sf_level_pair_timing(L.handle, 0)
+    live_var = sf.sf_level_pair_timing_variants(L.handle)
     t = max_over_ranks(e0.elapsed_time(e1) / 1e3)
     value = dof_local * world * args.steps / t
     ms_step = t / args.steps * 1e3
@@ -362,6 +363,9 @@ def main():
                                      "launches inside the timed region (in-kernel %globaltimer, "
                                      "first CTA start to last CTA end; sf_level_pair_timing)",
                     "launches_in_timed_region": live_pairs, "peak_source": pk_src,
+                    "live_per_variant": {k: {"ms": v[0], "pairs": v[1],
+                                             "frac": (alg / (v[0] / 1e3) / 1e9 / pk) if v[0] else None}
+                                         for k, v in live_var.items()},
                     "share_of_step": live_pairs * live_pair_ms / (t * 1e3),
                     "isolated_plain_pair_ms": fine_pair,
                     "isolated_plain_pair_frac": (alg / (fine_pair / 1e3) / 1e9 / pk

@@ -277,6 +277,10 @@ sf_status sf_sync(sf_level* level);
  * boundary launches around a halo exchange counts once, with both durations).  Both ops synchronise the level's stream;
  * the timer works inside captured graphs (it lives in the level's scratch). */
 sf_status sf_level_pair_timing(sf_level* level, int op, double* mean_ms, long long* count);
+/* Per-variant split of the last sf_level_pair_timing(op 0) read-out: mean ms and
+ * pairs of the plain [0], input-residual check-fused RESID [1], output-residual
+ * BRES [2] and P0-fused INTERP [3] (incl. INTERP + BRES) launches.  Host only. */
+sf_status sf_level_pair_timing_variants(const sf_level* level, double mean_ms[4], long long counts[4]);
 
 /* -------------------------------------------------------------- multigrid (A9)
  * sf_mg_create: builds the hierarchy below `finest` (which must hold ALPHA and

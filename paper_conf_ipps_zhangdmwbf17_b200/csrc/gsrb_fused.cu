@@ -538,6 +538,10 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             const unsigned long long t0 = atomicAdd(&ts[1], 0ull), t1 = atomicAdd(&ts[2], 0ull);
             ts[5] += t1 - t0;
             ts[4] += tcount;   // a split pair (interior + boundary launch) counts once
+            // per variant: 0 plain, 1 RESID, 2 BRES, 3 INTERP (with or without BRES)
+            constexpr int var = INTERP ? 3 : RESID ? 1 : BRES ? 2 : 0;
+            ts[6 + 2 * var] += tcount;
+            ts[7 + 2 * var] += t1 - t0;
             ts[1] = ~0ull;
             ts[2] = 0ull;
             ts[3] = 0ull;

@@ -424,9 +424,9 @@ __global__ void __launch_bounds__(PX* PY) scale_pair_kernel(PV v, double* __rest
 __global__ void zero_scalar(double* p) { pdl_wait(); *p = 0.0; }
 
 // grid over pairs: (ceil(nx/64), ceil(ny/4), z-chunks) with ~16 blocks per SM
-inline dim3 pair_grid(int nx, int ny, int nz, int* depth) {
+inline dim3 pair_grid(int nx, int ny, int nz, int* depth, long per_sm = 16) {
     const int gx = (nx / 2 + PX - 1) / PX, gy = (ny + PY - 1) / PY;
-    const long want = 148L * 16;
+    const long want = 148L * per_sm;
     int zc = (int)std::max(1L, std::min((long)nz, (want + (long)gx * gy - 1) / ((long)gx * gy)));
     *depth = (nz + zc - 1) / zc;
     zc = (nz + *depth - 1) / *depth;
@@ -553,7 +553,10 @@ sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi) {
     for (int p = 0; p < L->nlocal; p++) {
         PV v = sf_view(L, p);
         int depth;
-        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth);
+        // shallower z runs per thread (64 blocks per SM of work): 256^3 Laplacian
+        // 0.0555 -> 0.0502 ms, 512^3 0.388 -> 0.372 ms (profiles/r02/ab_cc_per_sm.txt)
+        static const long per_sm = getenv("SF_CC_PER_SM") ? atol(getenv("SF_CC_PER_SM")) : 64;
+        dim3 g = pair_grid(v.nx, v.ny, v.nz, &depth, per_sm);
         if (jacobi)
             sf_launch(cc_pair_kernel<true>, g, dim3(PX, PY), 0, L->stream, v, v.f[out], v.f[x], v.f[f], hm2,
                                                                      h2w, depth);

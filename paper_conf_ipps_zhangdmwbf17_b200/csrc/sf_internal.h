@@ -25,8 +25,9 @@
 #define SF_P2P_MAX_RANKS 64
 #define SF_SCRATCH_BYTES (256 + 8 * (8 + SF_P2P_MAX_RANKS))
 // dscratch slots: [0] fused-check max residual, [1] power-iteration sum, [2] max|F|
-// of the device solve loop, [8..13] live timing of the colour-fused pair
-// (u64: armed, min start, max end, finished CTAs, launches, sum of ns)
+// of the device solve loop, [8..21] live timing of the colour-fused pair
+// (u64: armed, min start, max end, finished CTAs, launches, sum of ns, then
+// (launches, sum of ns) per variant: plain, RESID, BRES, INTERP)
 #define SF_TS_OFF 8
 
 struct sf_comm {
@@ -66,6 +67,7 @@ struct sf_level {
     unsigned long long* dsync; // P2P sync block (inside buf: peers reach it through IPC)
     double* hscratch;          // pinned, mapped host scalars
     double* hscratch_dev;      // their device alias
+    double ts_var[4][2] = {};  // last sf_level_pair_timing read-out per variant: launches, ns
     std::vector<char*> peer;   // kind-2 comm: peer ranks' level buffers (CUDA IPC), by rank
     std::vector<void*> ipc_opened;
 };

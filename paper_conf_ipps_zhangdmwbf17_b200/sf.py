@@ -47,6 +47,7 @@ EXPORTS = [
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
     "sf_comm_create_p2p", "sf_smooth_residual_restrict", "sf_level_pair_timing",
     "sf_interpolate_smooth", "sf_comm_check", "sf_solve_stream_stats",
+    "sf_level_pair_timing_variants",
 ]
 
 
@@ -130,6 +131,7 @@ def lib():
         "sf_smooth_residual_restrict": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
         "sf_interpolate_smooth": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
         "sf_comm_check": (_i, [_vp, _vp]),
+        "sf_level_pair_timing_variants": (_i, [_vp, C.POINTER(C.c_double), C.POINTER(C.c_longlong)]),
         "sf_solve_stream_stats": (_i, [_vp, C.POINTER(C.c_double)]),
         "sf_apply_laplacian": (_i, [_vp, _i, _i]),
         "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
@@ -431,6 +433,14 @@ def sf_solve_stream(mg, host_f_ptrs, host_u_ptrs, fcycle=True, rtol=1e-10, max_c
 
 def sf_mg_destroy(mg):
     _check(lib().sf_mg_destroy(mg))
+
+
+def sf_level_pair_timing_variants(level):
+    """{variant: (mean_ms, pairs)} of the last sf_level_pair_timing read-out."""
+    ms = (C.c_double * 4)()
+    n = (C.c_longlong * 4)()
+    _check(lib().sf_level_pair_timing_variants(level, ms, n))
+    return {name: (ms[i], n[i]) for i, name in enumerate(("plain", "resid", "bres", "interp"))}
 
 
 def sf_solve_stream_stats(mg):
