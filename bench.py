@@ -388,7 +388,7 @@ def main():
         }
         line.update({k: v for k, v in side.items() if k in (
             "e2e", "gsrb_c3", "vcycle", "fcycle", "fcycle_strong", "read_bw", "cpu_baseline", "fig7_256",
-            "gsrb_size_sweep", "dsl_256", "c1_16", "c2_64")})
+            "gsrb_size_sweep", "dsl_256", "c1_16", "c2_64") or k.startswith("fig7_")})
         print(json.dumps(line), flush=True)
     M.close()
     L.close()
@@ -450,6 +450,21 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
     out["read_bw"] = {"ms": rms, "gbs": 8 * dof_local / (rms / 1e3) / 1e9,
                       "kernel": "norm_pair_kernel (sum of squares, 8 B/cell read)",
                       "note": "includes per-call host sync; context for the copy peak"}
+    # Fig 7's CC operators (NEXT-2) at the workload's finest level as well
+    # (PAPER.md:698-784 quote them at 256^3 only; gsrb_c3 / fig7_256 below)
+    if rank == 0 and world == 1:
+        pk, _ = peaks()
+        fig7b = {}
+        for name, fn, bpc in (
+                ("cc_7pt_laplacian", lambda: sf.sf_apply_laplacian(L.handle, sf.SF_R, sf.SF_U), 16),
+                ("cc_jacobi_w2/3", lambda: sf.sf_jacobi(L.handle, sf.SF_R, sf.SF_U, sf.SF_F,
+                                                         2.0 / 3.0), 24)):
+            m_ = timed(fn, 20, warm=3)
+            fig7b[name] = {"ms": m_, "gstencil_s": dof_local / (m_ / 1e3) / 1e9,
+                           "alg_gbs": bpc * dof_local / (m_ / 1e3) / 1e9,
+                           "frac_of_peak": bpc * dof_local / (m_ / 1e3) / 1e9 / pk,
+                           "bytes_per_cell": bpc}
+        out[f"fig7_{nx}"] = fig7b
     # pairs on the finest level per solve: F: (pre+post) ; each V: 4 pairs
     pairs_per_solve = 4 * cyc
     out["fine_pair_share"] = None

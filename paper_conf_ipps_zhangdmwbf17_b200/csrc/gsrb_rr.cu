@@ -29,6 +29,11 @@
 //
 // Single-part levels only (the extended z range reads 3 planes past the
 // chunk); the V-cycle falls back to pair + residual_restrict elsewhere.
+// Built only with SF_WITH_RR (build.py: environment SF_BUILD_RR=1): measured
+// slower than the separate passes on B200 (below), so the default library
+// carries the stubs at the end of this file and sf_smooth_residual_restrict
+// takes the composite path.
+#ifdef SF_WITH_RR
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -465,3 +470,15 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
     SF_LAUNCHED();
     return sf_check_launch("gsrb_rr");
 }
+
+#else   // !SF_WITH_RR
+
+#include "sf_internal.h"
+
+bool gsrb_rr_supported(const sf_level*, const sf_level*) { return false; }
+
+sf_status k_gsrb_pair_rr(sf_level*, int, int, int, double, double, sf_level*, int) {
+    return sf_fail(SF_ERR_SHAPE, "fused pair+residual+restriction not built (SF_BUILD_RR=1)");
+}
+
+#endif  // SF_WITH_RR

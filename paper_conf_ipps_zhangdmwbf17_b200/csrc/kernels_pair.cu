@@ -505,11 +505,11 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
             }
             // test / tuning overrides: chunk depth (coarse planes) and grid size,
             // so small levels take the multi-plane, multi-item paths of 512^3
-            if (const char* e = getenv("SF_RR_DEPTH"))
+            if (const char* e = getenv("SF_RRZS_DEPTH"))
                 if (atoi(e) > 0) best_d = std::min(nK, atoi(e));
             const int items = tiles * ((nK + best_d - 1) / best_d);
             int grid = std::min(items, G);
-            if (const char* e = getenv("SF_RR_GRID"))
+            if (const char* e = getenv("SF_RRZS_GRID"))
                 if (atoi(e) > 0) grid = std::min(items, atoi(e));
 #define SF_RRZS(MB)                                                                              \
     sf_launch(residual_restrict_zs_kernel<MB>, grid, dim3(PX, PY), 0, F->stream,                         \

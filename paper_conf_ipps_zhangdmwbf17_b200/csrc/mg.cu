@@ -13,7 +13,19 @@
 #include <cmath>
 #include <cstdlib>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "sf_internal.h"
+
+// NVTX ranges per cycle and level (Nsight timelines; inert without a tool)
+struct NvtxRange {
+    explicit NvtxRange(const char* fmt, int a = 0, int b = 0, int c = 0, int d = 0) {
+        char name[96];
+        snprintf(name, sizeof(name), fmt, a, b, c, d);
+        nvtxRangePushA(name);
+    }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 // Device-resident solve loop (sf_solve with graphs): termination is decided on
 // the device and drives a CUDA-graph WHILE node, so a whole solve is one graph
@@ -329,6 +341,7 @@ static sf_status bres_pair(sf_mg* m, sf_level* L) {
 static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
     const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
+    NvtxRange nv("sf V(l=%d) %dx%dx%d", l, L->gnx, L->gny, L->gnz);
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one launch
         return k_coarse_vcycle(&m->lv[l], (int)m->lv.size() - l, m->a, m->b, m->ainv,
@@ -381,6 +394,7 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
 
 static sf_status fcyc(sf_mg* m) {
     int nl = (int)m->lv.size();
+    NvtxRange nv("sf F-cycle %d levels", nl);
     for (int l = 1; l < nl; l++)
         SF_TRY(k_restrict(m->lv[l], SF_F, m->lv[l - 1], SF_F, SF_RESTRICT_CELL));
     SF_TRY(k_bottom_solve(m->lv[nl - 1], SF_U, SF_F, m->ainv));
@@ -783,6 +797,7 @@ extern "C" sf_status sf_fcycle(sf_mg* m) {
 extern "C" sf_status sf_solve(sf_mg* m, int fcycle, double rtol, int max_cycles, int* cycles,
                               double* hist) {
     if (!m) return sf_fail(SF_ERR_INVALID, "NULL mg");
+    NvtxRange nv("sf solve fcycle=%d max_cycles=%d", fcycle, max_cycles);
     // hist holds max_cycles entries (sf.h): a silent default cap would overrun it
     if (max_cycles < 1) return sf_fail(SF_ERR_INVALID, "max_cycles must be >= 1");
     if (!(rtol > 0)) rtol = m->o.rtol;

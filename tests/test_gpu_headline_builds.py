@@ -6,7 +6,7 @@ PAPER.md:597, 647-653) to the 32x16 / 5-deep build (level.cu, levels above
 2^24 cells), and the fused residual + restriction (A6 + A7) walks
 many multi-plane z-chunks per persistent CTA.  Small levels would take the
 32x8 build and one-plane chunks; the test-only overrides SF_INTERP_T32_CELLS,
-SF_RR_DEPTH and SF_RR_GRID force the headline's paths on sizes the oracle
+SF_RRZS_DEPTH and SF_RRZS_GRID force the headline's paths on sizes the oracle
 solves in seconds.  Tolerances: 1e-12 relative per pair / restriction (plus a
 max-abs bound relative to the largest value, so one wrong cell cannot hide in
 an L2 norm), 1e-11 per V/F-cycle."""
@@ -39,7 +39,7 @@ def maxrel(a, b):
     return np.abs(a - b).max() / max(np.abs(b).max(), 1e-300)
 
 
-HEADLINE_PATHS = {"SF_INTERP_T32_CELLS": "0", "SF_RR_DEPTH": "3", "SF_RR_GRID": "7"}
+HEADLINE_PATHS = {"SF_INTERP_T32_CELLS": "0", "SF_RRZS_DEPTH": "3", "SF_RRZS_GRID": "7"}
 
 
 @pytest.mark.parametrize("shape", [(16, 32, 64), (24, 48, 96), (64, 64, 64), (40, 16, 128)])
@@ -170,9 +170,9 @@ def test_smooth_residual_restrict_chunking(sf, oracle, depth, grid, monkeypatch)
     """sf_smooth_residual_restrict's coarse rhs = R_cell(rhs - A x) of the
     smoothed x, for z-chunkings from one plane per item to one item per CTA
     walking the whole level, vs the oracle (1e-12)."""
-    monkeypatch.setenv("SF_RR_DEPTH", depth)
+    monkeypatch.setenv("SF_RRZS_DEPTH", depth)
     if grid:
-        monkeypatch.setenv("SF_RR_GRID", grid)
+        monkeypatch.setenv("SF_RRZS_GRID", grid)
     shape = (26, 32, 64)
     nz, ny, nx = shape
     h = I.level_h(nx, ny, nz)
