@@ -83,7 +83,8 @@ enum sf_norm_kind { SF_NORM_MAX = 0, SF_NORM_L2 = 1 };
 enum sf_smoother_kind { SF_SMOOTH_AUTO = 0,     /* fused when the shape allows */
                         SF_SMOOTH_COLOUR = 1,   /* one kernel per colour sweep  */
                         SF_SMOOTH_FUSED = 2,    /* colour-fused RB pair         */
-                        SF_SMOOTH_CHEBY = 3 };  /* NEXT-3 Chebyshev (mg option) */
+                        SF_SMOOTH_CHEBY = 3,    /* NEXT-3 Chebyshev (mg option) */
+                        SF_SMOOTH_FUSED2 = 4 }; /* NEXT-1 two RB pairs per pass  */
 
 typedef struct sf_comm sf_comm;
 typedef struct sf_level sf_level;
@@ -208,6 +209,11 @@ sf_status sf_apply_op(sf_level* level, int out, int x, double a, double b);
  * two ids, so with x = SF_TMP and kind SF_SMOOTH_FUSED the buffer U named before
  * the call is overwritten.  SF_SMOOTH_AUTO takes the fused kernel only for
  * x = SF_U (TMP is then the clobbered scratch), otherwise the colour sweeps.
+ * SF_SMOOTH_FUSED2 (NEXT-1): every two pairs
+ * run as ONE pass of a temporally blocked kernel (4 sweeps per HBM pass, the
+ * result bit-identical to two fused pairs), an odd last pair as one fused
+ * pair; same field rules as FUSED, single-part levels with nx % 32 == 0 and
+ * ny % 8 == 0 (SF_ERR_SHAPE otherwise).
  * kind: enum sf_smoother_kind. */
 sf_status sf_smooth_gsrb(sf_level* level, int x, int rhs, double a, double b, int rb_pairs, int kind);
 /* A6: res = rhs - A x */

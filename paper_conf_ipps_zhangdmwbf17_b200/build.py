@@ -32,6 +32,7 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            # stubs unless SF_BUILD_RR=1
            ("gsrb_rr.cu", "gsrb_rr.o", ["-DSF_WITH_RR"] if os.environ.get("SF_BUILD_RR") == "1" else []),
            ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []), ("coarse.cu", "coarse.o", []),
+           ("gsrb_twopair.cu", "gsrb_twopair.o", []),
            ("stencil.cu", "stencil.o", [])]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -468,6 +468,22 @@ extern "C" sf_status sf_smooth_gsrb(sf_level* L, int x, int rhs, double a, doubl
         return sf_fail(SF_ERR_INVALID, "x, rhs and DINV must be distinct fields");
     bool fused_ok = gsrb_fused_supported(L) && (x == SF_U || x == SF_TMP) && rhs != SF_TMP &&
                     rhs != SF_U;
+    if (kind == SF_SMOOTH_FUSED2) {   // NEXT-1: two pairs per pass
+        if (!fused_ok || !gsrb_twopair_supported(L))
+            return sf_fail(SF_ERR_SHAPE, "two-pair smoother unsupported for this level/fields");
+        if (rb_pairs == 0) return SF_OK;
+        int other = (x == SF_U) ? SF_TMP : SF_U;
+        SF_TRY(sf_halo(L, rhs, 1));
+        for (int p = 0; p + 1 < rb_pairs; p += 2) {
+            SF_TRY(k_gsrb_twopair(L, x, other, rhs, a, b));
+            sf_swap_fields(L, x, other);
+        }
+        if (rb_pairs & 1) {
+            SF_TRY(k_gsrb_pair_halo(L, x, other, rhs, a, b));
+            sf_swap_fields(L, x, other);
+        }
+        return SF_OK;
+    }
     if (kind == SF_SMOOTH_FUSED && !fused_ok)
         return sf_fail(SF_ERR_SHAPE, "fused smoother unsupported for this level/fields");
     // the fused pair ping-pongs x through the other of U / TMP; AUTO only takes

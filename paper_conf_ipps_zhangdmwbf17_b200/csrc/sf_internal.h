@@ -205,6 +205,10 @@ sf_status k_gsrb_pair_halo(sf_level* L, int xin, int xout, int rhs, double a, do
                            int rmode = SF_RM_NONE);
 // halo exchange enqueued on stream s instead of the level's stream (kinds 0, 1, 3)
 sf_status sf_halo_on(sf_level* L, int field, int depth, cudaStream_t s);
+// NEXT-1: two RB pairs in one pass (gsrb_twopair.cu): xout = pair(pair(xin));
+// single-part levels, nx % 32 == 0, ny % 8 == 0
+bool gsrb_twopair_supported(const sf_level* L);
+sf_status k_gsrb_twopair(sf_level* L, int xin, int xout, int rhs, double a, double b);
 // last pre-smoothing pair fused with residual + restriction (gsrb_rr.cu):
 // xout = pair(xin); C.cf = R_cell(rhs - A xout).  Single-part levels, 32x16 tiles.
 bool gsrb_rr_supported(const sf_level* F, const sf_level* C);

@@ -29,7 +29,7 @@ SF_NFIELDS = 9
 SF_RESTRICT_CELL, SF_RESTRICT_FACE_I, SF_RESTRICT_FACE_J, SF_RESTRICT_FACE_K = range(4)
 SF_INTERP_P0, SF_INTERP_PL = 0, 1
 SF_NORM_MAX, SF_NORM_L2 = 0, 1
-SF_SMOOTH_AUTO, SF_SMOOTH_COLOUR, SF_SMOOTH_FUSED, SF_SMOOTH_CHEBY = 0, 1, 2, 3
+SF_SMOOTH_AUTO, SF_SMOOTH_COLOUR, SF_SMOOTH_FUSED, SF_SMOOTH_CHEBY, SF_SMOOTH_FUSED2 = 0, 1, 2, 3, 4
 
 FIELD_IDS = {"u": SF_U, "f": SF_F, "r": SF_R, "tmp": SF_TMP, "alpha": SF_ALPHA,
              "beta_i": SF_BETA_I, "beta_j": SF_BETA_J, "beta_k": SF_BETA_K, "dinv": SF_DINV}
