@@ -41,8 +41,8 @@ def _smooth(sf, shape, coeffs, x, f, kind, pairs, h):
     return u
 
 
-@pytest.mark.parametrize("shape", [(24, 16, 64), (37, 24, 96), (64, 64, 64), (9, 8, 32), (3, 16, 32),
-                                   (1, 8, 32)])
+@pytest.mark.parametrize("shape", [(24, 16, 64), (37, 32, 96), (64, 64, 64), (9, 16, 32), (3, 16, 32),
+                                   (2, 16, 32)])
 @pytest.mark.parametrize("depth", [None, "1", "2", "5"])
 def test_twopair_bit_identical_to_two_pairs(sf, oracle, shape, depth, monkeypatch):
     if depth:
