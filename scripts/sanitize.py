@@ -54,3 +54,31 @@ st, cyc, hist = M.solve(fcycle=True, rtol=1e-10, raise_on_error=False)
 sf.sf_sync(L.handle)
 print("ok graph solve", cyc, flush=True)
 M.close(); L.close()
+
+# r02 kernels: NEXT-1 two-pair smoother (4 chunk depths incl. ragged ones),
+# sf_interpolate_smooth on the 32x16 P0-fused build, the persistent residual +
+# restriction with forced multi-item chunking; the coarse single-CTA V-cycle
+# runs inside every solve above (levels <= 16^3)
+for dep in ("0", "1", "3", "7"):
+    if dep != "0":
+        os.environ["SF_TWOPAIR_DEPTH"] = dep
+    L = sf.Level(64, 32, 20, 1.0 / 64)
+    sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
+    sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+    sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 3, sf.SF_SMOOTH_FUSED2)
+    sf.sf_sync(L.handle)
+    L.close()
+os.environ.pop("SF_TWOPAIR_DEPTH", None)
+print("ok twopair", flush=True)
+os.environ["SF_INTERP_T32_CELLS"] = "0"
+os.environ["SF_RRZS_DEPTH"] = "3"
+os.environ["SF_RRZS_GRID"] = "5"
+F = sf.Level(64, 32, 24, 1.0 / 64)
+C = sf.Level(32, 16, 12, 2.0 / 64)
+sf.sf_init_problem(F.handle, 1, 1.0, 1.0, 1)
+sf.sf_rebuild_operator(F.handle, 1.0, 1.0)
+sf.sf_interpolate_smooth(F.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, sf.SF_U)
+sf.sf_smooth_residual_restrict(F.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, sf.SF_F)
+sf.sf_sync(F.handle)
+print("ok interp t32 / rr chunks", flush=True)
+F.close(); C.close()
