@@ -121,6 +121,8 @@ extern "C" sf_status sf_comm_create_nccl(sf_comm** out, const unsigned char id[1
     return SF_OK;
 }
 
+static void ensure_err_word();
+
 static sf_status create_ipc_comm(sf_comm** out, int nranks, int rank, sf_host_allgather_fn fn,
                                  void* user, int kind) {
     if (!out || !fn || nranks < 1 || rank < 0 || rank >= nranks)
@@ -134,6 +136,9 @@ static sf_status create_ipc_comm(sf_comm** out, int nranks, int rank, sf_host_al
     c->nccl = nullptr;
     c->hostfn = fn;
     c->hostuser = user;
+    // the p2p timeout's mapped host word is allocated here, never inside a
+    // stream capture (a pinned allocation there would abort the capture)
+    if (kind == 3) ensure_err_word();
     *out = c;
     return SF_OK;
 }
@@ -317,23 +322,24 @@ static unsigned long long* g_err_host = nullptr;
 static unsigned long long* g_err_dev = nullptr;
 static std::mutex g_err_mu;
 
+static void ensure_err_word() {
+    std::lock_guard<std::mutex> lk(g_err_mu);
+    if (g_err_host) return;
+    void* h = nullptr;
+    void* d = nullptr;
+    if (cudaHostAlloc(&h, 64, cudaHostAllocMapped) == cudaSuccess &&
+        cudaHostGetDevicePointer(&d, h, 0) == cudaSuccess) {
+        memset(h, 0, 64);
+        g_err_host = (unsigned long long*)h;
+        g_err_dev = (unsigned long long*)d;
+    } else {
+        cudaGetLastError();
+    }
+}
+
 static P2PPeers peers_init() {
     P2PPeers pe = {};
-    {
-        std::lock_guard<std::mutex> lk(g_err_mu);
-        if (!g_err_host) {
-            void* h = nullptr;
-            void* d = nullptr;
-            if (cudaHostAlloc(&h, 64, cudaHostAllocMapped) == cudaSuccess &&
-                cudaHostGetDevicePointer(&d, h, 0) == cudaSuccess) {
-                memset(h, 0, 64);
-                g_err_host = (unsigned long long*)h;
-                g_err_dev = (unsigned long long*)d;
-            } else {
-                cudaGetLastError();
-            }
-        }
-    }
+    ensure_err_word();
     pe.err = g_err_dev;
     static const double secs = getenv("SF_P2P_TIMEOUT_S") ? atof(getenv("SF_P2P_TIMEOUT_S")) : 60.0;
     pe.timeout_ns = (unsigned long long)(std::max(secs, 1e-3) * 1e9);
