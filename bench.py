@@ -279,11 +279,13 @@ def main():
             comm.close()
             print(f"bench: p2p transport unavailable ({e}); using NCCL", file=sys.stderr)
             comm = sf.Comm.nccl()
+            sf.sf_comm_check(comm.h, torch.cuda.current_stream().cuda_stream)   # health check
             transport = "nccl (p2p unavailable)"
             L = sf.Level(nx, ny, nz, h, comm=comm)
     else:
         if world > 1:
             comm = sf.Comm.nccl()
+            sf.sf_comm_check(comm.h, torch.cuda.current_stream().cuda_stream)   # health check
         L = sf.Level(nx, ny, nz, h, comm=comm)
     sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)       # HPGMG problem + manufactured f
     M = sf.MG(L, 1.0, 1.0)
