@@ -388,7 +388,9 @@ sf_status sf_stream_sync(sf_level* L) {
                 return sf_fail(SF_ERR_NCCL, "NCCL wait exceeded %.0f s (SF_NCCL_TIMEOUT_S); "
                                "communicator aborted", secs);
             }
-            std::this_thread::sleep_for(std::chrono::microseconds(50));
+            // spin for the first millisecond (a solve cycle's sync), then back off
+            if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > 1e-3)
+                std::this_thread::sleep_for(std::chrono::microseconds(50));
         }
     }
     cudaError_t e = cudaStreamSynchronize(L->stream);
