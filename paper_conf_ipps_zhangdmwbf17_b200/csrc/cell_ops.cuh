@@ -1,6 +1,6 @@
-// Per-cell A3 operator shared by the one-thread-per-cell kernels (kernels.cu)
-// and the coarse-level cluster V-cycle (coarse.cu): one definition, so both
-// evaluate the operator with the same terms, order and roundings.
+// Per-cell A3 operator of the one-thread-per-cell kernels (kernels.cu): one
+// definition, so every one of them evaluates the operator with the same terms,
+// order and roundings.
 #pragma once
 
 // x loads: plain (L1-cached) or .cg (L2 only: the cluster kernel reads values
