@@ -1,349 +1,651 @@
-// Coarse-level V-cycle in ONE launch of ONE CTA (A9 on the smallest levels).
+// Coarse-level V-cycle in ONE launch of ONE thread-block cluster (A9 on the
+// smallest levels).
 //
-// Levels of 16^3 cells and fewer are pure latency: every colour sweep,
+// Levels of 32^3 cells and fewer are pure latency: every colour sweep,
 // residual + restriction, P0 interpolation and the bottom solve of V(l)
-// (A5-A9) is well under a microsecond of
-// work behind a launch of its own -- ~30 launches per V-cycle below 32^3.
-// Here one 512-thread CTA runs the whole V(l0) .. bottom .. V(l0) recursion
-// with every operand in SHARED MEMORY OR REGISTERS, phases separated by
-// __syncthreads: after one staging pass at the start, no phase touches global
-// memory (the previous design read alpha / beta through L1/L2 in every phase,
-// ~1.2 us per phase; profiles/r02/coarse_smem_staging.txt).
+// (A5-A9) is a few microseconds of work
+// behind a launch of its own -- ~40 launches per V-cycle below 64^3.  Here one
+// cluster of C = nz/2 CTAs (entry level nz <= 32: up to 16 CTAs, one per SM)
+// runs the whole V(l0) .. bottom .. V(l0) recursion with every operand in
+// REGISTERS or SHARED MEMORY; phases are separated by cluster barriers and the
+// z-neighbours that live in the next CTA are read through distributed shared
+// memory (DSMEM).  After one staging pass no phase touches global memory.
 //
-// Shared memory, compact per level (nx*ny*nz cells, x fastest):
-//   U                              every level
-//   F, Dinv, alpha                 every level below the entry level
-//   beta_i (nx+1 faces per row), beta_j (ny+1 rows per plane),
-//   beta_k (nz+1 planes)           every level above the bottom
-// The entry level's F, Dinv and alpha (3 x 32 KB at 16^3 would not fit next to
-// its faces) live in REGISTERS: thread t owns the 2x2x2 block of entry cells
-// whose parent is coarse cell t (at most 512 blocks = 4096 cells), so its
-// colour sweeps, its residual + restriction into parent t and the P0
-// correction from parent t touch only its own F / Dinv / alpha.  Levels below
-// the entry run one thread per cell with everything in shared memory.
+// Ownership: on every smoothed level CTA c owns the 2-plane layer of 2x2x2
+// blocks whose parents form coarse plane c (planes 2c, 2c+1), so the
+// restriction of a block and the P0 correction of its cells involve only the
+// block's CTA and the owner of the parent plane (CTA c/2 on the next smoothed
+// level, CTA 0 for the bottom, which holds the whole coarsest level).
 //
-// Arithmetic: op_sh is op_at's expression (cell_ops.cuh: same terms, order and
+// Entry level: thread t of CTA c owns block t of the layer and keeps its
+// 8 x values, F, Dinv, alpha and the 36 face coefficients of the block in
+// registers; its x values are mirrored in shared memory for the neighbours'
+// reads.  Levels below: one thread per cell of a colour, U / F / Dinv / alpha
+// and the faces of the CTA's two planes in shared memory.
+//
+// Arithmetic: op7 is op_at's expression (cell_ops.cuh: same terms, order and
 // Dirichlet fold); the colour sweep is gsrb_colour_kernel's update
 // x += Dinv (rhs - A x); the residual + restriction sums rhs - A x over the 8
 // children in restrict_cell's order and divides by 8; P0 adds the parent; the
-// bottom applies the exact inverse in bottom_solve_kernel's order.
+// bottom applies the exact inverse in bottom_solve_kernel's order -- so the
+// launch reproduces the per-phase kernels bit for bit.
+#include <cooperative_groups.h>
+
+#include <algorithm>
 #include <cstdlib>
 
 #include "sf_internal.h"
 
+namespace cg = cooperative_groups;
+
 namespace {
 
-constexpr int CMAXL = 8;                    // levels per launch
-constexpr int CNT = 512;                    // threads = entry-level 2x2x2 blocks at most
-constexpr long CMAX_CELLS = 8L * CNT;       // entry level at most 4096 cells (16^3)
-constexpr int CSMEM_MAX = 227 * 1024;       // opt-in shared memory per CTA
+constexpr int CMAXL = 8;                 // levels per launch
+constexpr int NT = 256;                  // threads per CTA (entry blocks per layer at most)
+constexpr int CS_MAX = 16;               // CTAs per cluster (non-portable above 8)
+constexpr int BOT_MAX = 64;              // bottom cells (plan_levels: <= 64)
+constexpr int GMAX = 2 * NT;             // levels of at most this many cells are gathered on CTA 0
+constexpr int CSMEM_MAX = 225 * 1024;    // opt-in shared memory per CTA (2 KB for static use)
 
-struct CLevel {
-    PV v;                 // global view: coefficients, the entry level's U / F / Dinv
+struct KLevel {
+    PV v;                 // global view: coefficients; the entry level's U / F / Dinv
     double bh2;
-    int lx, ly, lz;       // log2 of nx, ny, nz (power-of-two levels: cell indices by shifts)
-    int u, f, d, al;      // shared offsets (doubles) of U, F, Dinv, alpha (f/d/al: below entry)
-    int bi, bj, bk;       // shared offsets of the face coefficients (above the bottom)
+    int lx, ly, lz;       // log2 of nx, ny, nz (power-of-two levels)
+    int u, f, d, al;      // shared offsets (doubles) of U, F, Dinv, alpha: the CTA's two planes
+    int bi, bj, bk;       // (gathered: every plane, on CTA 0; bottom: U and F only); faces
+    int g;                // gathered on CTA 0 (the coarsest levels, <= GMAX cells)
 };
 
-struct CoarseArgs {
-    CLevel lv[CMAXL];
-    int nlev;             // lv[0] = V's entry level, lv[nlev-1] = bottom
+struct KArgs {
+    KLevel lv[CMAXL];
+    int nlev;             // lv[0] = entry, lv[nlev-1] = bottom
     int pre, post;        // RB pairs
     double a;
-    const double* ainv;   // exact inverse of the bottom operator (n x n)
+    int ainv;             // shared offset of the bottom inverse (CTA 0)
+    int rscr;             // shared offset of the residual scratch (GMAX doubles)
+    const double* ainv_g; // n x n, row major
 };
 
-// A3 at (i,j,k) of a level held in shared memory; xc = x(i,j,k), al = alpha(i,j,k).
-// op_at's expression term by term.
-__device__ __forceinline__ double op_sh(const CLevel& L, const double* sm, int i, int j, int k,
-                                        double xc, double al, double a) {
-    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
-    const int sy = nx, sz = nx << L.ly;
-    const int c = i + (j << L.lx) + (k << (L.lx + L.ly));
-    const double* x = sm + L.u;
-    const double xw = (i == 0) ? -xc : x[c - 1];
-    const double xe = (i == nx - 1) ? -xc : x[c + 1];
-    const double xs = (j == 0) ? -xc : x[c - sy];
-    const double xn = (j == ny - 1) ? -xc : x[c + sy];
-    const double xb = (k == 0) ? -xc : x[c - sz];
-    const double xt = (k == nz - 1) ? -xc : x[c + sz];
-    const double* bi = sm + L.bi + i + (nx + 1) * (j + (k << L.ly));
-    const double* bj = sm + L.bj + i + ((j + (ny + 1) * k) << L.lx);
-    const double* bk = sm + L.bk + c;
-    double flux = bi[1] * (xe - xc);
-    flux += bi[0] * (xw - xc);
-    flux += bj[sy] * (xn - xc);
-    flux += bj[0] * (xs - xc);
-    flux += bk[sz] * (xt - xc);
-    flux += bk[0] * (xb - xc);
-    return a * al * xc - L.bh2 * flux;
+// A3 at one cell from its value, its six neighbours (Dirichlet ghosts already
+// folded in as -xc) and its six faces: op_at's expression term by term.
+__device__ __forceinline__ double op7(double xc, double xw, double xe, double xs, double xn,
+                                     double xb, double xt, double bw, double be, double bs,
+                                     double bn, double bb, double bt, double al, double a,
+                                     double bh2) {
+    double flux = be * (xe - xc);
+    flux += bw * (xw - xc);
+    flux += bn * (xn - xc);
+    flux += bs * (xs - xc);
+    flux += bt * (xt - xc);
+    flux += bb * (xb - xc);
+    return a * al * xc - bh2 * flux;
 }
 
-// The entry level's 2x2x2 block owned by this thread: origin (2I, 2J, 2K),
-// sub-cell s = di + 2 dj + 4 dk; F / Dinv / alpha in registers.
+// shared memory of this CTA and of its z-neighbours (DSMEM, generic pointers)
+struct Mem {
+    double* sm;
+    double* lo;   // CTA rank-1 (planes below), nullptr at rank 0
+    double* hi;   // CTA rank+1
+    int rank, csize;
+    // shared memory of the CTA that owns plane p of the next level (gathered: CTA 0)
+    __device__ __forceinline__ double* owner(cg::cluster_group& cl, int p, bool gathered) const {
+        const int r = gathered ? 0 : p >> 1;
+        return r == rank ? sm : cl.map_shared_rank(sm, r);
+    }
+};
+
+#ifdef SF_COARSE_TRACE   // phase clock trace (measurement builds only)
+__shared__ long long trace_t[128];
+__shared__ int trace_n;
+#define TRACE()                                                     \
+    do {                                                            \
+        if (threadIdx.x == 0 && trace_n < 128) trace_t[trace_n++] = clock64(); \
+    } while (0)
+#else
+#define TRACE() \
+    do {        \
+    } while (0)
+#endif
+
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                     : "memory");
+    TRACE();
+}
+
+// ------------------------------------------------------------ entry level
 struct Block {
-    int i0, j0, k0;
     bool own;
-    double F[8], D[8], A[8];
+    int i0, j0;                 // block origin (k0 = 2 * rank)
+    double X[8], F[8], D[8], A[8];
+    double BI[3][2][2];         // beta_i faces i0..i0+2 at (dj, dk)
+    double BJ[3][2][2];         // beta_j faces j0..j0+2 at (di, dk)
+    double BK[3][2][2];         // beta_k faces k0..k0+2 at (di, dj)
 };
 
-__device__ __forceinline__ int cell_of(const CLevel& L, int i, int j, int k) {
-    return i + (j << L.lx) + (k << (L.lx + L.ly));
+// A x at sub-cell s = di + 2 dj + 4 dk of the block, with the block's current x
+__device__ __forceinline__ double op_block(const KLevel& L, const Mem& M, const Block& B, int s,
+                                           double a) {
+    const int di = s & 1, dj = (s >> 1) & 1, dk = s >> 2;
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int i = B.i0 + di, j = B.j0 + dj, k = 2 * M.rank + dk;
+    const double xc = B.X[s];
+    const double* U = M.sm + L.u;
+    const int cp = i + (j << L.lx);                   // in-plane offset
+    const int c = cp + (dk << (L.lx + L.ly));         // local cell (plane dk of the CTA)
+    double xw, xe, xs, xn, xb, xt;
+    if (di) { xw = B.X[s - 1]; xe = (i == nx - 1) ? -xc : U[c + 1]; }
+    else    { xe = B.X[s + 1]; xw = (i == 0) ? -xc : U[c - 1]; }
+    if (dj) { xs = B.X[s - 2]; xn = (j == ny - 1) ? -xc : U[c + nx]; }
+    else    { xn = B.X[s + 2]; xs = (j == 0) ? -xc : U[c - nx]; }
+    if (dk) { xb = B.X[s - 4]; xt = (k == nz - 1) ? -xc : (M.hi + L.u)[cp]; }
+    else    { xt = B.X[s + 4]; xb = (k == 0) ? -xc : (M.lo + L.u)[cp + (1 << (L.lx + L.ly))]; }
+    return op7(xc, xw, xe, xs, xn, xb, xt, B.BI[di][dj][dk], B.BI[di + 1][dj][dk], B.BJ[dj][di][dk],
+               B.BJ[dj + 1][di][dk], B.BK[dk][di][dj], B.BK[dk + 1][di][dj], B.A[s], a, L.bh2);
 }
 
-// one colour sweep of the entry level: the thread's 4 cells of colour `colour`
-__device__ __forceinline__ void sweep_entry(const CLevel& L, double* sm, const Block& B, double a,
+__device__ __forceinline__ void sweep_entry(const KLevel& L, const Mem& M, Block& B, double a,
                                             int colour) {
     if (B.own) {
-        double* x = sm + L.u;
+        double* U = M.sm + L.u;
+        // every operator value first (the colour's cells read only the other
+        // colour), then the updates: the neighbour loads -- one of them from the
+        // next CTA -- are all in flight together
+        double ax[8];
+#pragma unroll
+        for (int s = 0; s < 8; s++)
+            if ((((s & 1) + ((s >> 1) & 1) + (s >> 2)) & 1) == colour) ax[s] = op_block(L, M, B, s, a);
 #pragma unroll
         for (int s = 0; s < 8; s++) {
             const int di = s & 1, dj = (s >> 1) & 1, dk = s >> 2;
             if (((di + dj + dk) & 1) != colour) continue;   // block origin is even
-            const int i = B.i0 + di, j = B.j0 + dj, k = B.k0 + dk;
-            const int c = cell_of(L, i, j, k);
-            const double xc = x[c];
-            const double ax = op_sh(L, sm, i, j, k, xc, B.A[s], a);
-            x[c] = xc + B.D[s] * (B.F[s] - ax);
+            B.X[s] = B.X[s] + B.D[s] * (B.F[s] - ax[s]);
+            U[B.i0 + di + ((B.j0 + dj + (dk << L.ly)) << L.lx)] = B.X[s];
         }
     }
-    __syncthreads();
+    cluster_sync();
 }
 
-// one colour sweep of a level below the entry: one thread per cell of the colour
-__device__ __forceinline__ void sweep_cells(const CLevel& L, double* sm, double a, int colour) {
-    const int lh = L.lx - 1;                    // nx >= 2 on every level that is smoothed
-    const int n = 1 << (lh + L.ly + L.lz);      // cells of one colour
-    double* x = sm + L.u;
-    for (int t = threadIdx.x; t < n; t += CNT) {
+// ------------------------------------------------------------ levels below
+// A x at (i, j, plane kl of this CTA) of a non-entry level in shared memory
+__device__ __forceinline__ double op_cell(const KLevel& L, const Mem& M, int i, int j, int kl,
+                                          double xc, double a) {
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int k = 2 * M.rank + kl;
+    const double* U = M.sm + L.u;
+    const int pl = 1 << (L.lx + L.ly);
+    const int cp = i + (j << L.lx), c = cp + kl * pl;
+    const double xw = (i == 0) ? -xc : U[c - 1];
+    const double xe = (i == nx - 1) ? -xc : U[c + 1];
+    const double xs = (j == 0) ? -xc : U[c - nx];
+    const double xn = (j == ny - 1) ? -xc : U[c + nx];
+    double xb, xt;
+    if (kl) { xb = U[cp]; xt = (k == nz - 1) ? -xc : (M.hi + L.u)[cp]; }
+    else    { xt = U[cp + pl]; xb = (k == 0) ? -xc : (M.lo + L.u)[cp + pl]; }
+    const double* bi = M.sm + L.bi + i + (nx + 1) * (j + (kl << L.ly));
+    const double* bj = M.sm + L.bj + i + ((j + (ny + 1) * kl) << L.lx);
+    const double* bk = M.sm + L.bk + c;
+    return op7(xc, xw, xe, xs, xn, xb, xt, bi[0], bi[1], bj[0], bj[nx], bk[0], bk[pl],
+               M.sm[L.al + c], a, L.bh2);
+}
+
+// one colour sweep: thread t updates the t-th cell of the colour in the CTA's two planes
+__device__ __forceinline__ void sweep_cells(const KLevel& L, const Mem& M, double a, int colour) {
+    if (M.rank < (1 << (L.lz - 1))) {
+        const int lh = L.lx - 1;
+        const int n = 1 << (lh + L.ly + 1);   // cells of one colour in two planes
+        double* U = M.sm + L.u;
+        for (int t = threadIdx.x; t < n; t += NT) {
+            const int th = t & ((1 << lh) - 1), r = t >> lh;
+            const int j = r & ((1 << L.ly) - 1), kl = r >> L.ly;
+            const int i = 2 * th + ((j + kl + colour) & 1);   // plane 2*rank+kl: parity of kl
+            const int c = i + ((j + (kl << L.ly)) << L.lx);
+            const double xc = U[c];
+            const double ax = op_cell(L, M, i, j, kl, xc, a);
+            U[c] = xc + M.sm[L.d + c] * (M.sm[L.f + c] - ax);
+        }
+    }
+    cluster_sync();
+}
+
+__device__ __forceinline__ void smooth(const KLevel& L, const Mem& M, Block* B, double a, int pairs) {
+    for (int p = 0; p < pairs; p++) {
+        if (B) {
+            sweep_entry(L, M, *B, a, 0);
+            sweep_entry(L, M, *B, a, 1);
+        } else {
+            sweep_cells(L, M, a, 0);
+            sweep_cells(L, M, a, 1);
+        }
+    }
+}
+
+// coarse cell (I, J) of plane `rank` of level C: its slot in the owner's shared memory
+__device__ __forceinline__ int coarse_slot(const KLevel& C, const Mem& M, int I, int J, bool cgat) {
+    const int kl = cgat ? M.rank : (M.rank & 1);
+    return I + ((J + (kl << C.ly)) << C.lx);
+}
+
+// A6 + A7: C.F = R_cell(F - A U) for the CTA's layer of blocks (coarse plane
+// `rank`), C.U = 0; written into the owner of that coarse plane
+__device__ __forceinline__ void residual_restrict(cg::cluster_group& cl, const KLevel& F,
+                                                  const KLevel& C, const Mem& M, const Block* B,
+                                                  double a, bool cgat, int rscr) {
+    if (M.rank < (1 << (F.lz - 1))) {
+        double* dst = M.owner(cl, M.rank, cgat);
+        if (B) {
+            if (B->own) {
+                double r[8];   // the 8 residuals are independent: evaluated together
+#pragma unroll
+                for (int s = 0; s < 8; s++) r[s] = B->F[s] - op_block(F, M, *B, s, a);
+                double acc = 0.0;
+#pragma unroll
+                for (int s = 0; s < 8; s++) acc += r[s];
+                const int q = coarse_slot(C, M, B->i0 >> 1, B->j0 >> 1, cgat);
+                dst[C.f + q] = acc / 8.0;
+                dst[C.u + q] = 0.0;
+            }
+        } else {
+            // residual of every cell of the two planes (one thread per cell),
+            // then the ordered sums of 8 children (one thread per block)
+            double* R = M.sm + rscr;
+            const int nc = 1 << (F.lx + F.ly + 1);
+            for (int t = threadIdx.x; t < nc; t += NT) {
+                const int i = t & ((1 << F.lx) - 1), j = (t >> F.lx) & ((1 << F.ly) - 1);
+                const int kl = t >> (F.lx + F.ly);
+                R[t] = M.sm[F.f + t] - op_cell(F, M, i, j, kl, M.sm[F.u + t], a);
+            }
+            __syncthreads();
+            const int n = 1 << (F.lx + F.ly - 2);   // blocks of the layer
+            for (int t = threadIdx.x; t < n; t += NT) {
+                const int I = t & ((1 << (F.lx - 1)) - 1), J = t >> (F.lx - 1);
+                double acc = 0.0;
+#pragma unroll
+                for (int s = 0; s < 8; s++)
+                    acc += R[2 * I + (s & 1) + ((2 * J + ((s >> 1) & 1) + ((s >> 2) << F.ly)) << F.lx)];
+                const int q = coarse_slot(C, M, I, J, cgat);
+                dst[C.f + q] = acc / 8.0;
+                dst[C.u + q] = 0.0;
+            }
+        }
+    }
+    cluster_sync();
+}
+
+// A8 P0: the CTA's cells += their parent (coarse plane `rank`, in its owner)
+__device__ __forceinline__ void interp(cg::cluster_group& cl, const KLevel& F, const KLevel& C,
+                                       const Mem& M, Block* B, bool cgat) {
+    if (M.rank < (1 << (F.lz - 1))) {
+        const double* e = M.owner(cl, M.rank, cgat) + C.u;
+        if (B) {
+            if (B->own) {
+                const double ec = e[coarse_slot(C, M, B->i0 >> 1, B->j0 >> 1, cgat)];
+                double* U = M.sm + F.u;
+#pragma unroll
+                for (int s = 0; s < 8; s++) {
+                    B->X[s] = B->X[s] + ec;
+                    U[B->i0 + (s & 1) + ((B->j0 + ((s >> 1) & 1) + ((s >> 2) << F.ly)) << F.lx)] = B->X[s];
+                }
+            }
+        } else {
+            const int n = 1 << (F.lx + F.ly + 1);   // cells of the two planes
+            double* U = M.sm + F.u;
+            for (int t = threadIdx.x; t < n; t += NT) {
+                const int i = t & ((1 << F.lx) - 1), j = (t >> F.lx) & ((1 << F.ly) - 1);
+                U[t] = U[t] + e[coarse_slot(C, M, i >> 1, j >> 1, cgat)];
+            }
+        }
+    }
+    cluster_sync();
+}
+
+// ------------------------------------------------------------ gathered levels
+// The coarsest levels (<= GMAX cells) live whole on CTA 0, which runs their
+// part of the V-cycle alone with __syncthreads between phases (a cluster
+// barrier per phase would cost more than their work); the other CTAs wait at
+// the next cluster barrier.  One thread per cell of a colour / coarse cell.
+
+// A x at (i, j, k) of a gathered level
+__device__ __forceinline__ double op_g(const KLevel& L, const double* sm, int i, int j, int k,
+                                       double xc, double a) {
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int pl = 1 << (L.lx + L.ly);
+    const int c = i + ((j + (k << L.ly)) << L.lx);
+    const double* U = sm + L.u;
+    const double xw = (i == 0) ? -xc : U[c - 1];
+    const double xe = (i == nx - 1) ? -xc : U[c + 1];
+    const double xs = (j == 0) ? -xc : U[c - nx];
+    const double xn = (j == ny - 1) ? -xc : U[c + nx];
+    const double xb = (k == 0) ? -xc : U[c - pl];
+    const double xt = (k == nz - 1) ? -xc : U[c + pl];
+    const double* bi = sm + L.bi + i + (nx + 1) * (j + (k << L.ly));
+    const double* bj = sm + L.bj + i + ((j + (ny + 1) * k) << L.lx);
+    const double* bk = sm + L.bk + c;
+    return op7(xc, xw, xe, xs, xn, xb, xt, bi[0], bi[1], bj[0], bj[nx], bk[0], bk[pl],
+               sm[L.al + c], a, L.bh2);
+}
+
+__device__ __forceinline__ void sweep_g(const KLevel& L, double* sm, double a, int colour) {
+    const int lh = L.lx - 1;
+    const int n = 1 << (lh + L.ly + L.lz);   // cells of one colour
+    double* U = sm + L.u;
+    for (int t = threadIdx.x; t < n; t += NT) {
         const int th = t & ((1 << lh) - 1), r = t >> lh;
         const int j = r & ((1 << L.ly) - 1), k = r >> L.ly;
         const int i = 2 * th + ((j + k + colour) & 1);
-        const int c = cell_of(L, i, j, k);
-        const double xc = x[c];
-        const double ax = op_sh(L, sm, i, j, k, xc, sm[L.al + c], a);
-        x[c] = xc + sm[L.d + c] * (sm[L.f + c] - ax);
+        const int c = i + ((j + (k << L.ly)) << L.lx);
+        const double xc = U[c];
+        const double ax = op_g(L, sm, i, j, k, xc, a);
+        U[c] = xc + sm[L.d + c] * (sm[L.f + c] - ax);
     }
     __syncthreads();
+    TRACE();
 }
 
-__device__ __forceinline__ void smooth(const CLevel& L, double* sm, const Block* B, double a,
-                                       int pairs) {
-    for (int p = 0; p < pairs; p++) {
-        if (B) {
-            sweep_entry(L, sm, *B, a, 0);
-            sweep_entry(L, sm, *B, a, 1);
-        } else {
-            sweep_cells(L, sm, a, 0);
-            sweep_cells(L, sm, a, 1);
-        }
-    }
-}
-
-// A6 + A7 from the entry level: C.F[t] = R_cell(F - A U) over block t; C.U = 0
-__device__ __forceinline__ void residual_restrict_entry(const CLevel& F, const CLevel& C, double* sm,
-                                                        const Block& B, double a) {
-    if (B.own) {
-        const double* x = sm + F.u;
-        double acc = 0.0;
-#pragma unroll
-        for (int s = 0; s < 8; s++) {
-            const int i = B.i0 + (s & 1), j = B.j0 + ((s >> 1) & 1), k = B.k0 + (s >> 2);
-            const double xc = x[cell_of(F, i, j, k)];
-            acc += B.F[s] - op_sh(F, sm, i, j, k, xc, B.A[s], a);
-        }
-        sm[C.f + threadIdx.x] = acc / 8.0;
-        sm[C.u + threadIdx.x] = 0.0;
+// C.F = R_cell(F - A U), C.U = 0: one thread per coarse cell
+// (residual of every fine cell into the scratch R first, one thread per cell)
+__device__ __forceinline__ void restrict_g(const KLevel& F, const KLevel& C, double* sm, double a,
+                                           double* R) {
+    const int nf = 1 << (F.lx + F.ly + F.lz);
+    for (int t = threadIdx.x; t < nf; t += NT) {
+        const int i = t & ((1 << F.lx) - 1), r = t >> F.lx;
+        const int j = r & ((1 << F.ly) - 1), k = r >> F.ly;
+        R[t] = sm[F.f + t] - op_g(F, sm, i, j, k, sm[F.u + t], a);
     }
     __syncthreads();
-}
-
-// A6 + A7 below the entry level: one thread per coarse cell
-__device__ __forceinline__ void residual_restrict_cells(const CLevel& F, const CLevel& C, double* sm,
-                                                        double a) {
     const int n = 1 << (C.lx + C.ly + C.lz);
-    const double* x = sm + F.u;
-    for (int t = threadIdx.x; t < n; t += CNT) {
+    for (int t = threadIdx.x; t < n; t += NT) {
         const int I = t & ((1 << C.lx) - 1), r = t >> C.lx;
         const int J = r & ((1 << C.ly) - 1), K = r >> C.ly;
         double acc = 0.0;
 #pragma unroll
-        for (int s = 0; s < 8; s++) {
-            const int i = 2 * I + (s & 1), j = 2 * J + ((s >> 1) & 1), k = 2 * K + (s >> 2);
-            const int c = cell_of(F, i, j, k);
-            acc += sm[F.f + c] - op_sh(F, sm, i, j, k, x[c], sm[F.al + c], a);
-        }
+        for (int s = 0; s < 8; s++)
+            acc += R[2 * I + (s & 1) + ((2 * J + ((s >> 1) & 1) + ((2 * K + (s >> 2)) << F.ly)) << F.lx)];
         sm[C.f + t] = acc / 8.0;
         sm[C.u + t] = 0.0;
     }
     __syncthreads();
+    TRACE();
 }
 
-// A8 P0 into the entry level: the block's 8 cells += parent t
-__device__ __forceinline__ void interp_entry(const CLevel& F, const CLevel& C, double* sm,
-                                             const Block& B) {
-    if (B.own) {
-        double* y = sm + F.u;
-        const double e = sm[C.u + threadIdx.x];
-#pragma unroll
-        for (int s = 0; s < 8; s++) {
-            const int c = cell_of(F, B.i0 + (s & 1), B.j0 + ((s >> 1) & 1), B.k0 + (s >> 2));
-            y[c] = y[c] + e;
-        }
-    }
-    __syncthreads();
-}
-
-// A8 P0 below the entry level: one thread per fine cell
-__device__ __forceinline__ void interp_cells(const CLevel& F, const CLevel& C, double* sm) {
+// F.U += P0(C.U): one thread per fine cell
+__device__ __forceinline__ void interp_g(const KLevel& F, const KLevel& C, double* sm) {
     const int n = 1 << (F.lx + F.ly + F.lz);
-    double* y = sm + F.u;
-    const double* e = sm + C.u;
-    for (int t = threadIdx.x; t < n; t += CNT) {
+    double* U = sm + F.u;
+    for (int t = threadIdx.x; t < n; t += NT) {
         const int i = t & ((1 << F.lx) - 1), r = t >> F.lx;
         const int j = r & ((1 << F.ly) - 1), k = r >> F.ly;
-        y[t] = y[t] + e[cell_of(C, i >> 1, j >> 1, k >> 1)];
+        U[t] = U[t] + sm[C.u + (i >> 1) + (((j >> 1) + ((k >> 1) << C.ly)) << C.lx)];
     }
     __syncthreads();
+    TRACE();
 }
 
-// R-8: U = A^-1 F on the bottom level (<= 64 cells)
-__device__ __forceinline__ void bottom(const CLevel& B, double* sm, const double* __restrict__ ainv) {
-    const int n = 1 << (B.lx + B.ly + B.lz);
+// R-8: U = A^-1 F on the bottom level
+__device__ __forceinline__ void bottom_g(const KLevel& Bt, double* sm, int ainv) {
+    const int n = 1 << (Bt.lx + Bt.ly + Bt.lz);
     const int r = threadIdx.x;
     if (r < n) {
         double acc = 0.0;
-        for (int c = 0; c < n; c++) acc += __ldg(ainv + r * n + c) * sm[B.f + c];
-        sm[B.u + r] = acc;
+        for (int c = 0; c < n; c++) acc += sm[ainv + r * n + c] * sm[Bt.f + c];
+        sm[Bt.u + r] = acc;
     }
     __syncthreads();
+    TRACE();
 }
 
-// padded global -> compact shared, one 8-byte cp.async per value (no thread
-// waits on a load; one cp.async.wait_all before the first phase).  The box is
-// 2^lw values x 2^lrj rows x rk planes starting at (ioff, joff, 0); shared
-// element (i, j, k) at i + sw (j + srj k).
+// V(l0) .. bottom .. V(l0) over the gathered levels l0..nl-1 (CTA 0 only)
+__device__ __forceinline__ void gathered_cycle(const KArgs& A, double* sm, int l0) {
+    const int nl = A.nlev;
+    for (int l = l0; l + 1 < nl; l++) {
+        for (int p = 0; p < A.pre; p++) {
+            sweep_g(A.lv[l], sm, A.a, 0);
+            sweep_g(A.lv[l], sm, A.a, 1);
+        }
+        restrict_g(A.lv[l], A.lv[l + 1], sm, A.a, sm + A.rscr);
+    }
+    bottom_g(A.lv[nl - 1], sm, A.ainv);
+    for (int l = nl - 2; l >= l0; l--) {
+        interp_g(A.lv[l], A.lv[l + 1], sm);
+        for (int p = 0; p < A.post; p++) {
+            sweep_g(A.lv[l], sm, A.a, 0);
+            sweep_g(A.lv[l], sm, A.a, 1);
+        }
+    }
+}
+
+// padded global -> compact shared, one 8-byte cp.async per value: 2^lw values
+// x 2^lrj rows x rk planes starting at (ioff, joff, koff); shared element
+// (i, j, k) at i + sw (j + srj (k - koff)).
 __device__ __forceinline__ void stage_box(double* dst, const double* __restrict__ src, int lw, int lrj,
-                                          int rk, int ioff, int joff, int sw, int srj, long js,
-                                          long ks) {
+                                          int rk, int ioff, int joff, int koff, int sw, int srj,
+                                          long js, long ks) {
     const unsigned d0 = (unsigned)__cvta_generic_to_shared(dst);
     const int n = rk << (lw + lrj);
-    for (int e = threadIdx.x; e < n; e += CNT) {
+    for (int e = threadIdx.x; e < n; e += NT) {
         const int i = (e & ((1 << lw) - 1)) + ioff, r = e >> lw;
-        const int j = (r & ((1 << lrj) - 1)) + joff, k = r >> lrj;
-        const double* g = src + (long)(k + SF_GZ) * ks + (long)(j + SF_GY) * js + SF_OX + i;
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d0 + 8u * (i + sw * (j + srj * k))),
+        const int j = (r & ((1 << lrj) - 1)) + joff, kr = r >> lrj;
+        const double* g = src + (long)(kr + koff + SF_GZ) * ks + (long)(j + SF_GY) * js + SF_OX + i;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d0 + 8u * (i + sw * (j + srj * kr))),
                      "l"(g)
                      : "memory");
     }
 }
 
-// a cell-centred field of level L (nx x ny x nz)
-__device__ __forceinline__ void stage_cells(double* dst, const double* src, const CLevel& L) {
-    stage_box(dst, src, L.lx, L.ly, 1 << L.lz, 0, 0, 1 << L.lx, 1 << L.ly, L.v.js, L.v.ks);
-}
-
-__global__ void __launch_bounds__(CNT, 1) coarse_vcycle_kernel(const __grid_constant__ CoarseArgs A) {
+__global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_constant__ KArgs A) {
     extern __shared__ double sm[];
+    cg::cluster_group cl = cg::this_cluster();
+    Mem M;
+    M.sm = sm;
+    M.rank = (int)cl.block_rank();
+    M.csize = (int)cl.num_blocks();
+    M.lo = M.rank > 0 ? cl.map_shared_rank(sm, M.rank - 1) : nullptr;
+    M.hi = M.rank + 1 < M.csize ? cl.map_shared_rank(sm, M.rank + 1) : nullptr;
+#ifdef SF_COARSE_NOREMOTE   // timing experiment only: z-neighbours read locally (wrong results)
+    M.lo = M.hi = sm;
+#endif
+#ifdef SF_COARSE_TRACE
+    if (threadIdx.x == 0) trace_n = 0;
+    __syncthreads();
+#endif
+    TRACE();
     pdl_wait();
+    TRACE();
     const int nl = A.nlev;
-    // ---- staging: faces of every smoothed level, Dinv / alpha below the
-    // entry, the entry's U (shared) and its F / Dinv / alpha (registers)
-    for (int l = 0; l + 1 < nl; l++) {
-        const CLevel& L = A.lv[l];
-        const PV& v = L.v;
-        const int nx = v.nx, ny = v.ny, nz = v.nz;
-        // beta_i: faces 0..nx-1 of every row, then face nx
-        stage_box(sm + L.bi, v.f[SF_BETA_I], L.lx, L.ly, nz, 0, 0, nx + 1, ny, v.js, v.ks);
-        stage_box(sm + L.bi, v.f[SF_BETA_I], 0, L.ly, nz, nx, 0, nx + 1, ny, v.js, v.ks);
-        // beta_j: rows 0..ny-1 of every plane, then row ny
-        stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, L.ly, nz, 0, 0, nx, ny + 1, v.js, v.ks);
-        stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, 0, nz, 0, ny, nx, ny + 1, v.js, v.ks);
-        // beta_k: planes 0..nz
-        stage_box(sm + L.bk, v.f[SF_BETA_K], L.lx, L.ly, nz + 1, 0, 0, nx, ny, v.js, v.ks);
-        if (l > 0) {
-            stage_cells(sm + L.d, v.f[SF_DINV], L);
-            stage_cells(sm + L.al, v.f[SF_ALPHA], L);
-        }
-    }
-    const CLevel& E = A.lv[0];
-    stage_cells(sm + E.u, E.v.f[SF_U], E);
-    asm volatile("cp.async.commit_group;" ::: "memory");
+    const int k0 = 2 * M.rank;
+    // ---- the entry block of this thread into registers (and its x into shared)
+    const KLevel& E = A.lv[0];
     Block B;
     {
         const int t = threadIdx.x;
-        const int lhx = E.lx - 1, lhy = E.ly - 1, lhz = E.lz - 1;
-        B.own = t < (1 << (lhx + lhy + lhz));
+        const int lhx = E.lx - 1;
+        B.own = t < (1 << (lhx + E.ly - 1));
         B.i0 = 2 * (t & ((1 << lhx) - 1));
-        B.j0 = 2 * ((t >> lhx) & ((1 << lhy) - 1));
-        B.k0 = 2 * (t >> (lhx + lhy));
+        B.j0 = 2 * (t >> lhx);
+        const PV& v = E.v;
+        const long q0 = sf_ix(v, B.i0, B.j0, k0);
+        // 16-byte loads of x-adjacent pairs (i0 even, rows 32-byte aligned):
+        // a warp reads whole contiguous row segments
+        auto ld2 = [&](int f, long q) {
+            return B.own ? __ldg((const double2*)(v.f[f] + q)) : make_double2(0.0, 0.0);
+        };
+        auto ld1 = [&](int f, long q) { return B.own ? __ldg(v.f[f] + q) : 0.0; };
 #pragma unroll
-        for (int s = 0; s < 8; s++) {
-            B.F[s] = B.D[s] = B.A[s] = 0.0;
-            if (B.own) {
-                const long q = sf_ix(E.v, B.i0 + (s & 1), B.j0 + ((s >> 1) & 1), B.k0 + (s >> 2));
-                B.F[s] = __ldg(E.v.f[SF_F] + q);
-                B.D[s] = __ldg(E.v.f[SF_DINV] + q);
-                B.A[s] = __ldg(E.v.f[SF_ALPHA] + q);
+        for (int r = 0; r < 4; r++) {   // rows (dj, dk) = (r & 1, r >> 1): sub-cells 2r, 2r+1
+            const long q = q0 + (r & 1) * v.js + (r >> 1) * v.ks;
+            double2 t2 = ld2(SF_U, q);
+            B.X[2 * r] = t2.x; B.X[2 * r + 1] = t2.y;
+            t2 = ld2(SF_F, q);
+            B.F[2 * r] = t2.x; B.F[2 * r + 1] = t2.y;
+            t2 = ld2(SF_DINV, q);
+            B.D[2 * r] = t2.x; B.D[2 * r + 1] = t2.y;
+            t2 = ld2(SF_ALPHA, q);
+            B.A[2 * r] = t2.x; B.A[2 * r + 1] = t2.y;
+            // beta_i faces i0, i0+1 (pair) and i0+2 at (dj, dk) = (r & 1, r >> 1)
+            t2 = ld2(SF_BETA_I, q);
+            B.BI[0][r & 1][r >> 1] = t2.x; B.BI[1][r & 1][r >> 1] = t2.y;
+            B.BI[2][r & 1][r >> 1] = ld1(SF_BETA_I, q + 2);
+        }
+#pragma unroll
+        for (int f = 0; f < 3; f++)
+#pragma unroll
+            for (int r = 0; r < 2; r++) {
+                // beta_j face j0+f at dk = r, beta_k face k0+f at dj = r: di = 0, 1 as a pair
+                double2 t2 = ld2(SF_BETA_J, q0 + f * v.js + r * v.ks);
+                B.BJ[f][0][r] = t2.x; B.BJ[f][1][r] = t2.y;
+                t2 = ld2(SF_BETA_K, q0 + r * v.js + f * v.ks);
+                B.BK[f][0][r] = t2.x; B.BK[f][1][r] = t2.y;
             }
+        if (B.own) {
+            double* U = sm + E.u;
+#pragma unroll
+            for (int s = 0; s < 8; s++)
+                U[B.i0 + (s & 1) + ((B.j0 + ((s >> 1) & 1) + ((s >> 2) << E.ly)) << E.lx)] = B.X[s];
         }
     }
-    asm volatile("cp.async.wait_all;" ::: "memory");
-    __syncthreads();
-    // ---- V(l0) down to the bottom and back
-    smooth(E, sm, &B, A.a, A.pre);
-    residual_restrict_entry(E, A.lv[1], sm, B, A.a);
+    // ---- staging (async): D / alpha / faces of the CTA's planes of every
+    // level below the entry, the bottom inverse on CTA 0
     for (int l = 1; l + 1 < nl; l++) {
-        smooth(A.lv[l], sm, nullptr, A.a, A.pre);
-        residual_restrict_cells(A.lv[l], A.lv[l + 1], sm, A.a);
+        const KLevel& L = A.lv[l];
+        const PV& v = L.v;
+        const int nx = v.nx, ny = v.ny;
+        if (L.g) {   // every plane, on CTA 0
+            if (M.rank != 0) continue;
+            const int nz = v.nz;
+            stage_box(sm + L.d, v.f[SF_DINV], L.lx, L.ly, nz, 0, 0, 0, nx, ny, v.js, v.ks);
+            stage_box(sm + L.al, v.f[SF_ALPHA], L.lx, L.ly, nz, 0, 0, 0, nx, ny, v.js, v.ks);
+            stage_box(sm + L.bi, v.f[SF_BETA_I], L.lx, L.ly, nz, 0, 0, 0, nx + 1, ny, v.js, v.ks);
+            stage_box(sm + L.bi, v.f[SF_BETA_I], 0, L.ly, nz, nx, 0, 0, nx + 1, ny, v.js, v.ks);
+            stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, L.ly, nz, 0, 0, 0, nx, ny + 1, v.js, v.ks);
+            stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, 0, nz, 0, ny, 0, nx, ny + 1, v.js, v.ks);
+            stage_box(sm + L.bk, v.f[SF_BETA_K], L.lx, L.ly, nz + 1, 0, 0, 0, nx, ny, v.js, v.ks);
+            continue;
+        }
+        if (M.rank >= (1 << (L.lz - 1))) continue;
+        stage_box(sm + L.d, v.f[SF_DINV], L.lx, L.ly, 2, 0, 0, k0, nx, ny, v.js, v.ks);
+        stage_box(sm + L.al, v.f[SF_ALPHA], L.lx, L.ly, 2, 0, 0, k0, nx, ny, v.js, v.ks);
+        stage_box(sm + L.bi, v.f[SF_BETA_I], L.lx, L.ly, 2, 0, 0, k0, nx + 1, ny, v.js, v.ks);
+        stage_box(sm + L.bi, v.f[SF_BETA_I], 0, L.ly, 2, nx, 0, k0, nx + 1, ny, v.js, v.ks);
+        stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, L.ly, 2, 0, 0, k0, nx, ny + 1, v.js, v.ks);
+        stage_box(sm + L.bj, v.f[SF_BETA_J], L.lx, 0, 2, 0, ny, k0, nx, ny + 1, v.js, v.ks);
+        stage_box(sm + L.bk, v.f[SF_BETA_K], L.lx, L.ly, 3, 0, 0, k0, nx, ny, v.js, v.ks);
     }
-    bottom(A.lv[nl - 1], sm, A.ainv);
-    for (int l = nl - 2; l >= 1; l--) {
-        interp_cells(A.lv[l], A.lv[l + 1], sm);
-        smooth(A.lv[l], sm, nullptr, A.a, A.post);
+    if (M.rank == 0) {
+        const KLevel& Bt = A.lv[nl - 1];
+        const int n = 1 << (Bt.lx + Bt.ly + Bt.lz);
+        const unsigned d0 = (unsigned)__cvta_generic_to_shared(sm + A.ainv);
+        for (int e = threadIdx.x; e < n * n; e += NT)
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d0 + 8u * e), "l"(A.ainv_g + e)
+                         : "memory");
     }
-    interp_entry(E, A.lv[1], sm, B);
-    smooth(E, sm, &B, A.a, A.post);
-    // ---- the entry level's U back to global memory
-    const PV& v = E.v;
-    const int n = v.nx * v.ny * v.nz;
-    for (int t = threadIdx.x; t < n; t += CNT) {
-        const int i = t & (v.nx - 1), r = t >> E.lx;
-        v.f[SF_U][sf_ix(v, i, r & (v.ny - 1), r >> E.ly)] = sm[E.u + t];
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    cluster_sync();
+    // ---- V(l0) down to the bottom and back
+    smooth(E, M, &B, A.a, A.pre);
+    asm volatile("cp.async.wait_all;" ::: "memory");   // staged levels visible after the next barrier
+    residual_restrict(cl, E, A.lv[1], M, &B, A.a, A.lv[1].g, A.rscr);
+    int lg = 1;   // first gathered level
+    for (; !A.lv[lg].g; lg++) {
+        smooth(A.lv[lg], M, nullptr, A.a, A.pre);
+        residual_restrict(cl, A.lv[lg], A.lv[lg + 1], M, nullptr, A.a, A.lv[lg + 1].g, A.rscr);
     }
+    if (M.rank == 0) gathered_cycle(A, sm, lg);
+    TRACE();
+    cluster_sync();
+    for (int l = lg - 1; l >= 1; l--) {
+        interp(cl, A.lv[l], A.lv[l + 1], M, nullptr, A.lv[l + 1].g);
+        smooth(A.lv[l], M, nullptr, A.a, A.post);
+    }
+    interp(cl, E, A.lv[1], M, &B, A.lv[1].g);
+    smooth(E, M, &B, A.a, A.post);
+    // ---- the entry block's x back to global memory
+    if (B.own) {
+        const PV& v = E.v;
+        const long q0 = sf_ix(v, B.i0, B.j0, k0);
+#pragma unroll
+        for (int s = 0; s < 8; s++)
+            v.f[SF_U][q0 + (s & 1) + ((s >> 1) & 1) * v.js + (s >> 2) * v.ks] = B.X[s];
+    }
+#ifdef SF_COARSE_TRACE
+    TRACE();
+    if (threadIdx.x == 0 && M.rank <= 1) {
+        for (int i = 1; i < trace_n; i++)
+            printf("trace rank %d phase %d: %lld\n", M.rank, i, trace_t[i] - trace_t[i - 1]);
+    }
+#endif
 }
 
-// shared-memory plan of a V(lv[0]) over n levels: offsets into lv[], total doubles
-long plan_smem(sf_level* const* lv, int n, CLevel* out) {
+// shared-memory plan (doubles per CTA): offsets into out[], total returned
+long plan_smem(sf_level* const* lv, int n, KLevel* out, int* ainv, int* rscr) {
     long off = 0;
+    if (rscr) *rscr = 0;   // residual scratch: two planes of a distributed level / a gathered level
+    off += GMAX;
     for (int l = 0; l < n; l++) {
-        const long nx = lv[l]->nx, ny = lv[l]->ny, nz = lv[l]->lnz, c = nx * ny * nz;
-        CLevel L = {};
-        L.u = (int)off;
-        off += c;
-        L.f = L.d = L.al = L.bi = L.bj = L.bk = -1;
-        if (l > 0) {
-            L.f = (int)off;
-            off += c;
-        }
-        if (l > 0 && l + 1 < n) {
-            L.d = (int)off;
-            off += c;
-            L.al = (int)off;
-            off += c;
-        }
-        if (l + 1 < n) {
-            L.bi = (int)off;
-            off += (nx + 1) * ny * nz;
-            L.bj = (int)off;
-            off += nx * (ny + 1) * nz;
-            L.bk = (int)off;
-            off += nx * ny * (nz + 1);
+        const long nx = lv[l]->nx, ny = lv[l]->ny, pl = nx * ny;
+        KLevel L = {};
+        L.u = L.f = L.d = L.al = L.bi = L.bj = L.bk = -1;
+        const long c = pl * lv[l]->lnz;
+        L.g = l > 0 && c <= GMAX;
+        if (l == 0) {
+            L.u = (int)off;
+            off += 2 * pl;
+        } else if (l + 1 < n && L.g) {   // every plane, on CTA 0
+            L.u = (int)off;  off += c;
+            L.f = (int)off;  off += c;
+            L.d = (int)off;  off += c;
+            L.al = (int)off; off += c;
+            L.bi = (int)off; off += (nx + 1) * ny * lv[l]->lnz;
+            L.bj = (int)off; off += nx * (ny + 1) * lv[l]->lnz;
+            L.bk = (int)off; off += pl * (lv[l]->lnz + 1);
+        } else if (l + 1 < n) {
+            L.u = (int)off;  off += 2 * pl;
+            L.f = (int)off;  off += 2 * pl;
+            L.d = (int)off;  off += 2 * pl;
+            L.al = (int)off; off += 2 * pl;
+            L.bi = (int)off; off += 2 * ny * (nx + 1);
+            L.bj = (int)off; off += 2 * (ny + 1) * nx;
+            L.bk = (int)off; off += 3 * pl;
+        } else {   // bottom: every plane (CTA 0)
+            L.g = 1;
+            L.u = (int)off; off += c;
+            L.f = (int)off; off += c;
+            if (ainv) *ainv = (int)off;
+            off += c * c;
         }
         if (out) out[l] = L;
     }
     return off;
+}
+
+// largest cluster the kernel may use: 16 CTAs if a 16-CTA cluster of it is
+// schedulable (non-portable size), else 8; SF_COARSE_MAX_CS caps it (A/B)
+int max_cluster() {
+    static int m = 0;
+    if (!m) {
+        m = 8;
+        if (cudaFuncSetAttribute(coarse_vcycle_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) ==
+                cudaSuccess &&
+            cudaFuncSetAttribute(coarse_vcycle_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 CSMEM_MAX) == cudaSuccess) {
+            cudaLaunchConfig_t c = {};
+            c.gridDim = dim3(CS_MAX);
+            c.blockDim = dim3(NT);
+            c.dynamicSmemBytes = 96 * 1024;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = CS_MAX;
+            at[0].val.clusterDim.y = 1;
+            at[0].val.clusterDim.z = 1;
+            c.attrs = at;
+            c.numAttrs = 1;
+            int nc = 0;
+            if (cudaOccupancyMaxActiveClusters(&nc, coarse_vcycle_kernel, &c) == cudaSuccess && nc >= 1)
+                m = CS_MAX;
+        }
+        cudaGetLastError();
+        if (const char* e = getenv("SF_COARSE_MAX_CS")) m = std::max(1, std::min(m, atoi(e)));
+    }
+    return m;
 }
 
 }  // namespace
@@ -351,36 +653,30 @@ long plan_smem(sf_level* const* lv, int n, CLevel* out) {
 int coarse_vcycle_max_levels() { return CMAXL; }
 
 // a V-cycle from lv[0] over n levels fits the kernel: single-part power-of-two
-// levels, the entry at most 4096 cells, every operand within shared memory
+// levels halving into each other, entry nz/2 <= the cluster limit and at most
+// NT blocks per layer, the bottom within BOT_MAX cells, shared memory within 227 KB
 bool coarse_vcycle_fits(sf_level* const* lv, int n) {
     if (n < 2 || n > CMAXL) return false;
     auto pow2 = [](int v) { return v >= 1 && (v & (v - 1)) == 0; };
     for (int l = 0; l < n; l++) {
         if (lv[l]->nparts != 1 || lv[l]->nlocal != 1) return false;
         if (!pow2(lv[l]->nx) || !pow2(lv[l]->ny) || !pow2(lv[l]->lnz)) return false;
-        // every smoothed level halves into the next in all three directions
         if (l + 1 < n && (lv[l]->nx < 2 || lv[l]->ny < 2 || lv[l]->lnz < 2 ||
                           lv[l + 1]->nx * 2 != lv[l]->nx || lv[l + 1]->ny * 2 != lv[l]->ny ||
                           lv[l + 1]->lnz * 2 != lv[l]->lnz))
             return false;
     }
     const long bot = (long)lv[n - 1]->nx * lv[n - 1]->ny * lv[n - 1]->lnz;
-    return (long)lv[0]->nx * lv[0]->ny * lv[0]->lnz <= CMAX_CELLS && bot <= CNT &&
-           plan_smem(lv, n, nullptr) * (long)sizeof(double) <= CSMEM_MAX;
+    return lv[0]->lnz / 2 <= max_cluster() && (long)lv[0]->nx * lv[0]->ny / 4 <= NT &&
+           bot <= BOT_MAX && plan_smem(lv, n, nullptr, nullptr, nullptr) * (long)sizeof(double) <= CSMEM_MAX;
 }
 
-// V(lv[0]) down to the bottom lv[n-1] and back, one single-CTA launch
+// V(lv[0]) down to the bottom lv[n-1] and back: one launch of one cluster
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
                           int pre, int post) {
     if (!coarse_vcycle_fits(lv, n)) return sf_fail(SF_ERR_SHAPE, "coarse V-cycle levels do not fit");
-    static bool attr = false;
-    if (!attr) {
-        SF_CUDA(cudaFuncSetAttribute(coarse_vcycle_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     CSMEM_MAX));
-        attr = true;
-    }
-    CoarseArgs A = {};
-    const long doubles = plan_smem(lv, n, A.lv);
+    KArgs A = {};
+    const long doubles = plan_smem(lv, n, A.lv, &A.ainv, &A.rscr);
     for (int l = 0; l < n; l++) {
         A.lv[l].v = sf_view(lv[l], 0);
         A.lv[l].bh2 = b / (lv[l]->h * lv[l]->h);
@@ -392,8 +688,28 @@ sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const 
     A.pre = pre;
     A.post = post;
     A.a = a;
-    A.ainv = ainv;
-    SF_CUDA(sf_launch(coarse_vcycle_kernel, 1, CNT, (size_t)doubles * sizeof(double), lv[0]->stream, A));
+    A.ainv_g = ainv;
+    const int C = lv[0]->lnz / 2;
+#ifdef SF_COARSE_TRACE
+    for (int l = 0; l < n; l++)
+        printf("plan l=%d %dx%dx%d g=%d u=%d f=%d d=%d bi=%d total=%ld C=%d\n", l, lv[l]->nx, lv[l]->ny,
+               lv[l]->lnz, A.lv[l].g, A.lv[l].u, A.lv[l].f, A.lv[l].d, A.lv[l].bi, doubles, C);
+#endif
+    cudaLaunchConfig_t c = {};
+    c.gridDim = dim3(C);
+    c.blockDim = dim3(NT);
+    c.dynamicSmemBytes = (size_t)doubles * sizeof(double);
+    c.stream = lv[0]->stream;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = C;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = 1;
+    c.attrs = at;
+    c.numAttrs = sf_pdl_on() ? 2 : 1;
+    SF_CUDA(cudaLaunchKernelEx(&c, coarse_vcycle_kernel, A));
     SF_LAUNCHED();
     return sf_check_launch("coarse_vcycle");
 }
