@@ -63,6 +63,7 @@ struct KArgs {
     double a;
     int ainv;             // shared offset of the bottom inverse (CTA 0)
     int rscr;             // shared offset of the residual scratch (GMAX doubles)
+    int uzero;            // the entry level's U is zero (V-cycle): not read
     const double* ainv_g; // n x n, row major
 };
 
@@ -473,7 +474,7 @@ __global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_const
 #pragma unroll
         for (int r = 0; r < 4; r++) {   // rows (dj, dk) = (r & 1, r >> 1): sub-cells 2r, 2r+1
             const long q = q0 + (r & 1) * v.js + (r >> 1) * v.ks;
-            double2 t2 = ld2(SF_U, q);
+            double2 t2 = A.uzero ? make_double2(0.0, 0.0) : ld2(SF_U, q);
             B.X[2 * r] = t2.x; B.X[2 * r + 1] = t2.y;
             t2 = ld2(SF_F, q);
             B.F[2 * r] = t2.x; B.F[2 * r + 1] = t2.y;
@@ -673,7 +674,7 @@ bool coarse_vcycle_fits(sf_level* const* lv, int n) {
 
 // V(lv[0]) down to the bottom lv[n-1] and back: one launch of one cluster
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
-                          int pre, int post) {
+                          int pre, int post, bool u_zero) {
     if (!coarse_vcycle_fits(lv, n)) return sf_fail(SF_ERR_SHAPE, "coarse V-cycle levels do not fit");
     KArgs A = {};
     const long doubles = plan_smem(lv, n, A.lv, &A.ainv, &A.rscr);
@@ -689,6 +690,7 @@ sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const 
     A.post = post;
     A.a = a;
     A.ainv_g = ainv;
+    A.uzero = u_zero ? 1 : 0;
     const int C = lv[0]->lnz / 2;
 #ifdef SF_COARSE_TRACE
     for (int l = 0; l < n; l++)

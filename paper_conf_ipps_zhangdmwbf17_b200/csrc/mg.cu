@@ -338,14 +338,16 @@ static sf_status bres_pair(sf_mg* m, sf_level* L) {
 
 // V(l): smooth, residual, restrict, zero e_{l+1}, V(l+1), e_l += P0 e_{l+1}, smooth.
 // skip_first: the first pre-smoothing pair was already run (fused check, below).
-static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
+// u_zero: U of level l is zero on entry (the V-cycle recursion zeroed it, or
+// leaves that to the coarse-level launch, which then does not read it)
+static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = false) {
     const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
     NvtxRange nv("sf V(l=%d) %dx%dx%d", l, L->gnx, L->gny, L->gnz);
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one launch
         return k_coarse_vcycle(&m->lv[l], (int)m->lv.size() - l, m->a, m->b, m->ainv,
-                               m->o.pre_pairs, m->o.post_pairs);
+                               m->o.pre_pairs, m->o.post_pairs, u_zero);
     sf_level* C = m->lv[l + 1];
     const int pre = m->o.pre_pairs - (skip_first ? 1 : 0);
     if (pre >= 1 && (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
@@ -364,8 +366,9 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false) {
             SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));
         }
     }
-    SF_TRY(k_zero(C, SF_U));
-    SF_TRY(vcyc(m, l + 1));
+    const bool cz = m->coarse_l0 >= 1 && l + 1 >= m->coarse_l0 && l + 1 < (int)m->lv.size() - 1;
+    if (!cz) SF_TRY(k_zero(C, SF_U));   // the coarse-level launch starts from zero itself
+    SF_TRY(vcyc(m, l + 1, false, cz));
     if (m->o.vcycle_interp == SF_INTERP_P0 && m->o.post_pairs >= 1 &&
         (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
         gsrb_fused_supported(L)) {

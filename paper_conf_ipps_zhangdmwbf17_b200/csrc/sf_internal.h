@@ -215,11 +215,13 @@ bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
                          int cf);
 
-// coarse-level V-cycle in one single-CTA launch, iterates in shared memory (coarse.cu)
+// coarse-level V-cycle in one thread-block-cluster launch, iterates in registers and
+// shared memory (coarse.cu)
 bool coarse_vcycle_fits(sf_level* const* lv, int n);
 int coarse_vcycle_max_levels();
+// u_zero: lv[0]'s U is zero on entry (V-cycle recursion): not read, not zeroed first
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
-                          int pre, int post);
+                          int pre, int post, bool u_zero);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.

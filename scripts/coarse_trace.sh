@@ -1,7 +1,6 @@
-# per-phase clock trace of the coarse V-cycle kernel (dbg builds: trace, trace without DSMEM)
-for v in trace noremote; do
-SF_LIB=dbg/libsf_$v.so python scripts/vcycle_once_n.py 64 > gpurun_out/trace64_$v.txt 2>&1
-echo $v
-grep "rank 0" gpurun_out/trace64_$v.txt | awk '{print $6}' | tail -52 | tr '\n' ' '; echo
-grep "rank 1" gpurun_out/trace64_$v.txt | awk '{print $6}' | tail -30 | tr '\n' ' '; echo
-done
+# coarse V-cycle kernel: parity, solve timings, warm launch list
+timeout 900 python -m pytest tests/test_gpu_coarse.py tests/test_gpu_parity.py -x -q 2>&1 | tail -2
+python scripts/small_pair_ab.py default
+SF_COARSE_MAX_CS=8 python scripts/small_pair_ab.py cs8
+timeout 300 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none --cache-control none --csv --log-file gpurun_out/vc_warm_64.csv python scripts/vcycle_once_n.py 64 > /dev/null 2>&1
+python scripts/launch_list.py gpurun_out/vc_warm_64.csv
