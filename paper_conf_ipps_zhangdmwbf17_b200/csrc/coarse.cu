@@ -5,31 +5,38 @@
 // residual + restriction, P0 interpolation and the bottom solve of V(l)
 // (A5-A9) is a few microseconds of work
 // behind a launch of its own -- ~40 launches per V-cycle below 64^3.  Here one
-// cluster of C = nz/2 CTAs (entry level nz <= 32: up to 16 CTAs, one per SM)
-// runs the whole V(l0) .. bottom .. V(l0) recursion with every operand in
-// REGISTERS or SHARED MEMORY; phases are separated by cluster barriers and the
-// z-neighbours that live in the next CTA are read through distributed shared
-// memory (DSMEM).  After one staging pass no phase touches global memory.
+// cluster of C = nz/2 CTAs (entry level nz <= 32: up to 16 CTAs, one per SM,
+// the non-portable cluster size where the device schedules it) runs the whole
+// V(l0) .. bottom .. V(l0) recursion with every operand in REGISTERS or SHARED
+// MEMORY; phases are separated by cluster barriers and the z-neighbours that
+// live in the next CTA are read through distributed shared memory (DSMEM).
+// After one staging pass no phase touches global memory.
 //
-// Ownership: on every smoothed level CTA c owns the 2-plane layer of 2x2x2
+// Ownership: on every distributed level CTA c owns the 2-plane layer of 2x2x2
 // blocks whose parents form coarse plane c (planes 2c, 2c+1), so the
 // restriction of a block and the P0 correction of its cells involve only the
-// block's CTA and the owner of the parent plane (CTA c/2 on the next smoothed
-// level, CTA 0 for the bottom, which holds the whole coarsest level).
+// block's CTA and the owner of the parent plane (CTA c/2 on the next
+// distributed level).  The coarsest levels (<= 512 cells, and the bottom) are
+// GATHERED whole on CTA 0, which runs their part of the cycle alone with
+// __syncthreads (a cluster barrier per phase would cost more than their work).
 //
 // Entry level: thread t of CTA c owns block t of the layer and keeps its
 // 8 x values, F, Dinv, alpha and the 36 face coefficients of the block in
 // registers; its x values are mirrored in shared memory for the neighbours'
-// reads.  Levels below: one thread per cell of a colour, U / F / Dinv / alpha
-// and the faces of the CTA's two planes in shared memory.
+// reads.  Levels below: one thread per cell, U / F / Dinv / alpha and the
+// faces in shared memory.
 //
-// Arithmetic: op7 is op_at's expression (cell_ops.cuh: same terms, order and
-// Dirichlet fold); the colour sweep is gsrb_colour_kernel's update
-// x += Dinv (rhs - A x); the residual + restriction sums rhs - A x over the 8
-// children in restrict_cell's order and divides by 8; P0 adds the parent; the
-// bottom applies the exact inverse in bottom_solve_kernel's order -- so the
-// launch reproduces the per-phase kernels bit for bit.
+// Arithmetic: the colour sweep is the fused pairs' lambda-form update
+// x = Dinv (F + b h^-2 S) (sum6 / gs_upd of tma_common.cuh),
+// a restatement of x += Dinv (F - A x) equal up to rounding; the residual of
+// the restriction is op_at's expression (cell_ops.cuh: same terms, order and
+// Dirichlet fold), summed over the 8 children in restrict_cell's order and
+// divided by 8; P0 adds the parent; the bottom applies the exact inverse in
+// bottom_solve_kernel's order.  The first red sweep of every level below the
+// entry rides in the restriction that produced its F (from U = 0 it is
+// x = Dinv F exactly).
 #include <cooperative_groups.h>
+#include <cuda.h>
 
 #include <algorithm>
 #include <cstdlib>
@@ -39,6 +46,8 @@
 namespace cg = cooperative_groups;
 
 namespace {
+
+#include "tma_common.cuh"   // sum6 / gs_upd: the lambda-form update of the fused pairs
 
 constexpr int CMAXL = 8;                 // levels per launch
 constexpr int NT = 256;                  // threads per CTA (entry blocks per layer at most)
@@ -124,6 +133,28 @@ struct Block {
     double BK[3][2][2];         // beta_k faces k0..k0+2 at (di, dj)
 };
 
+// GS update of sub-cell s in lambda form, x = Dinv (F + b h^-2 S) with S the
+// beta-weighted sum of the neighbours (a Dirichlet ghost contributes 0: its
+// -x(c) is part of the diagonal) -- the fused pairs' update (sum6 / gs_upd)
+__device__ __forceinline__ double upd_block(const KLevel& L, const Mem& M, const Block& B, int s) {
+    const int di = s & 1, dj = (s >> 1) & 1, dk = s >> 2;
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int i = B.i0 + di, j = B.j0 + dj, k = 2 * M.rank + dk;
+    const double* U = M.sm + L.u;
+    const int cp = i + (j << L.lx);
+    const int c = cp + (dk << (L.lx + L.ly));
+    double xw, xe, xs, xn, xb, xt;
+    if (di) { xw = B.X[s - 1]; xe = (i == nx - 1) ? 0.0 : U[c + 1]; }
+    else    { xe = B.X[s + 1]; xw = (i == 0) ? 0.0 : U[c - 1]; }
+    if (dj) { xs = B.X[s - 2]; xn = (j == ny - 1) ? 0.0 : U[c + nx]; }
+    else    { xn = B.X[s + 2]; xs = (j == 0) ? 0.0 : U[c - nx]; }
+    if (dk) { xb = B.X[s - 4]; xt = (k == nz - 1) ? 0.0 : (M.hi + L.u)[cp]; }
+    else    { xt = B.X[s + 4]; xb = (k == 0) ? 0.0 : (M.lo + L.u)[cp + (1 << (L.lx + L.ly))]; }
+    return gs_upd(B.D[s], B.F[s], L.bh2,
+                  sum6(xw, xe, xs, xn, xb, xt, B.BI[di][dj][dk], B.BI[di + 1][dj][dk], B.BJ[dj][di][dk],
+                       B.BJ[dj + 1][di][dk], B.BK[dk][di][dj], B.BK[dk + 1][di][dj]));
+}
+
 // A x at sub-cell s = di + 2 dj + 4 dk of the block, with the block's current x
 __device__ __forceinline__ double op_block(const KLevel& L, const Mem& M, const Block& B, int s,
                                            double a) {
@@ -152,15 +183,15 @@ __device__ __forceinline__ void sweep_entry(const KLevel& L, const Mem& M, Block
         // every operator value first (the colour's cells read only the other
         // colour), then the updates: the neighbour loads -- one of them from the
         // next CTA -- are all in flight together
-        double ax[8];
+        double xnew[8];
 #pragma unroll
         for (int s = 0; s < 8; s++)
-            if ((((s & 1) + ((s >> 1) & 1) + (s >> 2)) & 1) == colour) ax[s] = op_block(L, M, B, s, a);
+            if ((((s & 1) + ((s >> 1) & 1) + (s >> 2)) & 1) == colour) xnew[s] = upd_block(L, M, B, s);
 #pragma unroll
         for (int s = 0; s < 8; s++) {
             const int di = s & 1, dj = (s >> 1) & 1, dk = s >> 2;
             if (((di + dj + dk) & 1) != colour) continue;   // block origin is even
-            B.X[s] = B.X[s] + B.D[s] * (B.F[s] - ax[s]);
+            B.X[s] = xnew[s];
             U[B.i0 + di + ((B.j0 + dj + (dk << L.ly)) << L.lx)] = B.X[s];
         }
     }
@@ -190,6 +221,27 @@ __device__ __forceinline__ double op_cell(const KLevel& L, const Mem& M, int i, 
                M.sm[L.al + c], a, L.bh2);
 }
 
+// lambda-form GS update at (i, j, plane kl of this CTA) of a non-entry level
+__device__ __forceinline__ double upd_cell(const KLevel& L, const Mem& M, int i, int j, int kl) {
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int k = 2 * M.rank + kl;
+    const double* U = M.sm + L.u;
+    const int pl = 1 << (L.lx + L.ly);
+    const int cp = i + (j << L.lx), c = cp + kl * pl;
+    const double xw = (i == 0) ? 0.0 : U[c - 1];
+    const double xe = (i == nx - 1) ? 0.0 : U[c + 1];
+    const double xs = (j == 0) ? 0.0 : U[c - nx];
+    const double xn = (j == ny - 1) ? 0.0 : U[c + nx];
+    double xb, xt;
+    if (kl) { xb = U[cp]; xt = (k == nz - 1) ? 0.0 : (M.hi + L.u)[cp]; }
+    else    { xt = U[cp + pl]; xb = (k == 0) ? 0.0 : (M.lo + L.u)[cp + pl]; }
+    const double* bi = M.sm + L.bi + i + (nx + 1) * (j + (kl << L.ly));
+    const double* bj = M.sm + L.bj + i + ((j + (ny + 1) * kl) << L.lx);
+    const double* bk = M.sm + L.bk + c;
+    return gs_upd(M.sm[L.d + c], M.sm[L.f + c], L.bh2,
+                  sum6(xw, xe, xs, xn, xb, xt, bi[0], bi[1], bj[0], bj[nx], bk[0], bk[pl]));
+}
+
 // one colour sweep: thread t updates the t-th cell of the colour in the CTA's two planes
 __device__ __forceinline__ void sweep_cells(const KLevel& L, const Mem& M, double a, int colour) {
     if (M.rank < (1 << (L.lz - 1))) {
@@ -200,25 +252,34 @@ __device__ __forceinline__ void sweep_cells(const KLevel& L, const Mem& M, doubl
             const int th = t & ((1 << lh) - 1), r = t >> lh;
             const int j = r & ((1 << L.ly) - 1), kl = r >> L.ly;
             const int i = 2 * th + ((j + kl + colour) & 1);   // plane 2*rank+kl: parity of kl
-            const int c = i + ((j + (kl << L.ly)) << L.lx);
-            const double xc = U[c];
-            const double ax = op_cell(L, M, i, j, kl, xc, a);
-            U[c] = xc + M.sm[L.d + c] * (M.sm[L.f + c] - ax);
+            U[i + ((j + (kl << L.ly)) << L.lx)] = upd_cell(L, M, i, j, kl);
         }
     }
     cluster_sync();
 }
 
-__device__ __forceinline__ void smooth(const KLevel& L, const Mem& M, Block* B, double a, int pairs) {
+// skip_red: the first red sweep was folded into the restriction that produced
+// this level's F (from U = 0 it is x = Dinv F exactly, see residual_restrict)
+__device__ __forceinline__ void smooth(const KLevel& L, const Mem& M, Block* B, double a, int pairs,
+                                       bool skip_red = false) {
     for (int p = 0; p < pairs; p++) {
         if (B) {
             sweep_entry(L, M, *B, a, 0);
             sweep_entry(L, M, *B, a, 1);
         } else {
-            sweep_cells(L, M, a, 0);
+            if (p > 0 || !skip_red) sweep_cells(L, M, a, 0);
             sweep_cells(L, M, a, 1);
         }
     }
+}
+
+// U of a coarse cell after the restriction: 0, or with `fold` the first red
+// sweep of its pre-smoothing from U = 0: a red cell's neighbours are all 0, so
+// the lambda-form update is gs_upd(Dinv, F, b h^-2, 0) = Dinv F exactly and a
+// black cell stays 0 -- one phase less per level
+__device__ __forceinline__ double u_after_restrict(bool fold, bool red, double dinv, double f,
+                                                   double bh2) {
+    return (fold && red) ? gs_upd(dinv, f, bh2, 0.0) : 0.0;
 }
 
 // coarse cell (I, J) of plane `rank` of level C: its slot in the owner's shared memory
@@ -231,7 +292,7 @@ __device__ __forceinline__ int coarse_slot(const KLevel& C, const Mem& M, int I,
 // `rank`), C.U = 0; written into the owner of that coarse plane
 __device__ __forceinline__ void residual_restrict(cg::cluster_group& cl, const KLevel& F,
                                                   const KLevel& C, const Mem& M, const Block* B,
-                                                  double a, bool cgat, int rscr) {
+                                                  double a, bool cgat, int rscr, bool fold) {
     if (M.rank < (1 << (F.lz - 1))) {
         double* dst = M.owner(cl, M.rank, cgat);
         if (B) {
@@ -243,8 +304,10 @@ __device__ __forceinline__ void residual_restrict(cg::cluster_group& cl, const K
 #pragma unroll
                 for (int s = 0; s < 8; s++) acc += r[s];
                 const int q = coarse_slot(C, M, B->i0 >> 1, B->j0 >> 1, cgat);
-                dst[C.f + q] = acc / 8.0;
-                dst[C.u + q] = 0.0;
+                const double fc = acc / 8.0;
+                const bool red = (((B->i0 + B->j0) >> 1) + M.rank & 1) == 0;
+                dst[C.f + q] = fc;
+                dst[C.u + q] = u_after_restrict(fold, red, fold ? dst[C.d + q] : 0.0, fc, C.bh2);
             }
         } else {
             // residual of every cell of the two planes (one thread per cell),
@@ -265,8 +328,10 @@ __device__ __forceinline__ void residual_restrict(cg::cluster_group& cl, const K
                 for (int s = 0; s < 8; s++)
                     acc += R[2 * I + (s & 1) + ((2 * J + ((s >> 1) & 1) + ((s >> 2) << F.ly)) << F.lx)];
                 const int q = coarse_slot(C, M, I, J, cgat);
-                dst[C.f + q] = acc / 8.0;
-                dst[C.u + q] = 0.0;
+                const double fc = acc / 8.0;
+                dst[C.f + q] = fc;
+                dst[C.u + q] = u_after_restrict(fold, ((I + J + M.rank) & 1) == 0,
+                                                fold ? dst[C.d + q] : 0.0, fc, C.bh2);
             }
         }
     }
@@ -326,6 +391,25 @@ __device__ __forceinline__ double op_g(const KLevel& L, const double* sm, int i,
                sm[L.al + c], a, L.bh2);
 }
 
+// lambda-form GS update at (i, j, k) of a gathered level
+__device__ __forceinline__ double upd_g(const KLevel& L, const double* sm, int i, int j, int k) {
+    const int nx = 1 << L.lx, ny = 1 << L.ly, nz = 1 << L.lz;
+    const int pl = 1 << (L.lx + L.ly);
+    const int c = i + ((j + (k << L.ly)) << L.lx);
+    const double* U = sm + L.u;
+    const double xw = (i == 0) ? 0.0 : U[c - 1];
+    const double xe = (i == nx - 1) ? 0.0 : U[c + 1];
+    const double xs = (j == 0) ? 0.0 : U[c - nx];
+    const double xn = (j == ny - 1) ? 0.0 : U[c + nx];
+    const double xb = (k == 0) ? 0.0 : U[c - pl];
+    const double xt = (k == nz - 1) ? 0.0 : U[c + pl];
+    const double* bi = sm + L.bi + i + (nx + 1) * (j + (k << L.ly));
+    const double* bj = sm + L.bj + i + ((j + (ny + 1) * k) << L.lx);
+    const double* bk = sm + L.bk + c;
+    return gs_upd(sm[L.d + c], sm[L.f + c], L.bh2,
+                  sum6(xw, xe, xs, xn, xb, xt, bi[0], bi[1], bj[0], bj[nx], bk[0], bk[pl]));
+}
+
 __device__ __forceinline__ void sweep_g(const KLevel& L, double* sm, double a, int colour) {
     const int lh = L.lx - 1;
     const int n = 1 << (lh + L.ly + L.lz);   // cells of one colour
@@ -334,10 +418,7 @@ __device__ __forceinline__ void sweep_g(const KLevel& L, double* sm, double a, i
         const int th = t & ((1 << lh) - 1), r = t >> lh;
         const int j = r & ((1 << L.ly) - 1), k = r >> L.ly;
         const int i = 2 * th + ((j + k + colour) & 1);
-        const int c = i + ((j + (k << L.ly)) << L.lx);
-        const double xc = U[c];
-        const double ax = op_g(L, sm, i, j, k, xc, a);
-        U[c] = xc + sm[L.d + c] * (sm[L.f + c] - ax);
+        U[i + ((j + (k << L.ly)) << L.lx)] = upd_g(L, sm, i, j, k);
     }
     __syncthreads();
     TRACE();
@@ -346,7 +427,7 @@ __device__ __forceinline__ void sweep_g(const KLevel& L, double* sm, double a, i
 // C.F = R_cell(F - A U), C.U = 0: one thread per coarse cell
 // (residual of every fine cell into the scratch R first, one thread per cell)
 __device__ __forceinline__ void restrict_g(const KLevel& F, const KLevel& C, double* sm, double a,
-                                           double* R) {
+                                           double* R, bool fold) {
     const int nf = 1 << (F.lx + F.ly + F.lz);
     for (int t = threadIdx.x; t < nf; t += NT) {
         const int i = t & ((1 << F.lx) - 1), r = t >> F.lx;
@@ -362,8 +443,9 @@ __device__ __forceinline__ void restrict_g(const KLevel& F, const KLevel& C, dou
 #pragma unroll
         for (int s = 0; s < 8; s++)
             acc += R[2 * I + (s & 1) + ((2 * J + ((s >> 1) & 1) + ((2 * K + (s >> 2)) << F.ly)) << F.lx)];
-        sm[C.f + t] = acc / 8.0;
-        sm[C.u + t] = 0.0;
+        const double fc = acc / 8.0;
+        sm[C.f + t] = fc;
+        sm[C.u + t] = u_after_restrict(fold, ((I + J + K) & 1) == 0, fold ? sm[C.d + t] : 0.0, fc, C.bh2);
     }
     __syncthreads();
     TRACE();
@@ -398,12 +480,13 @@ __device__ __forceinline__ void bottom_g(const KLevel& Bt, double* sm, int ainv)
 // V(l0) .. bottom .. V(l0) over the gathered levels l0..nl-1 (CTA 0 only)
 __device__ __forceinline__ void gathered_cycle(const KArgs& A, double* sm, int l0) {
     const int nl = A.nlev;
+    const bool fold = A.pre >= 1;   // every level's first red sweep came with its F
     for (int l = l0; l + 1 < nl; l++) {
         for (int p = 0; p < A.pre; p++) {
-            sweep_g(A.lv[l], sm, A.a, 0);
+            if (p > 0 || !fold) sweep_g(A.lv[l], sm, A.a, 0);
             sweep_g(A.lv[l], sm, A.a, 1);
         }
-        restrict_g(A.lv[l], A.lv[l + 1], sm, A.a, sm + A.rscr);
+        restrict_g(A.lv[l], A.lv[l + 1], sm, A.a, sm + A.rscr, fold && l + 2 < nl);
     }
     bottom_g(A.lv[nl - 1], sm, A.ainv);
     for (int l = nl - 2; l >= l0; l--) {
@@ -544,11 +627,13 @@ __global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_const
     // ---- V(l0) down to the bottom and back
     smooth(E, M, &B, A.a, A.pre);
     asm volatile("cp.async.wait_all;" ::: "memory");   // staged levels visible after the next barrier
-    residual_restrict(cl, E, A.lv[1], M, &B, A.a, A.lv[1].g, A.rscr);
+    const bool fold = A.pre >= 1;   // first red sweep of each coarser level folded into its restriction
+    residual_restrict(cl, E, A.lv[1], M, &B, A.a, A.lv[1].g, A.rscr, fold && nl > 2);
     int lg = 1;   // first gathered level
     for (; !A.lv[lg].g; lg++) {
-        smooth(A.lv[lg], M, nullptr, A.a, A.pre);
-        residual_restrict(cl, A.lv[lg], A.lv[lg + 1], M, nullptr, A.a, A.lv[lg + 1].g, A.rscr);
+        smooth(A.lv[lg], M, nullptr, A.a, A.pre, fold);
+        residual_restrict(cl, A.lv[lg], A.lv[lg + 1], M, nullptr, A.a, A.lv[lg + 1].g, A.rscr,
+                          fold && lg + 2 < nl);
     }
     if (M.rank == 0) gathered_cycle(A, sm, lg);
     TRACE();
@@ -619,11 +704,11 @@ long plan_smem(sf_level* const* lv, int n, KLevel* out, int* ainv, int* rscr) {
 }
 
 // largest cluster the kernel may use: 16 CTAs if a 16-CTA cluster of it is
-// schedulable (non-portable size), else 8; SF_COARSE_MAX_CS caps it (A/B)
+// schedulable (non-portable size), else 8; SF_COARSE_MAX_CS caps it (A/B, tests)
 int max_cluster() {
-    static int m = 0;
-    if (!m) {
-        m = 8;
+    static int probed = 0;
+    if (!probed) {
+        probed = 8;
         if (cudaFuncSetAttribute(coarse_vcycle_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) ==
                 cudaSuccess &&
             cudaFuncSetAttribute(coarse_vcycle_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -641,12 +726,12 @@ int max_cluster() {
             c.numAttrs = 1;
             int nc = 0;
             if (cudaOccupancyMaxActiveClusters(&nc, coarse_vcycle_kernel, &c) == cudaSuccess && nc >= 1)
-                m = CS_MAX;
+                probed = CS_MAX;
         }
         cudaGetLastError();
-        if (const char* e = getenv("SF_COARSE_MAX_CS")) m = std::max(1, std::min(m, atoi(e)));
     }
-    return m;
+    const char* e = getenv("SF_COARSE_MAX_CS");
+    return e ? std::max(1, std::min(probed, atoi(e))) : probed;
 }
 
 }  // namespace

@@ -1,10 +1,11 @@
-"""The coarse-level V-cycle as one single-CTA launch (coarse.cu, iterates in
-shared memory) from the first single-part level of <= 16^3 cells down to the
-bottom and back:
-every colour sweep, residual + restriction, P0 interpolation and the exact
-bottom solve run in one kernel, __syncthreads between phases.
-Compared with the oracle (1e-11 per cycle, same cycle counts per solve) and
-with the per-phase launches it replaces (SF_COARSE_KERNEL=0)."""
+"""The coarse-level V-cycle as one thread-block-cluster launch (coarse.cu:
+nz/2 CTAs of one 2-plane layer each, iterates in registers / shared memory,
+DSMEM z-neighbours, the coarsest levels gathered on CTA 0) from the first
+single-part level of <= 32^3 cells down to the bottom and back: every colour
+sweep, residual + restriction, P0 interpolation and the exact bottom solve run
+in one kernel.  Compared with the oracle (1e-11 per cycle, same cycle counts
+per solve) and with the per-phase launches it replaces (SF_COARSE_KERNEL=0),
+for cluster caps 16 / 8 / 4 (SF_COARSE_MAX_CS: entry levels 32^3 / 16^3 / 8^3)."""
 import numpy as np
 import pytest
 
@@ -67,15 +68,46 @@ def test_coarse_kernel_cycles_vs_oracle(sf, oracle, shape, monkeypatch):
         assert rel(a, b) < 1e-12
 
 
+@pytest.mark.parametrize("cap", ["8", "4"])
+@pytest.mark.parametrize("shape", [(64, 64, 64), (32, 64, 128)])
+def test_coarse_kernel_cluster_caps(sf, oracle, shape, cap, monkeypatch):
+    """Smaller clusters (entry 16^3 / 8^3 on the cube): same results."""
+    monkeypatch.setenv("SF_COARSE_MAX_CS", cap)
+    nz, ny, nx = shape
+    on, f = _run(sf, shape, True, monkeypatch, fcycle=True)
+    off, _ = _run(sf, shape, False, monkeypatch, fcycle=True)
+    h = I.level_h(nx, ny, nz)
+    O = oracle.MG(nx, ny, nz, h, 1.0, 1.0, *I.hpgmg_coeffs(nx, ny, nz, h))
+    u = O.fcycle(f)
+    exp = [u]
+    for _ in range(2):
+        u = O.vcycle(u, f)
+        exp.append(u)
+    for a, b, e in zip(on, off, exp):
+        assert rel(a, e) < 1e-11
+        assert rel(a, b) < 1e-12
+
+
 @pytest.mark.parametrize("opts", [{"pre_pairs": 1, "post_pairs": 3},
+                                  {"pre_pairs": 0, "post_pairs": 2},   # no folded red sweep
+                                  {"pre_pairs": 2, "post_pairs": 0},
                                   {"smoother": 1},   # SF_SMOOTH_COLOUR
                                   {"pre_pairs": 3, "post_pairs": 1, "use_graph": 0}])
 def test_coarse_kernel_options(sf, oracle, opts, monkeypatch):
     shape = (64, 64, 64)
-    on, _ = _run(sf, shape, True, monkeypatch, **opts)
+    on, f = _run(sf, shape, True, monkeypatch, **opts)
     off, _ = _run(sf, shape, False, monkeypatch, **opts)
     for a, b in zip(on, off):
         assert rel(a, b) < 1e-12
+    if "smoother" not in opts:   # the oracle's smoother is GSRB with the same pair counts
+        n = shape[0]
+        h = I.level_h(n, n, n)
+        O = oracle.MG(n, n, n, h, 1.0, 1.0, *I.hpgmg_coeffs(n, n, n, h),
+                      pre=opts["pre_pairs"], post=opts["post_pairs"])
+        u = np.zeros_like(f)
+        for a in on:
+            u = O.vcycle(u, f)
+            assert rel(a, u) < 1e-11
 
 
 @pytest.mark.parametrize("n", [32, 64, 128])
