@@ -1,6 +1,7 @@
-// Device helpers shared by the TMA-fed colour-fused smoothers (gsrb_fused.cu,
-// gsrb_rr.cu): mbarrier / cp.async.bulk.tensor wrappers and the lambda-form
-// stencil sum.  Included inside each translation unit's anonymous namespace.
+// Device helpers shared by the TMA-fed smoothers (gsrb_fused.cu, gsrb_twopair.cu,
+// gsrb_rr.cu) and the coarse V-cycle (coarse.cu): mbarrier /
+// cp.async.bulk.tensor wrappers and the lambda-form stencil sum.  Included
+// inside each translation unit's anonymous namespace.
 #pragma once
 
 __device__ __forceinline__ unsigned smem_u32(const void* p) {
