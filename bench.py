@@ -479,7 +479,9 @@ def side_measurements(args, sf, torch, L, M, world, rank, barrier, max_over_rank
               for _ in range(2)]
     L.download(sf.SF_F, host_f.numpy())
     nb = host_f.numel() * 8
-    reps = max(2, min(args.steps, 8))   # right-hand sides per streamed call (fill / drain amortised)
+    # right-hand sides per streamed call: the timed region's K steps (fill and
+    # drain -- the first upload, the last download -- amortised over them)
+    reps = max(2, min(args.steps, 32))
     M.solve_stream([host_f] * 2, host_u)          # warm-up (staging allocation paths)
     barrier()
     t0 = time.perf_counter()

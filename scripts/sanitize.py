@@ -57,7 +57,7 @@ M.close(); L.close()
 
 # r02 kernels: NEXT-1 two-pair smoother (4 chunk depths incl. ragged ones),
 # sf_interpolate_smooth on the 32x16 P0-fused build, the persistent residual +
-# restriction with forced multi-item chunking; the coarse single-CTA V-cycle
+# restriction with forced multi-item chunking; the coarse cluster V-cycle
 # runs inside every solve above (levels <= 16^3)
 for dep in ("0", "1", "3", "7"):
     if dep != "0":
