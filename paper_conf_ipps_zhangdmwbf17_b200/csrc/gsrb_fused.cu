@@ -251,7 +251,9 @@ __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
                      CoarseView cv, int c0, int cstride, unsigned long long* ts, int bd,
-                     int nch, int tcount) { pdl_wait();
+                     int nch, int tcount, int zero_rmax) { pdl_wait();
+    // SF_RM_ZERO: reset the BRES scalar of a later pair (no separate launch)
+    if (zero_rmax && blockIdx.x == 0 && threadIdx.x == 0) *rmax = 0.0;
     // live timing (sf_level_pair_timing): thread 0 of every CTA stamps its start
     // and end on the global timer; the last CTA to finish books end - start
     bool timing = false;
@@ -719,14 +721,16 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
             sf_launch(zero_bits, 1, 1, 0, L->stream, rmax);
             SF_LAUNCHED();
         }
+        const int zr = rmode == SF_RM_ZERO && p == 0 && phase != 2;
+        const bool bres = rmode == SF_RM_OUTPUT_BLACK || rmode == SF_RM_OUTPUT_BLACK_ZEROED;
         double* xo = v.f[xout];
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
     sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride, \
-              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1)
+              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1, zr)
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
-        else if (rmode == SF_RM_OUTPUT_BLACK && C) SF_LAUNCH_PAIR(false, true, true);
-        else if (rmode == SF_RM_OUTPUT_BLACK) SF_LAUNCH_PAIR(false, false, true);
+        else if (bres && C) SF_LAUNCH_PAIR(false, true, true);
+        else if (bres) SF_LAUNCH_PAIR(false, false, true);
         else if (C) SF_LAUNCH_PAIR(false, true, false);
         else SF_LAUNCH_PAIR(false, false, false);
 #undef SF_LAUNCH_PAIR

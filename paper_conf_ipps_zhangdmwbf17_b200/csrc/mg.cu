@@ -328,10 +328,11 @@ static bool fused_check_ok(const sf_mg* m);
 // The finest level's last post-smoothing pair of a cycle also reduces the black
 // part of max|F - A U| of its output into dscratch (BRES); the next cycle's
 // first pair adds the red part of the same iterate (fused check, below).
-static sf_status bres_pair(sf_mg* m, sf_level* L) {
+// zeroed: an earlier pair of the cycle already reset dscratch[0] (SF_RM_ZERO).
+static sf_status bres_pair(sf_mg* m, sf_level* L, bool zeroed = false) {
     SF_TRY(sf_halo(L, SF_F, 1));
     SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, L->dscratch, nullptr, 0,
-                            SF_RM_OUTPUT_BLACK));
+                            zeroed ? SF_RM_OUTPUT_BLACK_ZEROED : SF_RM_OUTPUT_BLACK));
     sf_swap_fields(L, SF_U, SF_TMP);
     return SF_OK;
 }
@@ -375,13 +376,14 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = fa
         // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
         SF_TRY(sf_halo(C, SF_U, 1));
         SF_TRY(sf_halo(L, SF_F, 1));
+        // (a later BRES pair: this one resets its scalar, saving a launch)
         const bool last = bres && m->o.post_pairs == 1;
-        SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, last ? L->dscratch : nullptr, C,
-                                SF_U, last ? SF_RM_OUTPUT_BLACK : SF_RM_NONE));
+        SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, bres ? L->dscratch : nullptr, C,
+                                SF_U, last ? SF_RM_OUTPUT_BLACK : bres ? SF_RM_ZERO : SF_RM_NONE));
         sf_swap_fields(L, SF_U, SF_TMP);
         if (bres && m->o.post_pairs >= 2) {
             SF_TRY(smooth(m, L, m->o.post_pairs - 2));
-            return bres_pair(m, L);
+            return bres_pair(m, L, true);
         }
         SF_TRY(smooth(m, L, m->o.post_pairs - 1));
         return SF_OK;

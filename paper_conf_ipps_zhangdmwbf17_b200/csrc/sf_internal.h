@@ -142,7 +142,10 @@ void sf_count_launch(long long n = 1);
 sf_status sf_check_launch(const char* what);
 
 // residual reductions riding in a fused pair (rmax = device scalar)
-enum { SF_RM_NONE = 0, SF_RM_INPUT_RED = 1, SF_RM_OUTPUT_BLACK = 2 };
+// SF_RM_ZERO: the pair only zeroes *rmax (for a BRES pair later in the stream,
+// which then skips its own reset launch: SF_RM_OUTPUT_BLACK_ZEROED)
+enum { SF_RM_NONE = 0, SF_RM_INPUT_RED = 1, SF_RM_OUTPUT_BLACK = 2, SF_RM_ZERO = 3,
+       SF_RM_OUTPUT_BLACK_ZEROED = 4 };
 
 // ------------------------------------------------------------------ kernels (kernels.cu)
 sf_status k_apply_op(sf_level* L, int out, int x, double a, double b);
