@@ -443,6 +443,35 @@ def test_c2_solve_parity(sf, oracle, fcycle):
     assert abs(np.abs(u - ue).max() - 5.19e-7) < 0.05e-6
 
 
+@pytest.mark.parametrize("pre,post", [(1, 3), (3, 1), (2, 2), (1, 1)])
+@pytest.mark.parametrize("use_graph", [0, 1])
+def test_fused_check_pair_counts(sf, oracle, pre, post, use_graph):
+    """The convergence check fused into the pairs (red part reduced by the next
+    cycle's first pair, black part by the last post pair, whose reset rides in
+    the P0-fused pair when post >= 2) for several pre/post pair counts: the
+    oracle's cycle count and residual history, u within 1e-10.  V(1,1) with P0
+    interpolation stalls at relres ~1 on this problem -- in the oracle too --
+    so it is compared over 12 cycles (SF_ERR_NOT_CONVERGED on both sides)."""
+    n = 64
+    h = 1.0 / n
+    coeffs = I.hpgmg_coeffs(n, n, n, h)
+    L = make_level(sf, (n, n, n), coeffs, h=h)
+    M = sf.MG(L, 1.0, 1.0, pre_pairs=pre, post_pairs=post, use_graph=use_graph)
+    O = oracle.MG(n, n, n, h, 1.0, 1.0, *coeffs, pre=pre, post=post)
+    _, f = I.manufactured(n, n, n, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    maxc = 12 if (pre, post) == (1, 1) else 50
+    st, cyc, hist = M.solve(fcycle=False, rtol=1e-10, max_cycles=maxc, raise_on_error=False)
+    u_o, hist_o = O.solve(f, fcycle=False, rtol=1e-10, maxc=maxc)
+    assert cyc == len(hist_o)
+    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-14)
+    assert rel(L.download(sf.SF_U), u_o) < 1e-10
+    if (pre, post) == (1, 1):
+        assert st == sf.SF_ERR_NOT_CONVERGED and hist[-1] > 0.5
+    else:
+        assert st == sf.SF_OK and hist[-1] < 1e-10
+
+
 @pytest.mark.parametrize("shape", [(32, 16, 64), (64, 32, 32), (32, 64, 32)])
 @pytest.mark.parametrize("use_graph", [0, 1])
 def test_noncube_solve_parity(sf, oracle, shape, use_graph):
