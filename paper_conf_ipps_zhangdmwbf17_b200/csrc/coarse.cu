@@ -533,60 +533,11 @@ __global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_const
     __syncthreads();
 #endif
     TRACE();
-    pdl_wait();
-    TRACE();
     const int nl = A.nlev;
     const int k0 = 2 * M.rank;
-    // ---- the entry block of this thread into registers (and its x into shared)
-    const KLevel& E = A.lv[0];
-    Block B;
-    {
-        const int t = threadIdx.x;
-        const int lhx = E.lx - 1;
-        B.own = t < (1 << (lhx + E.ly - 1));
-        B.i0 = 2 * (t & ((1 << lhx) - 1));
-        B.j0 = 2 * (t >> lhx);
-        const PV& v = E.v;
-        const long q0 = sf_ix(v, B.i0, B.j0, k0);
-        // 16-byte loads of x-adjacent pairs (i0 even, rows 32-byte aligned):
-        // a warp reads whole contiguous row segments
-        auto ld2 = [&](int f, long q) {
-            return B.own ? __ldg((const double2*)(v.f[f] + q)) : make_double2(0.0, 0.0);
-        };
-        auto ld1 = [&](int f, long q) { return B.own ? __ldg(v.f[f] + q) : 0.0; };
-#pragma unroll
-        for (int r = 0; r < 4; r++) {   // rows (dj, dk) = (r & 1, r >> 1): sub-cells 2r, 2r+1
-            const long q = q0 + (r & 1) * v.js + (r >> 1) * v.ks;
-            double2 t2 = A.uzero ? make_double2(0.0, 0.0) : ld2(SF_U, q);
-            B.X[2 * r] = t2.x; B.X[2 * r + 1] = t2.y;
-            t2 = ld2(SF_F, q);
-            B.F[2 * r] = t2.x; B.F[2 * r + 1] = t2.y;
-            t2 = ld2(SF_DINV, q);
-            B.D[2 * r] = t2.x; B.D[2 * r + 1] = t2.y;
-            t2 = ld2(SF_ALPHA, q);
-            B.A[2 * r] = t2.x; B.A[2 * r + 1] = t2.y;
-            // beta_i faces i0, i0+1 (pair) and i0+2 at (dj, dk) = (r & 1, r >> 1)
-            t2 = ld2(SF_BETA_I, q);
-            B.BI[0][r & 1][r >> 1] = t2.x; B.BI[1][r & 1][r >> 1] = t2.y;
-            B.BI[2][r & 1][r >> 1] = ld1(SF_BETA_I, q + 2);
-        }
-#pragma unroll
-        for (int f = 0; f < 3; f++)
-#pragma unroll
-            for (int r = 0; r < 2; r++) {
-                // beta_j face j0+f at dk = r, beta_k face k0+f at dj = r: di = 0, 1 as a pair
-                double2 t2 = ld2(SF_BETA_J, q0 + f * v.js + r * v.ks);
-                B.BJ[f][0][r] = t2.x; B.BJ[f][1][r] = t2.y;
-                t2 = ld2(SF_BETA_K, q0 + r * v.js + f * v.ks);
-                B.BK[f][0][r] = t2.x; B.BK[f][1][r] = t2.y;
-            }
-        if (B.own) {
-            double* U = sm + E.u;
-#pragma unroll
-            for (int s = 0; s < 8; s++)
-                U[B.i0 + (s & 1) + ((B.j0 + ((s >> 1) & 1) + ((s >> 2) << E.ly)) << E.lx)] = B.X[s];
-        }
-    }
+    // Constant operands first -- before griddepcontrol.wait, so with an early
+    // trigger in the previous kernel (k_residual_restrict) they load while it
+    // still runs; only F and U of the entry are that kernel's output.
     // ---- staging (async): D / alpha / faces of the CTA's planes of every
     // level below the entry, the bottom inverse on CTA 0
     for (int l = 1; l + 1 < nl; l++) {
@@ -623,6 +574,59 @@ __global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_const
                          : "memory");
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
+    // ---- the entry block of this thread into registers: Dinv, alpha, faces
+    const KLevel& E = A.lv[0];
+    const PV& ev = E.v;
+    Block B;
+    B.own = threadIdx.x < (1 << (E.lx - 1 + E.ly - 1));
+    B.i0 = 2 * (threadIdx.x & ((1 << (E.lx - 1)) - 1));
+    B.j0 = 2 * (threadIdx.x >> (E.lx - 1));
+    const long q0 = sf_ix(ev, B.i0, B.j0, k0);
+    // 16-byte loads of x-adjacent pairs (i0 even, rows 32-byte aligned): a warp
+    // reads whole contiguous row segments
+    auto ld2 = [&](int f, long q) {
+        return B.own ? __ldg((const double2*)(ev.f[f] + q)) : make_double2(0.0, 0.0);
+    };
+    auto ld1 = [&](int f, long q) { return B.own ? __ldg(ev.f[f] + q) : 0.0; };
+#pragma unroll
+    for (int r = 0; r < 4; r++) {   // rows (dj, dk) = (r & 1, r >> 1): sub-cells 2r, 2r+1
+        const long q = q0 + (r & 1) * ev.js + (r >> 1) * ev.ks;
+        double2 t2 = ld2(SF_DINV, q);
+        B.D[2 * r] = t2.x; B.D[2 * r + 1] = t2.y;
+        t2 = ld2(SF_ALPHA, q);
+        B.A[2 * r] = t2.x; B.A[2 * r + 1] = t2.y;
+        // beta_i faces i0, i0+1 (pair) and i0+2 at (dj, dk) = (r & 1, r >> 1)
+        t2 = ld2(SF_BETA_I, q);
+        B.BI[0][r & 1][r >> 1] = t2.x; B.BI[1][r & 1][r >> 1] = t2.y;
+        B.BI[2][r & 1][r >> 1] = ld1(SF_BETA_I, q + 2);
+    }
+#pragma unroll
+    for (int f = 0; f < 3; f++)
+#pragma unroll
+        for (int r = 0; r < 2; r++) {
+            // beta_j face j0+f at dk = r, beta_k face k0+f at dj = r: di = 0, 1 as a pair
+            double2 t2 = ld2(SF_BETA_J, q0 + f * ev.js + r * ev.ks);
+            B.BJ[f][0][r] = t2.x; B.BJ[f][1][r] = t2.y;
+            t2 = ld2(SF_BETA_K, q0 + r * ev.js + f * ev.ks);
+            B.BK[f][0][r] = t2.x; B.BK[f][1][r] = t2.y;
+        }
+    pdl_wait();   // the previous kernel's output from here on
+    TRACE();
+    // ---- the entry's F and U (registers; U mirrored in shared memory)
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        const long q = q0 + (r & 1) * ev.js + (r >> 1) * ev.ks;
+        double2 t2 = A.uzero ? make_double2(0.0, 0.0) : ld2(SF_U, q);
+        B.X[2 * r] = t2.x; B.X[2 * r + 1] = t2.y;
+        t2 = ld2(SF_F, q);
+        B.F[2 * r] = t2.x; B.F[2 * r + 1] = t2.y;
+    }
+    if (B.own) {
+        double* U = sm + E.u;
+#pragma unroll
+        for (int s = 0; s < 8; s++)
+            U[B.i0 + (s & 1) + ((B.j0 + ((s >> 1) & 1) + ((s >> 2) << E.ly)) << E.lx)] = B.X[s];
+    }
     cluster_sync();
     // ---- V(l0) down to the bottom and back
     smooth(E, M, &B, A.a, A.pre);

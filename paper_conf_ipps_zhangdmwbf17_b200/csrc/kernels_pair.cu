@@ -171,7 +171,11 @@ __device__ __forceinline__ double2 neg2(double2 u) { return make_double2(-u.x, -
 template <int MINB>
 __global__ void __launch_bounds__(PX* PY, MINB) residual_restrict_zs_kernel(
     PV f, const double* __restrict__ x, const double* __restrict__ rhs, double a, double bh2, PV c,
-    double* __restrict__ cx, int zoff, int depth, int tgx, int ntiles, int nitems) { pdl_wait();
+    double* __restrict__ cx, int zoff, int depth, int tgx, int ntiles, int nitems, int trig) { pdl_wait();
+    // trig: the next launch (the coarse cluster V-cycle) may start now -- it
+    // stages its constant coefficients while this kernel runs and waits for
+    // this kernel's output (the coarse rhs) in griddepcontrol.wait
+    if (trig) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int nK = f.nz / 2;
     const double* bj = f.f[SF_BETA_J];
     const double* bk = f.f[SF_BETA_K];
@@ -484,7 +488,8 @@ sf_status k_residual_pair(sf_level* L, int res, int x, int rhs, double a, double
     return sf_check_launch("residual_pair");
 }
 
-sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf) {
+sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf,
+                              bool trigger_next) {
     const double bh2 = b / (F->h * F->h);
     const bool rep = C->nparts == 1 && F->nparts > 1;
     SF_TRY(sf_halo(F, x, 1));
@@ -513,7 +518,8 @@ sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, s
                 if (atoi(e) > 0) grid = std::min(items, atoi(e));
 #define SF_RRZS(MB)                                                                              \
     sf_launch(residual_restrict_zs_kernel<MB>, grid, dim3(PX, PY), 0, F->stream,                         \
-        f, f.f[x], f.f[rhs], a, bh2, c, c.f[cf], rep ? f.z0 / 2 : 0, best_d, tgx, tiles, items)
+        f, f.f[x], f.f[rhs], a, bh2, c, c.f[cf], rep ? f.z0 / 2 : 0, best_d, tgx, tiles, items, \
+        trigger_next && !rep ? 1 : 0)
             if (rr_zs() == 2) SF_RRZS(6);
             else if (rr_zs() == 3) SF_RRZS(8);
             else SF_RRZS(4);

@@ -361,7 +361,10 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = fa
     } else {
         SF_TRY(smooth(m, L, pre));
         if (pair_ok(L)) {  // residual never stored: A6 + A7 in one pass
-            SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F));
+            // the coarse cluster V-cycle follows directly: it may launch early
+            const bool next_coarse = m->coarse_l0 >= 1 && l + 1 == m->coarse_l0 &&
+                                     l + 1 < (int)m->lv.size() - 1;
+            SF_TRY(k_residual_restrict(L, SF_U, SF_F, m->a, m->b, C, SF_F, next_coarse));
         } else {
             SF_TRY(k_residual(L, SF_R, SF_U, SF_F, m->a, m->b));
             SF_TRY(k_restrict(C, SF_F, L, SF_R, SF_RESTRICT_CELL));

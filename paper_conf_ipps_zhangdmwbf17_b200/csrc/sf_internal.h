@@ -166,7 +166,10 @@ sf_status k_bottom_solve(sf_level* L, int x, int rhs, const double* ainv);
 bool pair_ok(const sf_level* L);
 sf_status k_residual_pair(sf_level* L, int res /* -1: do not write */, int x, int rhs, double a,
                           double b, double* max_out /* NULL: no norm */);
-sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf);
+// trigger_next: let the next launch start early (PDL trigger; it must only
+// read this kernel's output after griddepcontrol.wait -- the coarse cluster V-cycle)
+sf_status k_residual_restrict(sf_level* F, int x, int rhs, double a, double b, sf_level* C, int cf,
+                              bool trigger_next = false);
 sf_status k_interp_p0_pair(sf_level* F, int ff, double s, sf_level* C, int cf);
 sf_status k_norm_pair(sf_level* L, int field, int kind, double* dst);
 sf_status k_cc(sf_level* L, int out, int x, int f, double omega, bool jacobi);  // NEXT-2
