@@ -773,3 +773,36 @@ def test_chebyshev_multigrid(sf, oracle, graph):
     st, cyc, hist = M.solve(fcycle=True, rtol=1e-10)
     u_o, hist_o = O.solve(f, fcycle=True, rtol=1e-10)
     assert cyc == len(hist_o) and rel(L.download(sf.SF_U), u_o) < 1e-10
+
+
+# ------------------------------------------------------- NEXT-2 / NEXT-3 at the bench size
+def test_next2_next3_full_size_256(sf, oracle):
+    """The Fig-7 operators at the 256^3 the bench times them on: the CC 7-point
+    Laplacian, the CC weighted Jacobi step and one degree-2 Chebyshev
+    application on the VC operator, every cell against the oracle (rel-L2 and
+    max-abs relative to the largest value)."""
+    shape = (256, 256, 256)
+    nz, ny, nx = shape
+    h = I.level_h(nx, ny, nz)
+    x, f = I.random_field(shape, 0), I.random_field(shape, 1)
+    L = sf.Level(nx, ny, nz, h)
+    L.upload(sf.SF_U, x)
+    L.upload(sf.SF_F, f)
+    sf.sf_apply_laplacian(L.handle, sf.SF_R, sf.SF_U)
+    e = oracle.laplacian_cc(x, h)
+    out = L.download(sf.SF_R)
+    assert rel(out, e) < TOL and np.abs(out - e).max() <= TOL * np.abs(e).max()
+    sf.sf_jacobi(L.handle, sf.SF_TMP, sf.SF_U, sf.SF_F, 2.0 / 3.0)
+    e = oracle.jacobi_cc(x, f, h)
+    out = L.download(sf.SF_TMP)
+    assert rel(out, e) < TOL and np.abs(out - e).max() <= TOL * np.abs(e).max()
+    coeffs = I.hpgmg_coeffs(nx, ny, nz, h)
+    L.set_coeffs(*coeffs)
+    sf.sf_rebuild_operator(L.handle, 1.0, 1.0)
+    P = oracle.Problem(oracle.Grid(nx, ny, nz, h), 1.0, 1.0, *coeffs)
+    L.upload(sf.SF_U, x)
+    sf.sf_smooth_chebyshev(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 2, 20.0, 900.0)
+    e = P.chebyshev(x, f, 2, 20.0, 900.0)
+    out = L.download(sf.SF_U)
+    assert rel(out, e) < TOL and np.abs(out - e).max() <= 10 * TOL * np.abs(e).max()
+    L.close()
