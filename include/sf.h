@@ -295,6 +295,12 @@ sf_status sf_level_pair_timing_variants(const sf_level* level, double mean_ms[4]
  *   every level, down to min dim 2 (exact bottom solve, R-8).  Levels whose
  *   slabs would hold fewer than opts->agglom_min_planes planes are
  *   agglomerated (replicated on every part/rank).  opts NULL = defaults.
+ *   From the first single-part power-of-two level of <= 32^3 cells down, a
+ *   V-cycle runs as ONE thread-block-cluster launch (up to 16 CTAs, operands
+ *   in registers / shared memory; coarse.cu); same arithmetic as the per-phase
+ *   kernels up to rounding (the sweeps in the fused pairs' lambda form).  The
+ *   environment variable SF_COARSE_KERNEL=0, read at sf_mg_create, keeps the
+ *   per-phase launches.
  * sf_vcycle: one V-cycle on level l (U_l corrected for rhs F_l), enqueued.
  * sf_fcycle: one F-cycle from scratch for rhs F_0 into U_0, enqueued.
  * sf_solve: optional F-cycle, then V-cycles until ||F-AU||inf/||F||inf <
