@@ -73,6 +73,7 @@ struct KArgs {
     int ainv;             // shared offset of the bottom inverse (CTA 0)
     int rscr;             // shared offset of the residual scratch (GMAX doubles)
     int uzero;            // the entry level's U is zero (V-cycle): not read
+    int trig;             // let the next launch start early (it reads only our U of the entry)
     const double* ainv_g; // n x n, row major
 };
 
@@ -611,6 +612,7 @@ __global__ void __launch_bounds__(NT, 1) coarse_vcycle_kernel(const __grid_const
             B.BK[f][0][r] = t2.x; B.BK[f][1][r] = t2.y;
         }
     pdl_wait();   // the previous kernel's output from here on
+    if (A.trig) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     TRACE();
     // ---- the entry's F and U (registers; U mirrored in shared memory)
 #pragma unroll
@@ -763,7 +765,7 @@ bool coarse_vcycle_fits(sf_level* const* lv, int n) {
 
 // V(lv[0]) down to the bottom lv[n-1] and back: one launch of one cluster
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
-                          int pre, int post, bool u_zero) {
+                          int pre, int post, bool u_zero, bool trigger_next) {
     if (!coarse_vcycle_fits(lv, n)) return sf_fail(SF_ERR_SHAPE, "coarse V-cycle levels do not fit");
     KArgs A = {};
     const long doubles = plan_smem(lv, n, A.lv, &A.ainv, &A.rscr);
@@ -780,6 +782,7 @@ sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const 
     A.a = a;
     A.ainv_g = ainv;
     A.uzero = u_zero ? 1 : 0;
+    A.trig = trigger_next ? 1 : 0;
     const int C = lv[0]->lnz / 2;
 #ifdef SF_COARSE_TRACE
     for (int l = 0; l < n; l++)

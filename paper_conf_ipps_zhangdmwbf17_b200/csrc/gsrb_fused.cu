@@ -251,9 +251,19 @@ __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
                      CoarseView cv, int c0, int cstride, unsigned long long* ts, int bd,
-                     int nch, int tcount, int zero_rmax) { pdl_wait();
-    // SF_RM_ZERO: reset the BRES scalar of a later pair (no separate launch)
-    if (zero_rmax && blockIdx.x == 0 && threadIdx.x == 0) *rmax = 0.0;
+                     int nch, int tcount, int zero_rmax, int early) {
+    // early: the launch before this one triggered early and wrote nothing this
+    // pair reads but the P0 source -- the first item's TMA prologue is issued
+    // before griddepcontrol.wait (it overlaps that launch)
+    bool waited = !early;
+    auto after_wait = [&]() {
+        // SF_RM_ZERO: reset the BRES scalar of a later pair (no separate launch)
+        if (zero_rmax && blockIdx.x == 0 && threadIdx.x == 0) *rmax = 0.0;
+    };
+    if (!early) {
+        pdl_wait();
+        after_wait();
+    }
     // live timing (sf_level_pair_timing): thread 0 of every CTA stamps its start
     // and end on the global timer; the last CTA to finish books end - start
     bool timing = false;
@@ -335,6 +345,11 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, zplane(g, z0 - 1), b);
             tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, zplane(g, z0 - 1), b);
             for (int q = z0 - 1; q <= min(z0 + PF - 2, z1); q++) issue(q);  // step t: t+PF+1
+        }
+        if (!waited) {
+            pdl_wait();
+            after_wait();
+            waited = true;
         }
 
         // this thread's pair: row gy, cells gxa (even) and gxa+1
@@ -721,13 +736,16 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
             sf_launch(zero_bits, 1, 1, 0, L->stream, rmax);
             SF_LAUNCHED();
         }
+        // (after a zero_bits launch the pair cannot start early)
+        const int early = L->pdl_early && phase == 0 && L->nlocal == 1 && rmode != SF_RM_OUTPUT_BLACK &&
+                          sf_pdl_on();
         const int zr = rmode == SF_RM_ZERO && p == 0 && phase != 2;
         const bool bres = rmode == SF_RM_OUTPUT_BLACK || rmode == SF_RM_OUTPUT_BLACK_ZEROED;
         double* xo = v.f[xout];
 #define SF_LAUNCH_PAIR(R, I, B)                                                                     \
     sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride, \
-              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1, zr)
+              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1, zr, early)
         if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (bres && C) SF_LAUNCH_PAIR(false, true, true);
         else if (bres) SF_LAUNCH_PAIR(false, false, true);
@@ -736,5 +754,6 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
 #undef SF_LAUNCH_PAIR
         SF_LAUNCHED();
     }
+    L->pdl_early = 0;
     return sf_check_launch("gsrb_pair_tma");
 }

@@ -341,14 +341,17 @@ static sf_status bres_pair(sf_mg* m, sf_level* L, bool zeroed = false) {
 // skip_first: the first pre-smoothing pair was already run (fused check, below).
 // u_zero: U of level l is zero on entry (the V-cycle recursion zeroed it, or
 // leaves that to the coarse-level launch, which then does not read it)
-static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = false) {
+// trig: the launch after this V(l) may start early (the P0-fused pair above a
+// coarse cluster V-cycle)
+static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = false,
+                      bool trig = false) {
     const bool bres = l == 0 && fused_check_ok(m);   // last post pair reduces the black residual
     sf_level* L = m->lv[l];
     NvtxRange nv("sf V(l=%d) %dx%dx%d", l, L->gnx, L->gny, L->gnz);
     if (l == (int)m->lv.size() - 1) return k_bottom_solve(L, SF_U, SF_F, m->ainv);
     if (m->coarse_l0 >= 1 && l >= m->coarse_l0)   // the whole V(l) in one launch
         return k_coarse_vcycle(&m->lv[l], (int)m->lv.size() - l, m->a, m->b, m->ainv,
-                               m->o.pre_pairs, m->o.post_pairs, u_zero);
+                               m->o.pre_pairs, m->o.post_pairs, u_zero, trig);
     sf_level* C = m->lv[l + 1];
     const int pre = m->o.pre_pairs - (skip_first ? 1 : 0);
     if (pre >= 1 && (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
@@ -372,15 +375,21 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = fa
     }
     const bool cz = m->coarse_l0 >= 1 && l + 1 >= m->coarse_l0 && l + 1 < (int)m->lv.size() - 1;
     if (!cz) SF_TRY(k_zero(C, SF_U));   // the coarse-level launch starts from zero itself
-    SF_TRY(vcyc(m, l + 1, false, cz));
-    if (m->o.vcycle_interp == SF_INTERP_P0 && m->o.post_pairs >= 1 &&
-        (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
-        gsrb_fused_supported(L)) {
+    // P0-fused pair right after a coarse cluster V-cycle: it may start under it
+    // (its TMA prologue reads only operands older than that launch)
+    const bool p0_pair = m->o.vcycle_interp == SF_INTERP_P0 && m->o.post_pairs >= 1 &&
+                         (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
+                         gsrb_fused_supported(L);
+    const bool early = p0_pair && cz && L->nparts == 1 && C->nparts == 1 &&
+                       !(bres && m->o.post_pairs == 1);
+    SF_TRY(vcyc(m, l + 1, false, cz, early));
+    if (p0_pair) {
         // e_l += P0 e_{l+1} fused into the first post-smoothing pair (A8 + A5)
         SF_TRY(sf_halo(C, SF_U, 1));
         SF_TRY(sf_halo(L, SF_F, 1));
         // (a later BRES pair: this one resets its scalar, saving a launch)
         const bool last = bres && m->o.post_pairs == 1;
+        L->pdl_early = early ? 1 : 0;
         SF_TRY(k_gsrb_pair_halo(L, SF_U, SF_TMP, SF_F, m->a, m->b, bres ? L->dscratch : nullptr, C,
                                 SF_U, last ? SF_RM_OUTPUT_BLACK : bres ? SF_RM_ZERO : SF_RM_NONE));
         sf_swap_fields(L, SF_U, SF_TMP);

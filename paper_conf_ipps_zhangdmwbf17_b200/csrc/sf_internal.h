@@ -68,6 +68,10 @@ struct sf_level {
     double* hscratch;          // pinned, mapped host scalars
     double* hscratch_dev;      // their device alias
     double ts_var[4][2] = {};  // last sf_level_pair_timing read-out per variant: launches, ns
+    // the next fused pair may start under the launch before it (that launch
+    // triggers early and writes nothing the pair reads except the P0 source;
+    // set by the V-cycle, consumed by the pair launch)
+    int pdl_early = 0;
     std::vector<char*> peer;   // kind-2 comm: peer ranks' level buffers (CUDA IPC), by rank
     std::vector<void*> ipc_opened;
 };
@@ -226,8 +230,9 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
 bool coarse_vcycle_fits(sf_level* const* lv, int n);
 int coarse_vcycle_max_levels();
 // u_zero: lv[0]'s U is zero on entry (V-cycle recursion): not read, not zeroed first
+// trigger_next: the launch after it may start early (griddepcontrol.launch_dependents)
 sf_status k_coarse_vcycle(sf_level* const* lv, int n, double a, double b, const double* ainv,
-                          int pre, int post, bool u_zero);
+                          int pre, int post, bool u_zero, bool trigger_next = false);
 
 // ------------------------------------------------------------------ comm (comm.cu)
 // Exchange `depth` z-halo planes of `field` between neighbouring parts.
