@@ -16,8 +16,13 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-BUILD = os.path.join(PKG, "_build")
-LIB = os.path.join(PKG, "libsf.so")
+# SF_VARIANT=name (A/B builds only): objects under _build_<name>, library
+# libsf_<name>.so, SF_VARIANT_FLAGS added to the fused-pair objects; loaded
+# with SF_LIB=<path> (sf.py)
+_VARIANT = os.environ.get("SF_VARIANT", "")
+BUILD = os.path.join(PKG, "_build" + (f"_{_VARIANT}" if _VARIANT else ""))
+LIB = os.path.join(PKG, f"libsf_{_VARIANT}.so" if _VARIANT else "libsf.so")
+_VFLAGS = os.environ.get("SF_VARIANT_FLAGS", "").split() if _VARIANT else []
 # (source, object, extra flags): the fused GSRB source is built for two tile shapes
 SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            ("kernels_pair.cu", "kernels_pair.o", []),
@@ -56,6 +61,8 @@ def _compile(spec, force):
             os.path.join(INCLUDE, "sf.h")]
     if not force and not _needs(o, deps):
         return o, ""
+    if src == "gsrb_fused.cu":
+        extra = [*extra, *_VFLAGS]
     cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", s, "-o", o]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:

@@ -103,6 +103,15 @@ static_assert(TX % 2 == 0 && 32 % PPR == 0, "tile shape");
 enum { CA_DV = 0, CA_RH = 1, CA_BI = 2, CA_BJ = 3 };
 constexpr int NRING = TX + TY;         // red ring cells per plane (half of the 1-ring)
 
+// measurement knob: SF_DBG_NOBC builds drop the Dirichlet selects (wrong
+// results at global faces; instruction-count A/B only,
+// profiles/r02/ab_nobc_selects.txt)
+#ifdef SF_DBG_NOBC
+#define BCZ(c) false
+#else
+#define BCZ(c) (c)
+#endif
+
 struct Maps {
     CUtensorMap x, dv, rh, bi, bj, bk;
 };
@@ -169,12 +178,12 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
         xw = xp2.x; xe = s.Xk[xo_ + 2];
     }
     const int gxr = gx + SEL;
-    if (gxr == 0) xw = 0.0;
-    if (gxr == g.nx - 1) xe = 0.0;
-    const double xs = (gy == 0) ? 0.0 : s.Xk[col - W];
-    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
-    const double xb = zlo ? 0.0 : (SEL ? pb.y : pb.x);
-    const double xt = zhi ? 0.0 : (SEL ? pt.y : pt.x);
+    if (BCZ(gxr == 0)) xw = 0.0;
+    if (BCZ(gxr == g.nx - 1)) xe = 0.0;
+    const double xs = BCZ(gy == 0) ? 0.0 : s.Xk[col - W];
+    const double xn = BCZ(gy == g.ny - 1) ? 0.0 : s.Xk[col + W];
+    const double xb = BCZ(zlo) ? 0.0 : (SEL ? pb.y : pb.x);
+    const double xt = BCZ(zhi) ? 0.0 : (SEL ? pt.y : pt.x);
     double r, S;
     if (SEL == 0) {
         S = sum6(xw, xe, xs, xn, xb, xt, bi2.x, bi2.y, bjl.x, bjh.x, bkl.x, bkh.x);
@@ -215,13 +224,13 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
         xw = rn_same; xe = s.Xm[xo_ + 2];
     }
     const int gxb = gx + SEL;
-    if (gxb == 0) xw = 0.0;
-    if (gxb == g.nx - 1) xe = 0.0;
+    if (BCZ(gxb == 0)) xw = 0.0;
+    if (BCZ(gxb == g.nx - 1)) xe = 0.0;
     const int col = xo_ + SEL;
-    const double xs = (gy == 0) ? 0.0 : s.Xm[col - W];
-    const double xn = (gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
-    const double xb = (gkm == 0) ? 0.0 : rn_below;
-    const double xt = (gkm == g.gnz - 1) ? 0.0 : rn_above;
+    const double xs = BCZ(gy == 0) ? 0.0 : s.Xm[col - W];
+    const double xn = BCZ(gy == g.ny - 1) ? 0.0 : s.Xm[col + W];
+    const double xb = BCZ(gkm == 0) ? 0.0 : rn_below;
+    const double xt = BCZ(gkm == g.gnz - 1) ? 0.0 : rn_above;
     const double q = gs_q(rb[7], bh2, sum6(xw, xe, xs, xn, xb, xt, rb[0], rb[1], rb[2], rb[3], rb[4], rb[5]));
     const double bnew = __dmul_rn(rb[6], q);
     if (BRES) bres = __fma_rn(-bnew, inv_fast(rb[6]), q);
@@ -231,12 +240,12 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
 // Ring red cell at smem offsets (xo_, co_) (scalar loads; bounds in flags)
 __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, int flags, double bh2,
                                            bool zlo, bool zhi) {
-    const double xw = (flags & 1) ? 0.0 : s.Xk[xo_ - 1];
-    const double xe = (flags & 2) ? 0.0 : s.Xk[xo_ + 1];
-    const double xs = (flags & 4) ? 0.0 : s.Xk[xo_ - W];
-    const double xn = (flags & 8) ? 0.0 : s.Xk[xo_ + W];
-    const double xb = zlo ? 0.0 : s.Xm[xo_];
-    const double xt = zhi ? 0.0 : s.Xp[xo_];
+    const double xw = BCZ(flags & 1) ? 0.0 : s.Xk[xo_ - 1];
+    const double xe = BCZ(flags & 2) ? 0.0 : s.Xk[xo_ + 1];
+    const double xs = BCZ(flags & 4) ? 0.0 : s.Xk[xo_ - W];
+    const double xn = BCZ(flags & 8) ? 0.0 : s.Xk[xo_ + W];
+    const double xb = BCZ(zlo) ? 0.0 : s.Xm[xo_];
+    const double xt = BCZ(zhi) ? 0.0 : s.Xp[xo_];
     const double S = sum6(xw, xe, xs, xn, xb, xt, s.C[CA_BI * CARR + co_],
                           s.C[CA_BI * CARR + co_ + 1], s.C[CA_BJ * CARR + co_],
                           s.C[CA_BJ * CARR + co_ + W], s.Klo[co_], s.Khi[co_]);
