@@ -324,9 +324,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
 
         // bundle q: x(q+1), Dinv/rhs/beta_i/beta_j (q), beta_k(q+1); needed by R(q).
         // Part k of the bundle (0: arrive.expect_tx + x, 1..4: coefficient
-        // arrays, 5: beta_k) -- in the steady state lane 0 of warp k issues part
-        // k, so no single warp carries the whole issue latency into the next
-        // step (arrivals and complete_tx may come in any order within a phase).
+        // arrays, 5: beta_k), all issued by thread 0 after the step's barrier
+        // (spreading the parts over the warps' lane 0 measured slower, c1a7abc).
         const unsigned xs_u = smem_u32(Xs), cs_u = smem_u32(Cs), ks_u = smem_u32(Ks);
         const unsigned mb_u = smem_u32(mbar);
         auto issue_part = [&](int q, int part) {
