@@ -91,8 +91,15 @@ constexpr int NCA = 4;                 // staged coefficient arrays per plane (b
 constexpr int XSLOT = (XH * W + 15) / 16 * 16;   // doubles, 128-byte multiple
 constexpr int CARR = (CHH * W + 15) / 16 * 16;
 constexpr int CSLOT = NCA * CARR;
-constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8;
-constexpr int BUNDLE_BYTES = XBYTES + (NCA + 1) * CBYTES;
+// Only beta_j (north faces of the ring's top row) needs the last coefficient
+// row; Dinv, rhs, beta_i and beta_k boxes stop one row short (CHS rows; the
+// slot's last row is never read).  SF_TRIM_ROWS=0 restores full boxes.
+#ifndef SF_TRIM_ROWS
+#define SF_TRIM_ROWS 1
+#endif
+constexpr int CHS = CHH - SF_TRIM_ROWS;
+constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8, CBYTES_S = CHS * W * 8;
+constexpr int BUNDLE_BYTES = XBYTES + (NCA - 1) * CBYTES_S + CBYTES + CBYTES_S;
 constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR) + 64;
 static_assert(MINB * (SMEM + 1024) <= 228 * 1024, "MINB CTAs per SM must fit in shared memory");
 // fused P0 interpolation (INTERP): each x-box pair (2 cells, one parent) is
@@ -348,7 +355,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         if (tid == 0) {
             fence_proxy_async();  // generic smem writes of the previous item before TMA reuse
             unsigned long long* b = &mbar[seq0 % NMB];
-            mbar_expect(b, 2 * XBYTES + CBYTES);
+            mbar_expect(b, 2 * XBYTES + CBYTES_S);
             tma3(Xs + md(z0 - 2, NXS) * XSLOT, &mp.x, cx, cyx, zplane(g, z0 - 2), b);
             tma3(Xs + md(z0 - 1, NXS) * XSLOT, &mp.x, cx, cyx, zplane(g, z0 - 1), b);
             tma3(Ks + md(z0 - 1, NKS) * CARR, &mp.bk, cx, cyc, zplane(g, z0 - 1), b);
@@ -725,11 +732,11 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         PV v = sf_view(L, p);
         Maps mp;
         SF_TRY(encode(&mp.x, L, v.f[xin], XH));
-        SF_TRY(encode(&mp.dv, L, v.f[SF_DINV], CHH));
-        SF_TRY(encode(&mp.rh, L, v.f[rhs], CHH));
-        SF_TRY(encode(&mp.bi, L, v.f[SF_BETA_I], CHH));
+        SF_TRY(encode(&mp.dv, L, v.f[SF_DINV], CHS));
+        SF_TRY(encode(&mp.rh, L, v.f[rhs], CHS));
+        SF_TRY(encode(&mp.bi, L, v.f[SF_BETA_I], CHS));
         SF_TRY(encode(&mp.bj, L, v.f[SF_BETA_J], CHH));
-        SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHH));
+        SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHS));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks, 0};
         if (const char* ez = getenv("SF_DBG_ZMASK"))   // measurement only (see zplane)
             if (atoi(ez) > 0 && v.nz > atoi(ez)) g.zmask = atoi(ez);

@@ -13,7 +13,7 @@ for rep in $(seq $reps); do
 import json,sys
 d=json.loads(open(f"gpurun_out/bench_{sys.argv[1]}.json").read().strip().splitlines()[-1])
 r=d["roofline"]
-print(sys.argv[1], "ms/step %.2f" % d["ms_per_step"], "clk", d["clocks"]["sm_mhz"], "frac %.3f" % r["frac"],
+print(sys.argv[1], "ms/step %.2f" % d["ms_per_step"], "cyc", d["config"].get("cycles_per_solve"), "clk", d["clocks"]["sm_mhz"], "frac %.3f" % r["frac"],
       {k: round(v["ms"], 4) for k, v in r["live_per_variant"].items()}, flush=True)
 PY
   done
