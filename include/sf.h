@@ -377,7 +377,7 @@ sf_status sf_launch_count(long long* count, int reset);
  *     q = floor((mul*p + pre) / div) + off            (p = output point)
  * -- plain offsets have mul = div = 1, pre = 0; restriction reads a fine level
  * at 2p + o (mul 2), P0 interpolation a coarse level at floor((p+1)/2) (div 2,
- * pre 1).  Reads may reach the storage ghost zone (x: OX = 4, y/z: 2 layers).
+ * pre 1).  Reads may reach the storage ghost zone (2 layers on every axis).
  *
  * Semantics: every point of a stencil's domain is computed from the values
  * before the stencil (points of one stencil are independent); stencils of a

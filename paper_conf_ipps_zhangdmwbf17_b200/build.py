@@ -23,6 +23,7 @@ _VARIANT = os.environ.get("SF_VARIANT", "")
 BUILD = os.path.join(PKG, "_build" + (f"_{_VARIANT}" if _VARIANT else ""))
 LIB = os.path.join(PKG, f"libsf_{_VARIANT}.so" if _VARIANT else "libsf.so")
 _VFLAGS = os.environ.get("SF_VARIANT_FLAGS", "").split() if _VARIANT else []
+_VAFLAGS = os.environ.get("SF_VARIANT_ALL_FLAGS", "").split() if _VARIANT else []   # every object
 # (source, object, extra flags): the fused GSRB source is built for two tile shapes
 SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            ("kernels_pair.cu", "kernels_pair.o", []),
@@ -63,7 +64,7 @@ def _compile(spec, force):
         return o, ""
     if src == "gsrb_fused.cu":
         extra = [*extra, *_VFLAGS]
-    cmd = [NVCC, *ARCH, *FLAGS, *extra, "-c", s, "-o", o]
+    cmd = [NVCC, *ARCH, *FLAGS, *extra, *_VAFLAGS, "-c", s, "-o", o]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")

@@ -12,11 +12,16 @@
 // ------------------------------------------------------------------ layout (A1)
 // Per part and field: (lnz + 2*SF_GZ) planes x (ny + 2*SF_GY) rows x js doubles.
 // Element (i,j,k) at (k+SF_GZ)*ks + (j+SF_GY)*js + SF_OX + i, i in [-2, nx+1].
-// SF_OX = 4 puts i = 0 on a 32-byte boundary (js is a multiple of 16 doubles,
-// every field base is 256-byte aligned), so double2 / 16-byte cp.async loads
-// of interior rows are aligned.  Two ghost planes in z (depth-2 slab halos of
+// SF_OX = 2 puts i = -2 on a 128-byte row start (js is a multiple of 16
+// doubles, every field base 256-byte aligned) and i = 0 on a 16-byte boundary:
+// the colour-fused pair's TMA boxes (x0-2 .. x0+TX+1, 36 doubles) then cover
+// 9 instead of 10 32-byte sectors per row (-10 % L2 -> SM bytes; 512^3 pair
+// -3.4 % under the power cap, profiles/r02/ab_ox2.txt), and double2 loads of
+// interior pairs stay aligned.  (OX = 4 put i = 0 on a 32-byte boundary.)  Two ghost planes in z (depth-2 slab halos of
 // the colour-fused smoother) and two ghost rows in y (its 2-ring tile loads).
-#define SF_OX 4
+#ifndef SF_OX
+#define SF_OX 2
+#endif
 #define SF_GY 2
 #define SF_GZ 2
 // per-level device scratch after the fields: 32 doubles + the P2P sync block
