@@ -110,13 +110,18 @@ static_assert(TX % 2 == 0 && 32 % PPR == 0, "tile shape");
 enum { CA_DV = 0, CA_RH = 1, CA_BI = 2, CA_BJ = 3 };
 constexpr int NRING = TX + TY;         // red ring cells per plane (half of the 1-ring)
 
-// measurement knob: SF_DBG_NOBC builds drop the Dirichlet selects (wrong
-// results at global faces; instruction-count A/B only,
-// profiles/r02/ab_nobc_selects.txt)
-#ifdef SF_DBG_NOBC
-#define BCZ(c) false
-#else
+// Dirichlet faces: the pair reads the boundary-zeroed face coefficients
+// (SF_BI0/BJ0/BK0, sf_internal.h), so a boundary neighbour's term is
+// 0 * (finite ghost) and no select is needed (13 % fewer instructions; the
+// pair 1.4 % faster under the power cap, profiles/r02/ab_nobc_selects.txt).
+// SF_PAIR_SELECTS=1 builds keep the selects (A/B; same results).
+#ifndef SF_PAIR_SELECTS
+#define SF_PAIR_SELECTS 0
+#endif
+#if SF_PAIR_SELECTS
 #define BCZ(c) (c)
+#else
+#define BCZ(c) false
 #endif
 
 struct Maps {
@@ -734,9 +739,9 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY(encode(&mp.x, L, v.f[xin], XH));
         SF_TRY(encode(&mp.dv, L, v.f[SF_DINV], CHS));
         SF_TRY(encode(&mp.rh, L, v.f[rhs], CHS));
-        SF_TRY(encode(&mp.bi, L, v.f[SF_BETA_I], CHS));
-        SF_TRY(encode(&mp.bj, L, v.f[SF_BETA_J], CHH));
-        SF_TRY(encode(&mp.bk, L, v.f[SF_BETA_K], CHS));
+        SF_TRY(encode(&mp.bi, L, v.f[SF_BI0], CHS));
+        SF_TRY(encode(&mp.bj, L, v.f[SF_BJ0], CHH));
+        SF_TRY(encode(&mp.bk, L, v.f[SF_BK0], CHS));
         Geo g{v.nx, v.ny, v.nz, v.z0, v.gnz, v.js, v.ks, 0};
         if (const char* ez = getenv("SF_DBG_ZMASK"))   // measurement only (see zplane)
             if (atoi(ez) > 0 && v.nz > atoi(ez)) g.zmask = atoi(ez);

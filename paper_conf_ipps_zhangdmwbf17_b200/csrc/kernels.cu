@@ -438,6 +438,31 @@ sf_status k_gsrb_colour(sf_level* L, int x, int rhs, double a, double b, int col
     return sf_check_launch("gsrb_colour");
 }
 
+// Boundary-zeroed face coefficients (SF_BI0/BJ0/BK0, sf_internal.h): a copy of
+// each beta array, ghosts and halo planes included, with the global Dirichlet
+// faces (i = 0, nx; j = 0, ny; global k = 0, gnz) set to 0.
+__global__ void beta0_kernel(PV v, long n) { pdl_wait();
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long e = (long)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += stride) {
+        const long kk = e / v.ks, r = e - kk * v.ks, jj = r / v.js;
+        const int i = (int)(r - jj * v.js) - SF_OX, j = (int)jj - SF_GY, gk = v.z0 + (int)kk - SF_GZ;
+        v.f[SF_BI0][e] = (i == 0 || i == v.nx) ? 0.0 : v.f[SF_BETA_I][e];
+        v.f[SF_BJ0][e] = (j == 0 || j == v.ny) ? 0.0 : v.f[SF_BETA_J][e];
+        v.f[SF_BK0][e] = (gk == 0 || gk == v.gnz) ? 0.0 : v.f[SF_BETA_K][e];
+    }
+}
+
+sf_status k_beta0(sf_level* L) {
+    for (int p = 0; p < L->nlocal; p++) {
+        PV v = sf_view(L, p);
+        const long n = (long)L->felems;
+        const int blocks = (int)std::min<long>((n + 255) / 256, 148L * 16);
+        sf_launch(beta0_kernel, blocks, 256, 0, L->stream, v, n);
+        SF_LAUNCHED();
+    }
+    return sf_check_launch("beta0");
+}
+
 sf_status k_dinv(sf_level* L, double a, double b) {
     double bh2 = b / (L->h * L->h);
     for (int p = 0; p < L->nlocal; p++) {

@@ -87,7 +87,7 @@ extern "C" sf_status sf_level_bytes_needed(int gnx, int gny, int gnz, const sf_c
     long js, ks;
     size_t fe;
     layout(gnx, gny, gnz / np, &js, &ks, &fe);
-    *bytes = (size_t)nl * SF_NFIELDS * field_bytes_aligned(fe) + SF_SCRATCH_BYTES;
+    *bytes = (size_t)nl * SF_NF_ALL * field_bytes_aligned(fe) + SF_SCRATCH_BYTES;
     return SF_OK;
 }
 
@@ -134,7 +134,7 @@ extern "C" sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, 
         SfPart& P = L->parts[q];
         P.index = L->first + q;
         P.z0 = P.index * L->lnz;
-        for (int f = 0; f < SF_NFIELDS; f++) {
+        for (int f = 0; f < SF_NF_ALL; f++) {
             P.f[f] = (double*)p;
             p += fb;
         }
@@ -179,7 +179,7 @@ extern "C" sf_status sf_level_destroy(sf_level* L) {
 
 PV sf_view(const sf_level* L, int p) {
     PV v;
-    for (int f = 0; f < SF_NFIELDS; f++) v.f[f] = L->parts[p].f[f];
+    for (int f = 0; f < SF_NF_ALL; f++) v.f[f] = L->parts[p].f[f];
     v.nx = L->nx; v.ny = L->ny; v.nz = L->lnz;
     v.z0 = L->parts[p].z0; v.gnz = L->gnz;
     v.js = L->js; v.ks = L->ks;
@@ -272,6 +272,7 @@ extern "C" sf_status sf_rebuild_operator(sf_level* L, double a, double b) {
     // coefficient halos for the colour-fused smoother's redundant ring work
     for (int f : {SF_ALPHA, SF_BETA_I, SF_BETA_J, SF_BETA_K}) SF_TRY(sf_halo(L, f, 2));
     SF_TRY(k_dinv(L, a, b));
+    SF_TRY(k_beta0(L));   // boundary-zeroed faces of the colour-fused pair (halos included)
     return sf_halo(L, SF_DINV, 2);
 }
 

@@ -47,10 +47,21 @@ struct sf_comm {
     void* hostuser;
 };
 
+// Internal fields after the public ones (not addressable through the C ABI):
+// the face coefficients with every global Dirichlet face set to 0, read only by
+// the colour-fused pair.  With them a boundary neighbour's term beta_f * x_ghost
+// vanishes by itself (the ghost is finite: buffers are zeroed at creation), so
+// the pair needs no boundary selects; the face's -x(c) ghost term lives in
+// Dinv as before.  Rebuilt with Dinv by sf_rebuild_operator.
+#define SF_BI0 (SF_NFIELDS + 0)
+#define SF_BJ0 (SF_NFIELDS + 1)
+#define SF_BK0 (SF_NFIELDS + 2)
+#define SF_NF_ALL (SF_NFIELDS + 3)
+
 struct SfPart {
     int index;                 // global part index
     int z0;                    // global z of local plane 0
-    double* f[SF_NFIELDS];     // base of each field's allocation (plane -SF_GZ)
+    double* f[SF_NF_ALL];      // base of each field's allocation (plane -SF_GZ)
 };
 
 struct sf_level {
@@ -85,7 +96,7 @@ struct sf_level {
 // compile-time constants (a runtime index spills the struct to local memory);
 // fields chosen at run time are passed as separate pointers.
 struct PV {
-    double* f[SF_NFIELDS];
+    double* f[SF_NF_ALL];
     int nx, ny, nz;            // local interior dims
     int z0, gnz;               // global z offset / extent (Dirichlet faces at 0, gnz)
     long js, ks;
@@ -161,6 +172,7 @@ sf_status k_apply_op(sf_level* L, int out, int x, double a, double b);
 sf_status k_residual(sf_level* L, int res, int x, int rhs, double a, double b);
 sf_status k_gsrb_colour(sf_level* L, int x, int rhs, double a, double b, int colour);
 sf_status k_dinv(sf_level* L, double a, double b);
+sf_status k_beta0(sf_level* L);
 sf_status k_bc(sf_level* L, int field);
 sf_status k_restrict(sf_level* C, int cf, sf_level* F, int ff, int kind);
 sf_status k_interp(sf_level* F, int ff, double s, sf_level* C, int cf, int kind);
