@@ -180,9 +180,14 @@ sf_status sf_level_create(sf_level** out, int gnx, int gny, int gnz, double h,
 sf_status sf_level_destroy(sf_level* level);
 sf_status sf_level_upload(sf_level* level, int field, const double* host);
 sf_status sf_level_download(sf_level* level, int field, double* host);   /* syncs */
+/* Set every element of `field` (interior, ghosts and halo planes of every
+ * local part) to 0 on the device, enqueued on the level's stream -- e.g. the
+ * zero initial guess u = 0 of a V-cycle solve.
+ * SF_ERR_INVALID for a bad field id. */
+sf_status sf_level_zero(sf_level* level, int field);
 /* Borrowed device pointer of (local part `part`, field) and its strides in
  * doubles: element (i,j,k) of the part is dev[k*strides[2] + j*strides[1] + i]
- * for -2 <= j,k and -4 <= i (ghost/padding).  Valid until the next
+ * for -2 <= i,j,k (ghost/padding).  Valid until the next
  * sf_smooth_gsrb on that level (the fused smoother may swap U and TMP). */
 sf_status sf_level_field_ptr(sf_level* level, int part, int field, double** dev, long strides[3]);
 /* Fill ALPHA, BETA_* (and, if want_rhs, F with the manufactured right-hand

@@ -226,6 +226,12 @@ static sf_status copy3d(sf_level* L, int field, double* host, bool up) {
     return sf_copy_field(L, field, host, up, L->stream);
 }
 
+extern "C" sf_status sf_level_zero(sf_level* L, int field) {
+    if (!L) return sf_fail(SF_ERR_INVALID, "NULL level");
+    SF_TRY(check_field(field));
+    return k_zero(L, field);
+}
+
 extern "C" sf_status sf_level_upload(sf_level* L, int field, const double* host) {
     if (!L || !host) return sf_fail(SF_ERR_INVALID, "NULL argument");
     SF_TRY(check_field(field));

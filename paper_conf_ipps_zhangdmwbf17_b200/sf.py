@@ -38,7 +38,7 @@ EXPORTS = [
     "sf_mg_opts_default", "sf_last_error", "sf_version", "sf_comm_create_local",
     "sf_get_unique_id", "sf_comm_create_nccl", "sf_comm_destroy", "sf_comm_info",
     "sf_level_bytes_needed", "sf_level_create", "sf_level_destroy", "sf_level_upload",
-    "sf_level_download", "sf_level_field_ptr", "sf_init_problem", "sf_rebuild_operator",
+    "sf_level_download", "sf_level_zero", "sf_level_field_ptr", "sf_init_problem", "sf_rebuild_operator",
     "sf_apply_bc", "sf_apply_op", "sf_smooth_gsrb", "sf_residual", "sf_restrict",
     "sf_interpolate", "sf_norm", "sf_sync", "sf_mg_create", "sf_mg_num_levels", "sf_mg_level",
     "sf_vcycle", "sf_fcycle", "sf_solve", "sf_mg_destroy", "sf_launch_count", "sf_mg_plan",
@@ -121,6 +121,7 @@ def lib():
         "sf_level_destroy": (_i, [_vp]),
         "sf_level_upload": (_i, [_vp, _i, _vp]),
         "sf_level_download": (_i, [_vp, _i, _vp]),
+        "sf_level_zero": (_i, [_vp, _i]),
         "sf_level_field_ptr": (_i, [_vp, _i, _i, C.POINTER(_P), C.POINTER(C.c_long)]),
         "sf_init_problem": (_i, [_vp, _i, _d, _d, _i]),
         "sf_rebuild_operator": (_i, [_vp, _d, _d]),
@@ -287,6 +288,10 @@ def sf_level_destroy(level):
 
 def sf_level_upload(level, field, host):
     _check(lib().sf_level_upload(level, field, host))
+
+
+def sf_level_zero(level, field):
+    _check(lib().sf_level_zero(level, field))
 
 
 def sf_level_download(level, field, host):

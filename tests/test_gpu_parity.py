@@ -49,6 +49,13 @@ def test_upload_download_roundtrip(sf, shape):
     x = I.random_field(shape, 3)
     L.upload(sf.SF_U, x)
     assert np.array_equal(L.download(sf.SF_U), x)
+    # sf_level_zero clears one field, interior and ghosts (BC fill of zeros is zero)
+    sf.sf_apply_bc(L.handle, sf.SF_U)
+    sf.sf_level_zero(L.handle, sf.SF_U)
+    assert not L.download(sf.SF_U).any()
+    assert np.array_equal(L.download(sf.SF_BETA_I), coeffs[1])
+    with pytest.raises(sf.SfError):
+        sf.sf_level_zero(L.handle, 99)
 
 
 @pytest.mark.parametrize("shape", [(6, 5, 4), (16, 16, 16), (8, 8, 64)])
