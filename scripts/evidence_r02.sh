@@ -21,6 +21,9 @@ if [[ $what == all || $what == ncu ]]; then
      -f -o gpurun_out/ev/prof_gsrb_512 python scripts/prof_gsrb.py 512 > gpurun_out/ev/prof_gsrb_512.log 2>&1
   python scripts/ncu_summary.py gpurun_out/ev/prof_gsrb_512.ncu-rep > gpurun_out/ev/ncu_gsrb_pair_512.txt 2>&1
   python scripts/ncu_lines.py gpurun_out/ev/prof_gsrb_512.ncu-rep 0 25 >> gpurun_out/ev/ncu_gsrb_pair_512.txt 2>&1
+  timeout 900 ncu -k regex:gsrb_pair_tma --launch-skip 6 --launch-count 1 --set full --import-source on --clock-control none \
+     -f -o gpurun_out/ev/prof_gsrb_256 python scripts/prof_gsrb.py 256 > gpurun_out/ev/prof_gsrb_256.log 2>&1
+  python scripts/ncu_summary.py gpurun_out/ev/prof_gsrb_256.ncu-rep > gpurun_out/ev/ncu_gsrb_pair_256.txt 2>&1
 fi
 if [[ $what == all || $what == oracle ]]; then
   timeout 1200 python scripts/oracle_table.py > gpurun_out/ev/oracle_table.json 2> gpurun_out/ev/oracle_table.err; echo "oracle rc=$?"
@@ -28,6 +31,8 @@ fi
 if [[ $what == all || $what == probes ]]; then
   timeout 300 python scripts/e2e_phases.py > gpurun_out/ev/e2e_phases.txt 2>&1
   timeout 300 python scripts/pair_headroom.py 256 512 > gpurun_out/ev/pair_headroom.txt 2>&1
+  timeout 300 python scripts/pair_sustained.py 512 > gpurun_out/ev/pair_sustained.txt 2>&1
+  timeout 300 python scripts/pair_sustained.py 256 >> gpurun_out/ev/pair_sustained.txt 2>&1
   timeout 600 python scripts/coarse_ab.py > gpurun_out/ev/coarse_ab.txt 2>&1
   timeout 600 python scripts/solve_sizes.py > gpurun_out/ev/solve_sizes.txt 2>&1
 fi
