@@ -189,7 +189,7 @@ __device__ __forceinline__ double red_pair(const StepCtx& s, int xo_, int co_, i
     } else {
         xw = xp2.x; xe = s.Xk[xo_ + 2];
     }
-    const int gxr = gx + SEL;
+    [[maybe_unused]] const int gxr = gx + SEL;
     if (BCZ(gxr == 0)) xw = 0.0;
     if (BCZ(gxr == g.nx - 1)) xe = 0.0;
     const double xs = BCZ(gy == 0) ? 0.0 : s.Xk[col - W];
@@ -235,7 +235,7 @@ __device__ __forceinline__ double2 black_pair(const StepCtx& s, int xo_, int gx,
     } else {
         xw = rn_same; xe = s.Xm[xo_ + 2];
     }
-    const int gxb = gx + SEL;
+    [[maybe_unused]] const int gxb = gx + SEL;
     if (BCZ(gxb == 0)) xw = 0.0;
     if (BCZ(gxb == g.nx - 1)) xe = 0.0;
     const int col = xo_ + SEL;
@@ -423,20 +423,24 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         const int ep0 = tid, ep1 = tid + NT;   // x-box pairs of this thread
         // in-plane offsets of their coarse parents (fixed per item): only the
         // coarse plane (p >> 1) changes from step to step
-        auto e_inplane = [&](int pr) -> long {
+        // (32-bit offsets: a coarse part holds < 2^31 doubles; the step code
+        // then costs two integer ops per load instead of 64-bit address math)
+        auto e_inplane = [&](int pr) -> int {
             const int r = pr / (W / 2), c2 = pr - r * (W / 2);
             const int I = x0 / 2 - 1 + c2, J = y0 / 2 - 1 + (r >> 1);
-            return (long)(J + SF_GY) * cv.js + SF_OX + I;
+            return (J + SF_GY) * (int)cv.js + SF_OX + I;
         };
-        const long eo0 = INTERP ? e_inplane(ep0) : 0;
-        const long eo1 = (INTERP && ep1 < XPAIRS) ? e_inplane(ep1) : eo0;
+        const int eo0 = INTERP ? e_inplane(ep0) : 0;
+        const int eo1 = (INTERP && ep1 < XPAIRS) ? e_inplane(ep1) : eo0;
+        const double* ebase = cv.e + (long)(cv.zoff + SF_GZ) * cv.ks;   // coarse plane 0
+        const int cks = (int)cv.ks;
         auto load_e = [&](int p, double& e0, double& e1) {
-            const double* ep = cv.e + (long)((p >> 1) + cv.zoff + SF_GZ) * cv.ks;
-            e0 = __ldg(ep + eo0);
-            e1 = __ldg(ep + eo1);
+            const int o = (p >> 1) * cks;
+            e0 = __ldg(ebase + (o + eo0));
+            e1 = __ldg(ebase + (o + eo1));
         };
-        auto correct = [&](int p, double e0, double e1) {
-            double* X = Xs + md(p, NXS) * XSLOT;
+        auto correct_slot = [&](int slot, double e0, double e1) {
+            double* X = Xs + slot * XSLOT;
             double2 v = *(double2*)&X[2 * ep0];
             v.x = v.x + e0;
             v.y = v.y + e0;
@@ -448,9 +452,13 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 *(double2*)&X[2 * ep1] = u;
             }
         };
-        // parents of the next two planes to correct (loaded two steps ahead: the
-        // coarse field may come from DRAM, slower than one z step)
-        double ce0 = 0.0, ce1 = 0.0, cn0 = 0.0, cn1 = 0.0;
+        auto correct = [&](int p, double e0, double e1) { correct_slot(md(p, NXS), e0, e1); };
+        // parents of the plane a step corrects, loaded two steps ahead (the
+        // coarse field may come from DRAM, slower than one z step) into one of
+        // two register sets that alternate with the steps (A: steps z0-2, z0, ..;
+        // B: z0-1, z0+1, ..): each set is refilled right after its use, so no
+        // register copy waits on a load in flight
+        double eA0 = 0.0, eA1 = 0.0, eB0 = 0.0, eB1 = 0.0;
         if (INTERP) {
             mbar_wait(&mbar[(seq0 + 1) % NMB], ((seq0 + 1) / NMB) & 1);   // bundle z0-1: x(z0)
             for (int p = z0 - 2; p <= z0; p++) {
@@ -458,8 +466,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 load_e(p, e0, e1);
                 correct(p, e0, e1);
             }
-            if (z0 + 1 <= z1 + 1) load_e(z0 + 1, ce0, ce1);
-            if (z0 + 2 <= z1 + 1) load_e(z0 + 2, cn0, cn1);
+            if (z0 + 1 <= z1 + 1) load_e(z0 + 1, eA0, eA1);
+            if (z0 + 2 <= z1 + 1) load_e(z0 + 2, eB0, eB1);
             __syncthreads();
         }
 
@@ -468,7 +476,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         double2 pq0 = *(const double2*)&Xs[ix_0 * XSLOT + xoff];
         double2 pq1 = *(const double2*)&Xs[ix_p1 * XSLOT + xoff];
         double2 bkc = *(const double2*)&Ks[ik1 * CARR + coff];   // beta_k(t+1) at step t
-        auto step = [&](int t, double* stash) {
+        auto step = [&](int t, double* stash, double& ce0, double& ce1) {
             // --- wait for bundle t+1 (R(t+1) operands)
             const int q = t + 1;
             if (!INTERP && q <= z1) {
@@ -544,10 +552,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             if (INTERP && q + 1 <= z1) {
                 const unsigned sq = seq0 + 2 + (q + 1 - z0);
                 mbar_wait(&mbar[sq % NMB], (sq / NMB) & 1);
-                correct(t + 3, ce0, ce1);
-                ce0 = cn0;
-                ce1 = cn1;
-                if (t + 5 <= z1 + 1) load_e(t + 5, cn0, cn1);
+                correct_slot(ix_p2 + 1 == NXS ? 0 : ix_p2 + 1, ce0, ce1);   // x(t+3)
+                if (t + 5 <= z1 + 1) load_e(t + 5, ce0, ce1);                // this set's next plane
             }
             fence_proxy_async();
             __syncthreads();
@@ -561,8 +567,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         };
         // steps t = z0-2 .. z1; B(t-1) consumes the stash R(t-1) filled at step t-2
         for (int t = z0 - 2; t <= z1; t += 2) {
-            step(t, stA);
-            if (t + 1 <= z1) step(t + 1, stB);
+            step(t, stA, eA0, eA1);
+            if (t + 1 <= z1) step(t + 1, stB, eB0, eB1);
         }
         seq = seq0 + 2 + (z1 - z0) + 1;
         __syncthreads();  // all reads of this item's slots done before the next prologue
