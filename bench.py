@@ -318,6 +318,7 @@ def main():
     launches = sf.sf_launch_count(reset=True)
     live_pair_ms, live_pairs = sf.sf_level_pair_timing(L.handle, 0)
     live_var = sf.sf_level_pair_timing_variants(L.handle)
+    live_rrf = sf.sf_level_pair_timing_rrf(L.handle)
     t = max_over_ranks(e0.elapsed_time(e1) / 1e3)
     value = dof_local * world * args.steps / t
     ms_step = t / args.steps * 1e3
@@ -368,6 +369,12 @@ def main():
                     "live_per_variant": {k: {"ms": v[0], "pairs": v[1],
                                              "frac": (alg / (v[0] / 1e3) / 1e9 / pk) if v[0] else None}
                                          for k, v in live_var.items()},
+                    "live_pair_residual_restrict": {
+                        "ms": live_rrf[0], "launches": live_rrf[1],
+                        "what": "the last pre-smoothing pair fused with the delta-form "
+                                "residual + restriction (gsrb_rr.cu), in-kernel timed like the "
+                                "pairs; not in launch_ms (it replaces a pair AND the separate "
+                                "residual_restrict pass)"},
                     "share_of_step": live_pairs * live_pair_ms / (t * 1e3),
                     "isolated_plain_pair_ms": fine_pair,
                     "isolated_plain_pair_frac": (alg / (fine_pair / 1e3) / 1e9 / pk

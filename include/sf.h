@@ -293,6 +293,10 @@ sf_status sf_level_pair_timing(sf_level* level, int op, double* mean_ms, long lo
  * pairs of the plain [0], input-residual check-fused RESID [1], output-residual
  * BRES [2] and P0-fused INTERP [3] (incl. INTERP + BRES) launches.  Host only. */
 sf_status sf_level_pair_timing_variants(const sf_level* level, double mean_ms[4], long long counts[4]);
+/* Same read-out for the V-cycle's fused pair + residual + restriction launches
+ * (the last pre-smoothing pair with the delta-form restricted residual,
+ * gsrb_rr.cu) on this level, which the pair mean above excludes.  Host only. */
+sf_status sf_level_pair_timing_rrf(const sf_level* level, double* mean_ms, long long* count);
 
 /* -------------------------------------------------------------- multigrid (A9)
  * sf_mg_create: builds the hierarchy below `finest` (which must hold ALPHA and

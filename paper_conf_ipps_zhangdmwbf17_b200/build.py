@@ -34,9 +34,8 @@ SOURCES = [("level.cu", "level.o", []), ("kernels.cu", "kernels.o", []),
            ("gsrb_fused.cu", "gsrb_fused_t32w4.o",
             ["-DSF_GSRB_TX=32", "-DSF_GSRB_PF=2", "-DSF_GSRB_NWARP=4", "-DSF_GSRB_MINB=3",
              "-DSF_GSRB_SUFFIX=_t32w4"]),
-           # the fused pair + residual + restriction (measured slower):
-           # stubs unless SF_BUILD_RR=1
-           ("gsrb_rr.cu", "gsrb_rr.o", ["-DSF_WITH_RR"] if os.environ.get("SF_BUILD_RR") == "1" else []),
+           # the fused pair + residual + restriction (delta form; host side + fix-up)
+           ("gsrb_rr.cu", "gsrb_rr.o", []),
            ("comm.cu", "comm.o", []), ("mg.cu", "mg.o", []), ("coarse.cu", "coarse.o", []),
            ("gsrb_twopair.cu", "gsrb_twopair.o", []),
            ("stencil.cu", "stencil.o", [])]

@@ -267,12 +267,23 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
 // RESID: max |rhs - A x| over the red cells of the INPUT (the black part of
 // that residual was reduced by the BRES pair that produced the input).
 // BRES: max |rhs - A x| over the black cells of the OUTPUT.  Both into *rmax.
-template <bool RESID, bool INTERP, bool BRES>
+// RRF (pair + residual + restriction, gsrb_rr.cu; single-part levels, even
+// z-chunks): the residual of the pair's output in delta form.  A red cell's
+// residual vanished at its own update (lambda = 1/diag(A)) and the black sweep
+// then changed only its six black neighbours, so r(c) = b h^-2 sum_f beta_f
+// delta(n_f) with delta = x_new - x_old of a black cell; a black cell's own
+// residual vanishes likewise (both up to rounding).  Each black cell scatters
+// beta_f * b h^-2 * delta over its faces: three into its own 2x2x2 block, one
+// per axis into the neighbouring block; a thread accumulates its pair column's
+// two planes in registers and writes six partials per coarse cell, each array
+// entry with exactly one writer (SfRRF); the fix-up pass sums them (x 1/8).
+template <bool RESID, bool INTERP, bool BRES, bool RRF = false>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
                      double bh2, int depth, int ntx, int ntiles, int nitems, double* rmax,
                      CoarseView cv, int c0, int cstride, unsigned long long* ts, int bd,
-                     int nch, int tcount, int zero_rmax, int early) {
+                     int nch, int tcount, int zero_rmax, int early, const __grid_constant__ SfRRF rv) {
+    static_assert(!(RRF && (RESID || INTERP || BRES)), "RRF is a plain pair");
     // early: the launch before this one triggered early and wrote nothing this
     // pair reads but the P0 source -- the first item's TMA prologue is issued
     // before griddepcontrol.wait (it overlaps that launch)
@@ -472,6 +483,8 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
 
         double rn0 = 0.0, rn1 = 0.0, rn2 = 0.0;   // red-new of planes t, t-1, t-2 at step t
+        // RRF partials of the thread's pair column for the current coarse plane
+        double rP = 0.0, rY = 0.0, rXW = 0.0, rXE = 0.0, rZB = 0.0, rZT = 0.0;
         // own pair of planes t and t+1 at step t (INTERP: after their correction)
         double2 pq0 = *(const double2*)&Xs[ix_0 * XSLOT + xoff];
         double2 pq1 = *(const double2*)&Xs[ix_p1 * XSLOT + xoff];
@@ -515,6 +528,38 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
             } else {
                 if (rin) rn = red_pair<1, RESID>(s, xoff, coff, hl, gxa, gy, g, zlo, zhi, bh2, nb, rres, pq0, pq1, pn, bkc, bkn);
                 if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
+            }
+            if (RRF && bin) {   // delta-form residual + restriction partials (see the kernel head)
+                const int bs = 1 - sel;                        // black cell's position in the pair
+                const double bnew = bs ? o.y : o.x;
+                const double bold = sb.Xm[xoff + bs];          // still the input value
+                const double u = __dmul_rn(bh2, bnew - bold);
+                const int p = t - 1;                           // its plane (single part: global)
+                const bool pe = (p & 1) == 0, ye = (gy & 1) == 0;
+                // stash: w, e, s, n, b, t faces of this black cell (boundary-zeroed betas)
+                double own = __dmul_rn(bs ? stash[0] : stash[1], u);
+                own = __fma_rn(ye ? stash[3] : stash[2], u, own);
+                own = __fma_rn(pe ? stash[5] : stash[4], u, own);
+                const double xo2 = __dmul_rn(bs ? stash[1] : stash[0], u);
+                const double yo2 = __dmul_rn(ye ? stash[2] : stash[3], u);
+                const double zo2 = __dmul_rn(pe ? stash[4] : stash[5], u);
+                if (bs) rXE = xo2; else rXW = xo2;
+                if (pe) {
+                    rP = own; rY = yo2; rZB = zo2;
+                } else {
+                    rP = rP + own; rY = rY + yo2; rZT = zo2;
+                    const int I = gxa >> 1, J = gy >> 1, K = p >> 1, rp = gy & 1;
+                    auto at = [&](int i, int j, int k) {
+                        return (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
+                    };
+                    (rp ? rv.a[1] : rv.a[0])[at(I, J, K)] = rP;
+                    if (I > 0) (rp ? rv.a[3] : rv.a[2])[at(I - 1, J, K)] = rXW;
+                    if (I + 1 < rv.ncx) (rp ? rv.a[5] : rv.a[4])[at(I + 1, J, K)] = rXE;
+                    if (!rp && J > 0) rv.a[6][at(I, J - 1, K)] = rY;
+                    if (rp && J + 1 < rv.ncy) rv.a[7][at(I, J + 1, K)] = rY;
+                    if (K > 0) (rp ? rv.a[9] : rv.a[8])[at(I, J, K - 1)] = rZB;
+                    if (K + 1 < rv.ncz) (rp ? rv.a[11] : rv.a[10])[at(I, J, K + 1)] = rZT;
+                }
             }
             if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
                 const unsigned long long m2 = abits(rres);
@@ -579,10 +624,12 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         if (atomicAdd(&ts[3], 1ull) == gridDim.x - 1) {   // every CTA has stamped
             __threadfence();
             const unsigned long long t0 = atomicAdd(&ts[1], 0ull), t1 = atomicAdd(&ts[2], 0ull);
-            ts[5] += t1 - t0;
-            ts[4] += tcount;   // a split pair (interior + boundary launch) counts once
-            // per variant: 0 plain, 1 RESID, 2 BRES, 3 INTERP (with or without BRES)
-            constexpr int var = INTERP ? 3 : RESID ? 1 : BRES ? 2 : 0;
+            if (!RRF) {   // the pair roofline covers the four pair variants
+                ts[5] += t1 - t0;
+                ts[4] += tcount;   // a split pair (interior + boundary launch) counts once
+            }
+            // per variant: 0 plain, 1 RESID, 2 BRES, 3 INTERP (with or without BRES), 4 RRF
+            constexpr int var = RRF ? 4 : INTERP ? 3 : RESID ? 1 : BRES ? 2 : 0;
             ts[6 + 2 * var] += tcount;
             ts[7 + 2 * var] += t1 - t0;
             ts[1] = ~0ull;
@@ -651,12 +698,12 @@ bool SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(const sf_level* L) {
 
 static __global__ void zero_bits(double* p) { pdl_wait(); *p = 0.0; }
 
-template <bool R, bool I, bool B>
+template <bool R, bool I, bool B, bool F = false>
 static sf_status set_attrs() {
-    SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B>,
+    SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B, F>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM));
     if (MINB > 1)   // room for MINB CTAs per SM
-        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B>,
+        SF_CUDA(cudaFuncSetAttribute(gsrb_pair_tma_kernel<R, I, B, F>,
                                      cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     return SF_OK;
 }
@@ -672,7 +719,9 @@ static sf_status set_attrs() {
 // 3 chunks per part.
 sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
                                                     double b, double* rmax, sf_level* C, int cf,
-                                                    int phase, int reserve, int rmode) {
+                                                    int phase, int reserve, int rmode, const SfRRF* rrf) {
+    if (rrf && (phase != 0 || C || rmode != SF_RM_NONE || L->nlocal != 1 || L->nparts != 1 || (L->lnz & 1)))
+        return sf_fail(SF_ERR_INVALID, "RRF pair: single-part level, even nz, plain pair only");
     if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
     if (rmode != SF_RM_NONE && !rmax) return sf_fail(SF_ERR_INVALID, "residual mode needs a scalar");
     if (rmode == SF_RM_INPUT_RED && C) return sf_fail(SF_ERR_INVALID, "input residual with P0 fusion");
@@ -684,6 +733,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         SF_TRY((set_attrs<false, true, false>()));
         SF_TRY((set_attrs<false, false, true>()));
         SF_TRY((set_attrs<false, true, true>()));
+        SF_TRY((set_attrs<false, false, false, true>()));
         int dev;
         SF_CUDA(cudaGetDevice(&dev));
         SF_CUDA(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
@@ -733,6 +783,8 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         }
         if (ed && atoi(ed) > 0) best_d = std::min(P, atoi(ed));
     }
+    // RRF: every item holds whole coarse planes (even chunk depth)
+    if (rrf && (best_d & 1)) best_d = std::min(L->lnz, best_d + 1);
     const int depth = best_d;
     const int nch = phase ? 2 + (L->lnz - 2 * bd + depth - 1) / depth : (L->lnz + depth - 1) / depth;
     const int c0 = phase == 1 ? 1 : 0;
@@ -768,11 +820,13 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
         const int zr = rmode == SF_RM_ZERO && p == 0 && phase != 2;
         const bool bres = rmode == SF_RM_OUTPUT_BLACK || rmode == SF_RM_OUTPUT_BLACK_ZEROED;
         double* xo = v.f[xout];
-#define SF_LAUNCH_PAIR(R, I, B)                                                                     \
-    sf_launch(gsrb_pair_tma_kernel<R, I, B>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
+        const SfRRF rv = rrf ? *rrf : SfRRF{};
+#define SF_LAUNCH_PAIR(R, I, B, ...)                                                                \
+    sf_launch(gsrb_pair_tma_kernel<R, I, B, ##__VA_ARGS__>, grid, NT, SMEM, L->stream, mp, g, xo, a, bh2, depth, ntx, tiles, \
                                                                 items, rmax, cvw, c0, cstride, \
-              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1, zr, early)
-        if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
+              (unsigned long long*)(L->dscratch + SF_TS_OFF), bd, nch, phase == 1 ? 0 : 1, zr, early, rv)
+        if (rrf) SF_LAUNCH_PAIR(false, false, false, true);
+        else if (rmode == SF_RM_INPUT_RED) SF_LAUNCH_PAIR(true, false, false);
         else if (bres && C) SF_LAUNCH_PAIR(false, true, true);
         else if (bres) SF_LAUNCH_PAIR(false, false, true);
         else if (C) SF_LAUNCH_PAIR(false, true, false);

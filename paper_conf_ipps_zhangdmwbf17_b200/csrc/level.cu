@@ -171,6 +171,7 @@ extern "C" sf_status sf_level_destroy(sf_level* L) {
     if (L->ev_fork) cudaEventDestroy(L->ev_fork);
     if (L->ev_join) cudaEventDestroy(L->ev_join);
     sf_ipc_close(L);
+    if (L->rrf_buf) cudaFree(L->rrf_buf);
     if (L->owns) cudaFree(L->buf);
     cudaFreeHost(L->hscratch);
     delete L;
@@ -582,13 +583,13 @@ extern "C" sf_status sf_level_pair_timing(sf_level* L, int op, double* mean_ms, 
     if (!L || (op != 0 && op != 1)) return sf_fail(SF_ERR_INVALID, "NULL level or bad op");
     unsigned long long* ts = (unsigned long long*)(L->dscratch + SF_TS_OFF);
     if (op == 1) {
-        static const unsigned long long arm[14] = {1ull, ~0ull, 0ull, 0ull, 0ull, 0ull, 0ull,
-                                                   0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull};
+        static const unsigned long long arm[16] = {1ull, ~0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull,
+                                                   0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull, 0ull};
         SF_CUDA(cudaMemcpyAsync(ts, arm, sizeof(arm), cudaMemcpyHostToDevice, L->stream));
         SF_TRY(sf_stream_sync(L));
         return SF_OK;
     }
-    unsigned long long h[14];
+    unsigned long long h[16];
     SF_CUDA(cudaMemcpyAsync(h, ts, sizeof(h), cudaMemcpyDeviceToHost, L->stream));
     SF_TRY(sf_stream_sync(L));
     static const unsigned long long off = 0ull;
@@ -596,7 +597,14 @@ extern "C" sf_status sf_level_pair_timing(sf_level* L, int op, double* mean_ms, 
     SF_TRY(sf_stream_sync(L));
     if (count) *count = (long long)h[4];
     if (mean_ms) *mean_ms = h[4] ? (double)h[5] / (double)h[4] * 1e-6 : 0.0;
-    for (int v = 0; v < 4; v++) L->ts_var[v][0] = (double)h[6 + 2 * v], L->ts_var[v][1] = (double)h[7 + 2 * v];
+    for (int v = 0; v < 5; v++) L->ts_var[v][0] = (double)h[6 + 2 * v], L->ts_var[v][1] = (double)h[7 + 2 * v];
+    return SF_OK;
+}
+
+extern "C" sf_status sf_level_pair_timing_rrf(const sf_level* L, double* mean_ms, long long* count) {
+    if (!L || !mean_ms || !count) return sf_fail(SF_ERR_INVALID, "NULL argument");
+    *count = (long long)L->ts_var[4][0];
+    *mean_ms = *count ? L->ts_var[4][1] / L->ts_var[4][0] * 1e-6 : 0.0;
     return SF_OK;
 }
 

@@ -290,6 +290,11 @@ extern "C" sf_status sf_mg_create(sf_mg** out, sf_level* fine, double a, double 
         if (e != cudaSuccess) s = sf_fail(SF_ERR_CUDA, "mg setup: %s", cudaGetErrorString(e));
     }
     if (s == SF_OK) m->coarse_l0 = plan_coarse(m);
+    // partial arrays of the fused pair + residual + restriction, allocated here
+    // (outside any graph capture) for every level pair that will use it
+    for (size_t l = 0; s == SF_OK && l + 1 < m->lv.size(); l++)
+        if ((m->coarse_l0 < 1 || (int)l < m->coarse_l0) && gsrb_rr_supported(m->lv[l], m->lv[l + 1]))
+            s = sf_rrf_prepare(m->lv[l], m->lv[l + 1]);
     if (s != SF_OK) {
         sf_mg_destroy(m);
         return s;

@@ -83,7 +83,10 @@ struct sf_level {
     unsigned long long* dsync; // P2P sync block (inside buf: peers reach it through IPC)
     double* hscratch;          // pinned, mapped host scalars
     double* hscratch_dev;      // their device alias
-    double ts_var[4][2] = {};  // last sf_level_pair_timing read-out per variant: launches, ns
+    double ts_var[5][2] = {};  // last sf_level_pair_timing read-out per variant: launches, ns
+                               // (plain, RESID, BRES, INTERP, pair + residual + restriction)
+    double* rrf_buf = nullptr; // SfRRF partial arrays for the coarse level below (gsrb_rr.cu)
+    size_t rrf_felems = 0;
     // the next fused pair may start under the launch before it (that launch
     // triggers early and writes nothing the pair reads except the P0 source;
     // set by the V-cycle, consumed by the pair launch)
@@ -204,20 +207,31 @@ sf_status sf_chebyshev_impl(sf_level* L, int x, int rhs, double a, double b, int
 sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, bool start,
                              double* out);
 
+// Restriction partials of the pair + residual + restriction (gsrb_rr.cu): twelve
+// coarse-shaped arrays (coarse layout, allocation bases), each entry written by
+// exactly one thread of the fused pair's RRF launch; the fix-up pass sums them
+// into the coarse rhs.  Order: P (own block) even/odd fine row, XW, XE (from the
+// west / east neighbour block) even/odd, YS, YN (from the south / north block),
+// ZB, ZT (from the block above / below) even/odd.
+struct SfRRF {
+    double* a[12];
+    int cjs, cks, ncx, ncy, ncz;
+};
+
 // fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
 bool gsrb_fused_supported_t32(const sf_level* L);
 bool gsrb_fused_supported_t64(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0);
+                                int rmode = 0, const SfRRF* rrf = nullptr);
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0);
+                                int rmode = 0, const SfRRF* rrf = nullptr);
 // 32x8 tiles, 4 warps, 3 CTAs per SM (three independent z-step chains per SM)
 bool gsrb_fused_supported_t32w4(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32w4(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                   double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0);
+                                int rmode = 0, const SfRRF* rrf = nullptr);
 bool gsrb_fused_supported(const sf_level* L);
 // rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax;
 // C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)
@@ -241,6 +255,8 @@ sf_status k_gsrb_twopair(sf_level* L, int xin, int xout, int rhs, double a, doub
 bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
                          int cf);
+// allocate the fine level's RRF partial arrays for coarse level C (before any capture)
+sf_status sf_rrf_prepare(sf_level* F, const sf_level* C);
 
 // coarse-level V-cycle in one thread-block-cluster launch, iterates in registers and
 // shared memory (coarse.cu)

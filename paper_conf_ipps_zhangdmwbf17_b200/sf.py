@@ -47,7 +47,7 @@ EXPORTS = [
     "sf_stencil_plan", "sf_stencil_phases", "sf_stencil_destroy", "sf_solve_stream",
     "sf_comm_create_p2p", "sf_smooth_residual_restrict", "sf_level_pair_timing",
     "sf_interpolate_smooth", "sf_comm_check", "sf_solve_stream_stats",
-    "sf_level_pair_timing_variants",
+    "sf_level_pair_timing_variants", "sf_level_pair_timing_rrf",
 ]
 
 
@@ -133,6 +133,7 @@ def lib():
         "sf_interpolate_smooth": (_i, [_vp, _i, _i, _d, _d, _vp, _i]),
         "sf_comm_check": (_i, [_vp, _vp]),
         "sf_level_pair_timing_variants": (_i, [_vp, C.POINTER(C.c_double), C.POINTER(C.c_longlong)]),
+        "sf_level_pair_timing_rrf": (_i, [_vp, C.POINTER(C.c_double), C.POINTER(C.c_longlong)]),
         "sf_solve_stream_stats": (_i, [_vp, C.POINTER(C.c_double)]),
         "sf_apply_laplacian": (_i, [_vp, _i, _i]),
         "sf_jacobi": (_i, [_vp, _i, _i, _i, _d]),
@@ -376,6 +377,14 @@ def sf_norm(level, field, kind=SF_NORM_MAX):
 
 def sf_sync(level):
     _check(lib().sf_sync(level))
+
+
+def sf_level_pair_timing_rrf(level):
+    """(mean ms, launches) of the fused pair + residual + restriction since the
+    last sf_level_pair_timing(op 0) read-out."""
+    ms, n = C.c_double(), C.c_longlong()
+    _check(lib().sf_level_pair_timing_rrf(level, C.byref(ms), C.byref(n)))
+    return ms.value, n.value
 
 
 def sf_level_pair_timing(level, op):

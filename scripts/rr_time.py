@@ -1,4 +1,4 @@
-"""Time the fused pair+residual+restriction (gsrb_rr) against the plain fused
+"""Time the fused pair + delta-form residual + restriction (gsrb_rr.cu) against the plain fused
 pair, and a V-cycle with and without it.   python scripts/rr_time.py [n ...]"""
 import os
 import sys
@@ -29,14 +29,14 @@ for n in [int(v) for v in sys.argv[1:]] or [256, 512]:
     s = L.stream
     reps = 20 if n <= 256 else 10
     t_pair = timed(s, lambda: sf.sf_smooth_gsrb(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, 1, sf.SF_SMOOTH_FUSED), reps)
-    os.environ["SF_RR"] = "1"
+    os.environ["SF_RRF_CELLS"] = "0"
     t_rr = timed(s, lambda: sf.sf_smooth_residual_restrict(L.handle, sf.SF_U, sf.SF_F, 1.0, 1.0, C.handle, sf.SF_F), reps)
     print(f"n={n} pair {t_pair:.4f} ms  pair+res+restrict {t_rr:.4f} ms  extra {t_rr - t_pair:.4f} ms "
           f"(alg 64 B/cell: pair {64 * n**3 / t_pair / 1e6:.0f} GB/s)")
     del C, L
     torch.cuda.empty_cache()
     for off in ("1", ""):
-        os.environ["SF_RR"] = "0" if off else "1"
+        os.environ["SF_RRF"] = "0" if off else "1"
         L = sf.Level(n, n, n, 1.0 / n)
         sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
         M = sf.MG(L, 1.0, 1.0)
@@ -44,4 +44,4 @@ for n in [int(v) for v in sys.argv[1:]] or [256, 512]:
         print(f"n={n} V-cycle ({'separate residual_restrict' if off else 'fused rr'}): {t_v:.3f} ms")
         del M, L
         torch.cuda.empty_cache()
-os.environ.pop("SF_RR", None)
+os.environ.pop("SF_RRF", None); os.environ.pop("SF_RRF_CELLS", None)

@@ -24,7 +24,7 @@ for n, parts in ((32, 1), (64, 1), (64, 2)):
         comm.close()
 
 # halo exchange beside the interior chunks (2 parts x 24 planes), the pair +
-# residual + restriction kernel (SF_RR=1) and the 32x16 build (SF_GSRB_W4=0)
+# residual + restriction (delta form, SF_RRF_CELLS=0 forces it) and the 32x16 build (SF_GSRB_W4=0)
 os.environ["SF_HALO_OVERLAP"] = "1"   # force the split (2-plane boundary chunks)
 comm = sf.Comm.local(2)
 L = sf.Level(64, 32, 48, 1.0 / 64, comm=comm)
@@ -35,7 +35,7 @@ sf.sf_sync(L.handle)
 print("ok overlap", flush=True)
 L.close()
 comm.close()
-os.environ["SF_RR"] = "1"
+os.environ["SF_RRF_CELLS"] = "0"
 F = sf.Level(64, 32, 12, 1.0 / 64)
 C = sf.Level(32, 16, 6, 2.0 / 64)
 sf.sf_init_problem(F.handle, 1, 1.0, 1.0, 1)
@@ -46,7 +46,7 @@ print("ok rr", flush=True)
 F.close(); C.close()
 
 # graphs on: the device-resident solve loop (WHILE node) and PDL launches
-os.environ.pop("SF_RR", None)
+os.environ.pop("SF_RRF_CELLS", None)
 L = sf.Level(32, 32, 32, 1.0 / 32)
 sf.sf_init_problem(L.handle, 1, 1.0, 1.0, 1)
 M = sf.MG(L, 1.0, 1.0)

@@ -339,15 +339,17 @@ RR_SHAPES = [(4, 16, 32), (10, 32, 64), (16, 48, 96), (34, 16, 32), (64, 64, 64)
 @pytest.mark.parametrize("depth", [None, "2", "6"])
 @pytest.mark.parametrize("ab", [(1.0, 1.0), (2.5, 0.75)])
 def test_smooth_residual_restrict(sf, oracle, shape, depth, ab, monkeypatch):
-    """A5+A6+A7 fused (sf_smooth_residual_restrict): the smoothed x equals the
-    oracle's RB pair (1e-12) and bit-for-bit the plain fused pair; the coarse
-    rhs equals R_cell(rhs - A x) of the oracle (1e-12).  Chunk depths 2 and 6
-    put item boundaries (extended z ranges, recomputed planes) inside the grid."""
+    """A5+A6+A7 fused (sf_smooth_residual_restrict, the pair's delta-form
+    residual + restriction, gsrb_rr.cu, forced on every size): the smoothed x
+    equals the oracle's RB pair (1e-12) and bit-for-bit the plain fused pair; the
+    coarse rhs equals R_cell(rhs - A x) of the oracle (1e-12 rel-L2, 1e-11
+    max-abs relative).  Chunk depths 2 and 6 put item (z-chunk) boundaries inside
+    the grid, where the partials cross between items."""
     nz, ny, nx = shape
     a, b = ab
-    monkeypatch.setenv("SF_RR", "1")
+    monkeypatch.setenv("SF_RRF_CELLS", "0")
     if depth:
-        monkeypatch.setenv("SF_RR_DEPTH", depth)
+        monkeypatch.setenv("SF_GSRB_DEPTH", depth)
     h = I.level_h(nx, ny, nz)
     coeffs = I.hpgmg_coeffs(nx, ny, nz) if nx >= 64 else I.random_coeffs(nx, ny, nz, 5)
     L = make_level(sf, shape, coeffs)
@@ -359,14 +361,19 @@ def test_smooth_residual_restrict(sf, oracle, shape, depth, ab, monkeypatch):
         sf.sf_rebuild_operator(lv.handle, a, b)
         lv.upload(sf.SF_U, x)
         lv.upload(sf.SF_F, f)
+    sf.sf_level_pair_timing(L.handle, 1)
     sf.sf_smooth_residual_restrict(L.handle, sf.SF_U, sf.SF_F, a, b, C.handle, sf.SF_F)
+    sf.sf_level_pair_timing(L.handle, 0)
+    assert sf.sf_level_pair_timing_rrf(L.handle)[1] == 1   # the fused path ran
     sf.sf_smooth_gsrb(L2.handle, sf.SF_U, sf.SF_F, a, b, 1, sf.SF_SMOOTH_FUSED)
     got = L.download(sf.SF_U)
     assert np.array_equal(got, L2.download(sf.SF_U))
     xs = P.smooth(x, f, 1, dinv=P.dinv())
     assert rel(got, xs) < TOL
     exp = oracle.restrict_cell(P.residual(xs, f))
-    assert rel(C.download(sf.SF_F), exp) < TOL
+    gotc = C.download(sf.SF_F)
+    assert rel(gotc, exp) < TOL
+    assert np.abs(gotc - exp).max() <= 10 * TOL * np.abs(exp).max()
 
 
 def test_smooth_residual_restrict_general(sf, oracle):
@@ -394,11 +401,13 @@ def test_smooth_residual_restrict_general(sf, oracle):
 
 @pytest.mark.parametrize("n", [32, 64])
 def test_vcycle_rr_matches_separate_residual(sf, monkeypatch, n):
-    """The V-cycle with the fused last pre-smoothing pair (gsrb_rr) and with the
+    """The V-cycle with the fused last pre-smoothing pair (the delta-form
+    residual + restriction, gsrb_rr.cu, forced on every level) and with the
     separate residual_restrict pass agree to rounding (1e-13)."""
     out = []
+    monkeypatch.setenv("SF_RRF_CELLS", "0")
     for on in ("1", "0"):
-        monkeypatch.setenv("SF_RR", on)
+        monkeypatch.setenv("SF_RRF", on)
         h = 1.0 / n
         coeffs = I.hpgmg_coeffs(n, n, n)
         L = make_level(sf, (n, n, n), coeffs, h=h)
