@@ -1,11 +1,13 @@
 """The headline configuration cell by cell: the 512^3 HPGMG-FV solve (BASELINE
 C5: F-cycle + V-cycles to 1e-10 with the production kernel builds -- 32x8
-colour-fused pairs, the 32x16 P0-fused pair, the z-streamed residual +
-restriction, the coarse cluster V-cycle) against a complete oracle solve of the
+colour-fused pairs, the 32x16 P0-fused pair, the fused pair + delta-form
+residual + restriction on the levels >= 128^3, the z-streamed residual +
+restriction below, the coarse cluster V-cycle) against a complete oracle solve of the
 same problem.  The oracle runs in a subprocess with its OpenMP build on every
 host core (the library build is per process; GSRB colour sweeps and max-norms
 are independent of the thread count, so it computes what the single-thread
-build computes).  Same cycle count, residual history within 1e-6, u within
+build computes).  Same cycle count, residual history within 1e-6 relative plus
+the residual's absolute rounding floor (1e-12), u within
 1e-10 (rel-L2) and 1e-9 of max|u| cell by cell."""
 import os
 import subprocess
@@ -70,7 +72,9 @@ def test_512_solve_matches_oracle(tmp_path):
     M.close()
     L.close()
     assert cyc == len(hist_o)
-    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-14)
+    # atol: the max-norm residual's absolute rounding floor at 512^3 (~1e-13,
+    # DESIGN.md section 13, R-19); u itself is compared at 1e-10 below
+    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-12)
     rel = np.linalg.norm((u - u_o).ravel()) / np.linalg.norm(u_o.ravel())
     print(f"512^3 solve vs oracle: cycles {cyc} / {len(hist_o)}, final relres {hist[-1]:.3e} / "
           f"{hist_o[-1]:.3e}, u rel-L2 {rel:.3e}, max-abs {np.abs(u - u_o).max():.3e} "

@@ -147,6 +147,54 @@ def test_vcycle_fcycle_headline_paths_vs_oracle(sf, oracle, shape, monkeypatch):
     assert np.array_equal(res["default"][1], res["headline"][1])
 
 
+@pytest.mark.parametrize("shape", [(64, 64, 64), (128, 128, 128), (32, 64, 128)])
+def test_vcycle_fcycle_rrf_vs_oracle(sf, oracle, shape, monkeypatch):
+    """V- and F-cycles with the fused pair + delta-form residual + restriction
+    (gsrb_rr.cu) forced on every level it supports (the 512^3 headline takes it
+    on the levels >= 128^3) against the oracle cell by cell: 1e-11 rel-L2,
+    1e-10 max-abs relative (the restricted residual rounds differently from
+    rhs - Ax, R-19)."""
+    monkeypatch.setenv("SF_RRF_CELLS", "0")
+    nz, ny, nx = shape
+    _, f = I.manufactured(nx, ny, nz, 1.0, 1.0)
+    L, M, O = _mg(sf, oracle, shape)
+    L.upload(sf.SF_F, f)
+    sf.sf_level_pair_timing(L.handle, 1)
+    M.fcycle()
+    uf = L.download(sf.SF_U)
+    M.vcycle(0)
+    uv = L.download(sf.SF_U)
+    sf.sf_level_pair_timing(L.handle, 0)
+    assert sf.sf_level_pair_timing_rrf(L.handle)[1] >= 2   # the fused path ran on the finest level
+    M.close()
+    L.close()
+    uo_f = O.fcycle(f)
+    uo_v = O.vcycle(uo_f, f)
+    assert rel(uf, uo_f) < 1e-11 and maxrel(uf, uo_f) < 1e-10
+    assert rel(uv, uo_v) < 1e-11 and maxrel(uv, uo_v) < 1e-10
+
+
+@pytest.mark.parametrize("fcycle", [False, True])
+def test_solve_rrf_vs_oracle(sf, oracle, fcycle, monkeypatch):
+    """The device-loop solve with the fused residual + restriction forced: same
+    cycle count as the oracle, history within 1e-6 relative plus the residual's
+    absolute rounding floor (1e-12 at 512^3, scaled by
+    h^-2), u to 1e-10."""
+    monkeypatch.setenv("SF_RRF_CELLS", "0")
+    shape = (64, 64, 64)
+    nz, ny, nx = shape
+    L, M, O = _mg(sf, oracle, shape)
+    _, f = I.manufactured(nx, ny, nz, 1.0, 1.0)
+    L.upload(sf.SF_F, f)
+    st, cyc, hist = M.solve(fcycle=fcycle, rtol=1e-10)
+    u_o, hist_o = O.solve(f, fcycle=fcycle, rtol=1e-10)
+    assert cyc == len(hist_o)
+    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-12 * (nx / 512) ** 2)
+    assert rel(L.download(sf.SF_U), u_o) < 1e-10
+    M.close()
+    L.close()
+
+
 @pytest.mark.parametrize("fcycle", [False, True])
 def test_solve_headline_paths_vs_oracle(sf, oracle, fcycle, monkeypatch):
     """The whole device-loop solve (as bench.py runs it) with the headline's
