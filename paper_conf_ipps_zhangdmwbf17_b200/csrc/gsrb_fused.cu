@@ -274,9 +274,12 @@ __device__ __forceinline__ double red_ring(const StepCtx& s, int xo_, int co_, i
 // delta(n_f) with delta = x_new - x_old of a black cell; a black cell's own
 // residual vanishes likewise (both up to rounding).  Each black cell scatters
 // beta_f * b h^-2 * delta over its faces: three into its own 2x2x2 block, one
-// per axis into the neighbouring block; a thread accumulates its pair column's
-// two planes in registers and writes six partials per coarse cell, each array
-// entry with exactly one writer (SfRRF); the fix-up pass sums them (x 1/8).
+// per axis into the neighbouring block.  x shares go to the next pair column by
+// a lane shuffle, z shares stay in the thread's registers (carried to the next /
+// previous coarse plane), so a thread writes two partials per coarse cell: its
+// block's (P) and the y share (other warps); only shares crossing a tile or
+// z-chunk edge go to the edge arrays.  Each array entry has exactly one writer
+// (SfRRF); the fix-up pass sums them in a fixed order (x 1/8).
 template <bool RESID, bool INTERP, bool BRES, bool RRF = false>
 __global__ void __launch_bounds__(NT, MINB)
 gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict__ xo, double a,
@@ -483,8 +486,10 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
 
         double rn0 = 0.0, rn1 = 0.0, rn2 = 0.0;   // red-new of planes t, t-1, t-2 at step t
-        // RRF partials of the thread's pair column for the current coarse plane
-        double rP = 0.0, rY = 0.0, rXW = 0.0, rXE = 0.0, rZB = 0.0, rZT = 0.0;
+        // RRF partials of the thread's pair column: the coarse plane being summed,
+        // the previous one (waiting for its share of the next plane), the next
+        // one's share carried from an odd plane, and the y share
+        double rAcc = 0.0, rPend = 0.0, rCarry = 0.0, rY = 0.0;
         // own pair of planes t and t+1 at step t (INTERP: after their correction)
         double2 pq0 = *(const double2*)&Xs[ix_0 * XSLOT + xoff];
         double2 pq1 = *(const double2*)&Xs[ix_p1 * XSLOT + xoff];
@@ -530,7 +535,7 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 if (bin) o = black_pair<0, BRES>(sb, xoff, gxa, gy, g, gkm, bh2, stash, bres, rn2, rn1, rn0);
             }
             if (RRF && bin) {   // delta-form residual + restriction partials (see the kernel head)
-                const int bs = 1 - sel;                        // black cell's position in the pair
+                const int bs = 1 - sel;                        // black cell's position in the pair (warp-uniform)
                 const double bnew = bs ? o.y : o.x;
                 const double bold = sb.Xm[xoff + bs];          // still the input value
                 const double u = __dmul_rn(bh2, bnew - bold);
@@ -543,22 +548,43 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 const double xo2 = __dmul_rn(bs ? stash[1] : stash[0], u);
                 const double yo2 = __dmul_rn(ye ? stash[2] : stash[3], u);
                 const double zo2 = __dmul_rn(pe ? stash[4] : stash[5], u);
-                if (bs) rXE = xo2; else rXW = xo2;
+                const int I = gxa >> 1, J = gy >> 1, K = p >> 1, rp = gy & 1;
+                auto at = [&](int i, int j, int k) {
+                    return (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
+                };
+                // x: the neighbouring pair column of this row is lane hl -+ 1 of the
+                // 16-lane row segment; across the tile edge -> edge array (XW / XE)
+                double xr = bs ? __shfl_up_sync(0xffffffffu, xo2, 1, PPR)
+                               : __shfl_down_sync(0xffffffffu, xo2, 1, PPR);
+                if (bs ? hl == 0 : hl == PPR - 1) xr = 0.0;
+                if (!bs && hl == 0 && I > 0) (rp ? rv.a[3] : rv.a[2])[at(I - 1, J, K)] = xo2;
+                if (bs && hl == PPR - 1 && I + 1 < rv.ncx) (rp ? rv.a[5] : rv.a[4])[at(I + 1, J, K)] = xo2;
+                const double c2 = own + xr;
                 if (pe) {
-                    rP = own; rY = yo2; rZB = zo2;
+                    // z: down into block K-1 -- the pending partial when K-1 is this
+                    // item's (written now, complete), else the ZB edge array
+                    if (p > z0) {
+                        rPend = rPend + zo2;
+                        (rp ? rv.a[1] : rv.a[0])[at(I, J, K - 1)] = rPend;
+                    } else if (K > 0) {
+                        (rp ? rv.a[9] : rv.a[8])[at(I, J, K - 1)] = zo2;
+                    }
+                    rAcc = c2 + rCarry;   // rCarry: block K's share of plane 2K-1 (0 at the item start)
+                    rCarry = 0.0;
+                    rY = yo2;
                 } else {
-                    rP = rP + own; rY = rY + yo2; rZT = zo2;
-                    const int I = gxa >> 1, J = gy >> 1, K = p >> 1, rp = gy & 1;
-                    auto at = [&](int i, int j, int k) {
-                        return (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
-                    };
-                    (rp ? rv.a[1] : rv.a[0])[at(I, J, K)] = rP;
-                    if (I > 0) (rp ? rv.a[3] : rv.a[2])[at(I - 1, J, K)] = rXW;
-                    if (I + 1 < rv.ncx) (rp ? rv.a[5] : rv.a[4])[at(I + 1, J, K)] = rXE;
+                    rAcc = rAcc + c2;
+                    rY = rY + yo2;
+                    // y: into the neighbouring row of blocks (other warps): YS / YN arrays
                     if (!rp && J > 0) rv.a[6][at(I, J - 1, K)] = rY;
                     if (rp && J + 1 < rv.ncy) rv.a[7][at(I, J + 1, K)] = rY;
-                    if (K > 0) (rp ? rv.a[9] : rv.a[8])[at(I, J, K - 1)] = rZB;
-                    if (K + 1 < rv.ncz) (rp ? rv.a[11] : rv.a[10])[at(I, J, K + 1)] = rZT;
+                    if (p + 1 < z1) {     // block K+1 is this item's: carry, K waits for its ZB share
+                        rCarry = zo2;
+                        rPend = rAcc;
+                    } else {              // last block of the item: ZT edge, partial now
+                        if (K + 1 < rv.ncz) (rp ? rv.a[11] : rv.a[10])[at(I, J, K + 1)] = zo2;
+                        (rp ? rv.a[1] : rv.a[0])[at(I, J, K)] = rAcc;
+                    }
                 }
             }
             if (RESID && rin && q >= z0 && q < z1) {   // this item's planes only
@@ -719,7 +745,7 @@ static sf_status set_attrs() {
 // 3 chunks per part.
 sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xout, int rhs, double a,
                                                     double b, double* rmax, sf_level* C, int cf,
-                                                    int phase, int reserve, int rmode, const SfRRF* rrf) {
+                                                    int phase, int reserve, int rmode, SfRRF* rrf) {
     if (rrf && (phase != 0 || C || rmode != SF_RM_NONE || L->nlocal != 1 || L->nparts != 1 || (L->lnz & 1)))
         return sf_fail(SF_ERR_INVALID, "RRF pair: single-part level, even nz, plain pair only");
     if (!SF_CAT(gsrb_fused_supported, SF_GSRB_SUFFIX)(L)) return sf_fail(SF_ERR_SHAPE, "fused GSRB needs nx%%%d==0, ny%%%d==0", TX, TY);
@@ -785,6 +811,7 @@ sf_status SF_CAT(k_gsrb_pair_fused, SF_GSRB_SUFFIX)(sf_level* L, int xin, int xo
     }
     // RRF: every item holds whole coarse planes (even chunk depth)
     if (rrf && (best_d & 1)) best_d = std::min(L->lnz, best_d + 1);
+    if (rrf) rrf->zdepth = best_d;   // the fix-up reads the z-edge arrays at chunk edges
     const int depth = best_d;
     const int nch = phase ? 2 + (L->lnz - 2 * bd + depth - 1) / depth : (L->lnz + depth - 1) / depth;
     const int c0 = phase == 1 ? 1 : 0;

@@ -20,12 +20,15 @@
 // a scatter of every black cell's b h^-2 beta_f delta over its six faces: three
 // land in its own 2x2x2 block, one per axis in the neighbouring block.  Each
 // thread of the pair accumulates its pair column's two planes of a block in
-// registers and writes six partials per coarse cell into twelve coarse-shaped
-// arrays (SfRRF, sf_internal.h), each entry with exactly one writer, so the
-// result does not depend on scheduling; the fix-up kernel below sums them in a
-// fixed order into the coarse rhs.  Extra work in the pair: one shared-memory
-// load (the black cell's old value), ~10 FP64 operations and six 8-byte stores
-// per 4 fine cells -- instead of a second 48 B/cell pass.
+// registers; x shares move to the next pair column by a lane shuffle and z
+// shares stay in the thread (carried to the next / previous coarse plane), so a
+// thread writes two partials per coarse cell (its block's and the y share for
+// the neighbouring block row), plus the shares that cross a tile or z-chunk
+// edge into edge arrays (SfRRF, sf_internal.h).  Each entry has at most one
+// writer, so the result does not depend on scheduling; the fix-up kernel below
+// sums them in a fixed order into the coarse rhs.  Extra work in the pair: one
+// shared-memory load (the black cell's old value), ~10 FP64 operations, a
+// shuffle and ~4 B of stores per fine cell -- instead of a 48 B/cell pass.
 //
 // Scope: single-part fine and coarse levels (the headline's 512^3 hierarchy;
 // slab-decomposed levels keep pair + residual_restrict), the 32x8 fused-pair
@@ -41,15 +44,21 @@ namespace {
 
 constexpr int NPART = 12;
 
-// coarse rhs = 1/8 of the twelve partials, summed in array order
+// coarse rhs = 1/8 of the partials, summed in array order; the edge arrays are
+// read only where the current launch wrote them (tile-edge columns: the 32x8
+// build's coarse tiles are 16 wide; z-chunk edge planes: zdepth / 2 per chunk)
 __global__ void rrf_fixup_kernel(double* __restrict__ out, SfRRF rv) {
     pdl_wait();
     const int i = blockIdx.x * blockDim.x + threadIdx.x, j = blockIdx.y, k = blockIdx.z;
     if (i >= rv.ncx) return;
     const long q = (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
-    double s = rv.a[0][q];
-#pragma unroll
-    for (int m = 1; m < NPART; m++) s = s + rv.a[m][q];
+    const int cd = rv.zdepth / 2;
+    double s = rv.a[0][q] + rv.a[1][q];
+    if ((i & 15) == 15 && i + 1 < rv.ncx) s = s + rv.a[2][q] + rv.a[3][q];
+    if ((i & 15) == 0 && i > 0) s = s + rv.a[4][q] + rv.a[5][q];
+    s = s + rv.a[6][q] + rv.a[7][q];
+    if (k % cd == cd - 1 && k + 1 < rv.ncz) s = s + rv.a[8][q] + rv.a[9][q];
+    if (k % cd == 0 && k > 0) s = s + rv.a[10][q] + rv.a[11][q];
     out[q] = 0.125 * s;
 }
 
@@ -102,6 +111,7 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
     rv.ncx = C->nx;
     rv.ncy = C->ny;
     rv.ncz = C->lnz;
+    rv.zdepth = 2;
     SF_TRY(k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, nullptr, nullptr, 0, 0, 0, SF_RM_NONE, &rv));
     PV c = sf_view(C, 0);
     sf_launch(rrf_fixup_kernel, dim3((C->nx + 127) / 128, C->ny, C->lnz), 128, 0, L->stream, c.f[cf], rv);

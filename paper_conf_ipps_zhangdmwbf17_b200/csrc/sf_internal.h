@@ -209,13 +209,15 @@ sf_status sf_lambda_max_impl(sf_level* L, int v, double a, double b, int iters, 
 
 // Restriction partials of the pair + residual + restriction (gsrb_rr.cu): twelve
 // coarse-shaped arrays (coarse layout, allocation bases), each entry written by
-// exactly one thread of the fused pair's RRF launch; the fix-up pass sums them
-// into the coarse rhs.  Order: P (own block) even/odd fine row, XW, XE (from the
-// west / east neighbour block) even/odd, YS, YN (from the south / north block),
-// ZB, ZT (from the block above / below) even/odd.
+// at most one thread of the fused pair's RRF launch; the fix-up pass sums them
+// into the coarse rhs.  Order: P (the block's own, x and z shares) even / odd
+// fine row; XW, XE (shares from the east / west tile's edge column) even / odd;
+// YS, YN (from the block row north / south); ZB, ZT (from the z-chunk above /
+// below, edge planes only) even / odd.  zdepth: the launch's z-chunk depth
+// (set by the pair launch; the fix-up reads the z edges there).
 struct SfRRF {
     double* a[12];
-    int cjs, cks, ncx, ncy, ncz;
+    int cjs, cks, ncx, ncy, ncz, zdepth;
 };
 
 // fused colour pair (gsrb_fused.cu, built as 32x16 "_t32" and 64x8 "_t64"; dispatch in level.cu)
@@ -223,15 +225,15 @@ bool gsrb_fused_supported_t32(const sf_level* L);
 bool gsrb_fused_supported_t64(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0, const SfRRF* rrf = nullptr);
+                                int rmode = 0, SfRRF* rrf = nullptr);
 sf_status k_gsrb_pair_fused_t64(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                 double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0, const SfRRF* rrf = nullptr);
+                                int rmode = 0, SfRRF* rrf = nullptr);
 // 32x8 tiles, 4 warps, 3 CTAs per SM (three independent z-step chains per SM)
 bool gsrb_fused_supported_t32w4(const sf_level* L);
 sf_status k_gsrb_pair_fused_t32w4(sf_level* L, int xin, int xout, int rhs, double a, double b,
                                   double* rmax, sf_level* C, int cf, int phase = 0, int reserve = 0,
-                                int rmode = 0, const SfRRF* rrf = nullptr);
+                                int rmode = 0, SfRRF* rrf = nullptr);
 bool gsrb_fused_supported(const sf_level* L);
 // rmax != NULL: the pair also reduces max|rhs - A x_in| of its input into *rmax;
 // C != NULL: the pair first applies x_in += P0(C.cf) (V-cycle interpolation)
