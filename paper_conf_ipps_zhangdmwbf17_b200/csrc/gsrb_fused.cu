@@ -99,6 +99,7 @@ constexpr int CSLOT = NCA * CARR;
 #endif
 constexpr int CHS = CHH - SF_TRIM_ROWS;
 constexpr int XBYTES = XH * W * 8, CBYTES = CHH * W * 8, CBYTES_S = CHS * W * 8;
+static_assert(XSLOT >= TY * PPR, "RRF y shares fit one x slot");
 constexpr int BUNDLE_BYTES = XBYTES + (NCA - 1) * CBYTES_S + CBYTES + CBYTES_S;
 constexpr size_t SMEM = sizeof(double) * (NXS * XSLOT + NCS * CSLOT + NKS * CARR) + 64;
 static_assert(MINB * (SMEM + 1024) <= 228 * 1024, "MINB CTAs per SM must fit in shared memory");
@@ -486,6 +487,12 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
         }
 
         double rn0 = 0.0, rn1 = 0.0, rn2 = 0.0;   // red-new of planes t, t-1, t-2 at step t
+        // RRF: y shares crossing to the neighbouring block row (other warps) go
+        // through the x slot of plane t-2 at an odd-plane step t: its last
+        // reader was B(t-2) at step t-1 and its TMA refill is issued after step
+        // t+1, when the shares have been read (no extra shared memory: three
+        // CTAs per SM stay resident)
+        int yslot = 0;
         // RRF partials of the thread's pair column: the coarse plane being summed,
         // the previous one (waiting for its share of the next plane), the next
         // one's share carried from an odd plane, and the y share
@@ -562,9 +569,12 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 const double c2 = own + xr;
                 if (pe) {
                     // z: down into block K-1 -- the pending partial when K-1 is this
-                    // item's (written now, complete), else the ZB edge array
+                    // item's (written now, complete), else the ZB edge array;
+                    // the y share of K-1 from the neighbouring row of the other
+                    // block row arrived in shared memory at the last step
                     if (p > z0) {
                         rPend = rPend + zo2;
+                        if (rp ? row + 1 < TY : row > 0) rPend = rPend + Xs[yslot * XSLOT + row * PPR + hl];
                         (rp ? rv.a[1] : rv.a[0])[at(I, J, K - 1)] = rPend;
                     } else if (K > 0) {
                         (rp ? rv.a[9] : rv.a[8])[at(I, J, K - 1)] = zo2;
@@ -575,9 +585,15 @@ gsrb_pair_tma_kernel(const __grid_constant__ Maps mp, Geo g, double* __restrict_
                 } else {
                     rAcc = rAcc + c2;
                     rY = rY + yo2;
-                    // y: into the neighbouring row of blocks (other warps): YS / YN arrays
-                    if (!rp && J > 0) rv.a[6][at(I, J - 1, K)] = rY;
-                    if (rp && J + 1 < rv.ncy) rv.a[7][at(I, J + 1, K)] = rY;
+                    // y: into the neighbouring row of the next block row (another
+                    // warp) through shared memory -- read there next step, before
+                    // its partial is written; across the tile edge, or on the
+                    // item's last block (no next step), into the YS / YN arrays
+                    const int trow = rp ? row + 1 : row - 1;
+                    yslot = ix_m2;
+                    if (p + 1 < z1 && trow >= 0 && trow < TY) Xs[ix_m2 * XSLOT + trow * PPR + hl] = rY;
+                    else if (!rp && J > 0) rv.a[6][at(I, J - 1, K)] = rY;
+                    else if (rp && J + 1 < rv.ncy) rv.a[7][at(I, J + 1, K)] = rY;
                     if (p + 1 < z1) {     // block K+1 is this item's: carry, K waits for its ZB share
                         rCarry = zo2;
                         rPend = rAcc;

@@ -53,10 +53,15 @@ __global__ void rrf_fixup_kernel(double* __restrict__ out, SfRRF rv) {
     if (i >= rv.ncx) return;
     const long q = (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
     const int cd = rv.zdepth / 2;
+    // last coarse plane of a z-chunk (the last chunk may be shorter): every y share
+    const bool klast = k % cd == cd - 1 || k == rv.ncz - 1;
     double s = rv.a[0][q] + rv.a[1][q];
     if ((i & 15) == 15 && i + 1 < rv.ncx) s = s + rv.a[2][q] + rv.a[3][q];
     if ((i & 15) == 0 && i > 0) s = s + rv.a[4][q] + rv.a[5][q];
-    s = s + rv.a[6][q] + rv.a[7][q];
+    // y shares through memory: the tile-edge block rows (coarse tiles are 4 rows
+    // high), and every row on a chunk's last coarse plane
+    if ((klast || (j & 3) == 3) && j + 1 < rv.ncy) s = s + rv.a[6][q];
+    if ((klast || (j & 3) == 0) && j > 0) s = s + rv.a[7][q];
     if (k % cd == cd - 1 && k + 1 < rv.ncz) s = s + rv.a[8][q] + rv.a[9][q];
     if (k % cd == 0 && k > 0) s = s + rv.a[10][q] + rv.a[11][q];
     out[q] = 0.125 * s;
