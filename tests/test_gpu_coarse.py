@@ -113,7 +113,7 @@ def test_coarse_kernel_options(sf, oracle, opts, monkeypatch):
 @pytest.mark.parametrize("n", [32, 64, 128])
 def test_coarse_kernel_solve(sf, oracle, n, monkeypatch):
     """Solve to 1e-10 (device loop): same cycle count and history as the
-    oracle, u within 1e-10."""
+    oracle (1e-6 relative plus the residual's rounding floor), u within 1e-10."""
     monkeypatch.setenv("SF_COARSE_KERNEL", "1")
     h = 1.0 / n
     coeffs = I.hpgmg_coeffs(n, n, n, h)
@@ -126,7 +126,10 @@ def test_coarse_kernel_solve(sf, oracle, n, monkeypatch):
     O = oracle.MG(n, n, n, h, 1.0, 1.0, *coeffs)
     u_o, hist_o = O.solve(f, fcycle=False, rtol=1e-10)
     assert cyc == len(hist_o)
-    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-14)
+    # atol: the max-norm residual's absolute rounding floor, ~1e-13 at 512^3
+    # scaled by h^-2 (R-19); the 128^3 level takes the
+    # delta-form restricted residual, which rounds differently from rhs - Ax
+    assert np.allclose(hist, hist_o, rtol=1e-6, atol=1e-12 * (n / 512) ** 2)
     assert rel(L.download(sf.SF_U), u_o) < 1e-10
     M.close()
     L.close()
