@@ -225,13 +225,17 @@ sf_status sf_smooth_gsrb(sf_level* level, int x, int rhs, double a, double b, in
 sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double b);
 /* A5 + A6 + A7, the tail of V(l)'s pre-smoothing: one RB
  * pair on fine.x (exactly sf_smooth_gsrb with rb_pairs = 1), then
- * coarse.c_field = R_cell(rhs - A x) of the smoothed x.  By default the pair,
- * then one residual + restriction pass (even nx: the residual is never stored;
- * odd nx: residual into SF_R, then the restriction).  With the environment
- * variable SF_RR=1 in a library built with SF_BUILD_RR=1, on single-part levels
- * with nx % 32 == 0, ny % 16 == 0 and x = SF_U, one kernel does all three in a
- * single HBM pass (the U/TMP ids are swapped as by the fused smoother); it is
- * measured slower on B200, hence opt-in.
+ * coarse.c_field = R_cell(rhs - A x) of the smoothed x.  On single-part fine and
+ * coarse levels with x = SF_U, nx % 32 == 0, ny % 8 == 0, even nz and at least
+ * SF_RRF_CELLS fine cells (default 2^21; SF_RRF=0 disables), the pair forms the
+ * restricted residual itself in delta form (gsrb_rr.cu, DESIGN.md section 6:
+ * a red cell's residual after the pair is b h^-2 sum_f beta_f delta of its
+ * black neighbours; equal to rhs - A x up to rounding, reading R-19) and a
+ * small fix-up pass writes coarse.c_field (the U/TMP ids are swapped as by the
+ * fused smoother); the fine level keeps partial arrays for that coarse shape,
+ * allocated (zeroed) on first use -- not inside a graph capture.  Otherwise the
+ * pair, then one residual + restriction pass (even nx: the residual is never
+ * stored; odd nx: residual into SF_R, then the restriction).
  * x must differ from rhs, SF_R and SF_DINV.  coarse dims must be fine dims / 2
  * (SF_ERR_SHAPE); c_field must not be SF_DINV.  Enqueued on the fine level's
  * stream; the coarse level must be idle on its own stream. */
