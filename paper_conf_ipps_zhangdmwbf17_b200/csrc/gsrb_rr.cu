@@ -47,8 +47,11 @@ constexpr int NPART = 12;
 // coarse rhs = 1/8 of the partials, summed in array order; the edge arrays are
 // read only where the current launch wrote them (tile-edge columns: the 32x8
 // build's coarse tiles are 16 wide; z-chunk edge planes: zdepth / 2 per chunk)
-__global__ void rrf_fixup_kernel(double* __restrict__ out, SfRRF rv) {
+__global__ void rrf_fixup_kernel(double* __restrict__ out, SfRRF rv, int trig) {
     pdl_wait();
+    // trig: the next launch (the coarse cluster V-cycle) may start now -- it
+    // stages its constant operands and waits for this output in griddepcontrol.wait
+    if (trig) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     const int i = blockIdx.x * blockDim.x + threadIdx.x, j = blockIdx.y, k = blockIdx.z;
     if (i >= rv.ncx) return;
     const long q = (long)(k + SF_GZ) * rv.cks + (long)(j + SF_GY) * rv.cjs + SF_OX + i;
@@ -106,7 +109,7 @@ sf_status sf_rrf_prepare(sf_level* F, const sf_level* C) {
 }
 
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
-                         int cf) {
+                         int cf, bool trigger_next) {
     if (!gsrb_rr_supported(L, C)) return sf_fail(SF_ERR_SHAPE, "fused pair+residual+restriction unsupported");
     SF_TRY(sf_rrf_prepare(L, C));
     SfRRF rv;
@@ -119,7 +122,8 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
     rv.zdepth = 2;
     SF_TRY(k_gsrb_pair_fused_t32w4(L, xin, xout, rhs, a, b, nullptr, nullptr, 0, 0, 0, SF_RM_NONE, &rv));
     PV c = sf_view(C, 0);
-    sf_launch(rrf_fixup_kernel, dim3((C->nx + 127) / 128, C->ny, C->lnz), 128, 0, L->stream, c.f[cf], rv);
+    sf_launch(rrf_fixup_kernel, dim3((C->nx + 127) / 128, C->ny, C->lnz), 128, 0, L->stream, c.f[cf], rv,
+              trigger_next ? 1 : 0);
     SF_LAUNCHED();
     return sf_check_launch("rrf_fixup");
 }

@@ -364,7 +364,10 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = fa
         // the last pre-smoothing pair also forms the residual and restricts it
         // (A5 + A6 + A7 in one pass; gsrb_rr.cu)
         SF_TRY(smooth(m, L, pre - 1));
-        SF_TRY(k_gsrb_pair_rr(L, SF_U, SF_TMP, SF_F, m->a, m->b, C, SF_F));
+        // the coarse cluster V-cycle follows directly: it may launch early
+        const bool next_coarse = m->coarse_l0 >= 1 && l + 1 == m->coarse_l0 &&
+                                 l + 1 < (int)m->lv.size() - 1;
+        SF_TRY(k_gsrb_pair_rr(L, SF_U, SF_TMP, SF_F, m->a, m->b, C, SF_F, next_coarse));
         sf_swap_fields(L, SF_U, SF_TMP);
     } else {
         SF_TRY(smooth(m, L, pre));

@@ -256,7 +256,7 @@ sf_status k_gsrb_twopair(sf_level* L, int xin, int xout, int rhs, double a, doub
 // xout = pair(xin); C.cf = R_cell(rhs - A xout).  Single-part levels, 32x16 tiles.
 bool gsrb_rr_supported(const sf_level* F, const sf_level* C);
 sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, double b, sf_level* C,
-                         int cf);
+                         int cf, bool trigger_next = false);
 // allocate the fine level's RRF partial arrays for coarse level C (before any capture)
 sf_status sf_rrf_prepare(sf_level* F, const sf_level* C);
 
