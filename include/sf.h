@@ -233,7 +233,8 @@ sf_status sf_residual(sf_level* level, int res, int x, int rhs, double a, double
  * black neighbours; equal to rhs - A x up to rounding, reading R-19) and a
  * small fix-up pass writes coarse.c_field (the U/TMP ids are swapped as by the
  * fused smoother); the fine level keeps partial arrays for that coarse shape,
- * allocated (zeroed) on first use -- not inside a graph capture.  Otherwise the
+ * allocated (zeroed) on first use (sf_mg_create allocates its levels'; a call
+ * inside a graph capture without them takes the composite path).  Otherwise the
  * pair, then one residual + restriction pass (even nx: the residual is never
  * stored; odd nx: residual into SF_R, then the restriction).
  * x must differ from rhs, SF_R and SF_DINV.  coarse dims must be fine dims / 2

@@ -85,6 +85,13 @@ bool gsrb_rr_supported(const sf_level* F, const sf_level* C) {
            (long)F->nx * F->ny * F->lnz >= rrf_min_cells();
 }
 
+// the partial arrays exist, or can be allocated now (the stream is not capturing)
+bool sf_rrf_usable(const sf_level* F, const sf_level* C) {
+    if (F->rrf_buf && F->rrf_felems == C->felems) return true;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    return cudaStreamIsCapturing(F->stream, &cs) == cudaSuccess && cs == cudaStreamCaptureStatusNone;
+}
+
 // allocate (once, zeroed) the partial arrays of F for coarse level C
 sf_status sf_rrf_prepare(sf_level* F, const sf_level* C) {
     if (F->rrf_buf && F->rrf_felems == C->felems) return SF_OK;

@@ -394,7 +394,10 @@ extern "C" sf_status sf_smooth_residual_restrict(sf_level* F, int x, int rhs, do
     if (x == rhs || x == SF_DINV || rhs == SF_DINV || x == SF_R || rhs == SF_R || cf == SF_DINV)
         return sf_fail(SF_ERR_INVALID, "x, rhs, R and DINV must be distinct fields");
     if (!coarse_of(C, F)) return sf_fail(SF_ERR_SHAPE, "coarse dims must be fine dims / 2");
-    if (x == SF_U && rhs != SF_TMP && gsrb_fused_supported(F) && gsrb_rr_supported(F, C)) {
+    // (inside a graph capture the fused path needs its partial arrays from an
+    // earlier eager call or sf_mg_create; otherwise the composite path runs)
+    if (x == SF_U && rhs != SF_TMP && gsrb_fused_supported(F) && gsrb_rr_supported(F, C) &&
+        sf_rrf_usable(F, C)) {
         const int other = (x == SF_U) ? SF_TMP : SF_U;
         SF_TRY(sf_halo(F, rhs, 1));
         SF_TRY(sf_halo(F, x, 2));

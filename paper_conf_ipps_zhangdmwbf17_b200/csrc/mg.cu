@@ -360,7 +360,7 @@ static sf_status vcyc(sf_mg* m, int l, bool skip_first = false, bool u_zero = fa
     sf_level* C = m->lv[l + 1];
     const int pre = m->o.pre_pairs - (skip_first ? 1 : 0);
     if (pre >= 1 && (m->o.smoother == SF_SMOOTH_AUTO || m->o.smoother == SF_SMOOTH_FUSED) &&
-        gsrb_fused_supported(L) && gsrb_rr_supported(L, C)) {
+        gsrb_fused_supported(L) && gsrb_rr_supported(L, C) && sf_rrf_usable(L, C)) {
         // the last pre-smoothing pair also forms the residual and restricts it
         // (A5 + A6 + A7 in one pass; gsrb_rr.cu)
         SF_TRY(smooth(m, L, pre - 1));

@@ -259,6 +259,7 @@ sf_status k_gsrb_pair_rr(sf_level* L, int xin, int xout, int rhs, double a, doub
                          int cf, bool trigger_next = false);
 // allocate the fine level's RRF partial arrays for coarse level C (before any capture)
 sf_status sf_rrf_prepare(sf_level* F, const sf_level* C);
+bool sf_rrf_usable(const sf_level* F, const sf_level* C);
 
 // coarse-level V-cycle in one thread-block-cluster launch, iterates in registers and
 // shared memory (coarse.cu)
